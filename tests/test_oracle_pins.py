@@ -1,0 +1,405 @@
+"""Pins of the CPU oracle against things other than itself (-m "not gpu").
+
+Each test names the PAPER.md passage ("P:n") or the textbook result it pins.
+A plausible mistake anywhere in the oracle (dropped billing term, wrong sign,
+wrong predecessor, swapped case, wrong digit order, FMA in the cost) fails at
+least one of them.
+"""
+import glob
+import itertools
+import json
+import os
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+import workloads as W
+from oracle import OracleProblem, des
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def mk(preds, exec_us, init_us, arrivals, windows, sla=10**9, prices=None, n_configs=None):
+    ptr, idx = W.csr_from_preds(preds)
+    n = len(preds)
+    ncfg = np.ones(n, np.int32) if n_configs is None else np.asarray(n_configs, np.int32)
+    tot = int(ncfg.sum())
+    pr = np.ones(tot) if prices is None else np.asarray(prices, np.float64)
+    return W.Problem("t", ptr, idx, ncfg, np.asarray(exec_us, np.int32), np.asarray(init_us, np.int32),
+                     pr, np.asarray(arrivals, np.int64), int(sla), np.asarray(windows, np.int32))
+
+
+# ---------------------------------------------------------------------------
+# Worked examples (tests/golden, each with its citation and hand derivation)
+# ---------------------------------------------------------------------------
+
+@pytest.mark.parametrize("path", sorted(glob.glob(os.path.join(GOLDEN, "E*.json"))))
+def test_golden_worked_examples(path):
+    g = json.load(open(path))
+    assert g["citation"]
+    for case in g["cases"]:
+        p = mk(g["preds"], g["exec_us"], g["init_us"], g["arrivals_us"], case["windows_us"])
+        o = OracleProblem(p)
+        cfg = [0] * p.n_funcs
+        billed, lat = o.simulate(cfg, case["window_idx"])
+        assert billed.tolist() == case["billed"], (path, case)
+        assert lat.tolist() == case["latency"], (path, case)
+
+
+# ---------------------------------------------------------------------------
+# Closed forms from the paper
+# ---------------------------------------------------------------------------
+
+def test_eq5_case_I_chain_closed_form():
+    """P:177-179 Eq. (5): with periodic arrivals and T_k + I_k < IT, the window
+    IT - T_k - I_k hides every init: L = sum of I, C_k = (T_k + I_k) U per invocation."""
+    rng = np.random.default_rng(11)
+    for _ in range(200):
+        n = int(rng.integers(1, 7))
+        J = int(rng.integers(1, 30))
+        IT = int(rng.integers(10_000, 100_000))
+        I = rng.integers(0, IT // 3, size=n)
+        T = rng.integers(0, IT // 3, size=n)
+        windows = sorted(set(int(IT - T[k] - I[k]) for k in range(n)))
+        r = np.arange(J, dtype=np.int64) * IT + int(rng.integers(0, 10**6))
+        p = mk([[]] + [[k - 1] for k in range(1, n)], I, T, r, windows)
+        widx = [windows.index(int(IT - T[k] - I[k])) for k in range(n)]
+        billed, lat = OracleProblem(p).simulate([0] * n, widx)
+        assert (lat == int(I.sum())).all()
+        assert billed.tolist() == [J * int(T[k] + I[k]) for k in range(n)]
+
+
+def test_case_II_keepalive_closed_form():
+    """keep-alive (window 0) costs IT * U per invocation after the
+    first (T + I); latency as Eq. (5)."""
+    rng = np.random.default_rng(12)
+    for _ in range(200):
+        n = int(rng.integers(1, 6))
+        J = int(rng.integers(1, 30))
+        IT = int(rng.integers(1000, 100_000))
+        I = rng.integers(0, IT // n + 1, size=n)    # sum I <= IT: never busy
+        I = np.minimum(I, IT // n)
+        T = rng.integers(0, 10 * IT, size=n)
+        r = np.arange(J, dtype=np.int64) * IT
+        p = mk([[]] + [[k - 1] for k in range(1, n)], I, T, r, [0])
+        billed, lat = OracleProblem(p).simulate([0] * n, [0] * n)
+        assert (lat == int(I.sum())).all()
+        assert billed.tolist() == [int(T[k] + I[k]) + (J - 1) * IT for k in range(n)]
+
+
+def test_theorem_5_1_window_minimises_cost():
+    """P:184 Theorem 5.1: when I1 + I2 < SLA and T2 + I2 < IT, the Case-I window
+    gives the minimum cost.  Over a dense window grid the lowest-index window of
+    minimum F2 cost that also meets SLA = I1 + I2 is exactly IT - T2 - I2."""
+    rng = np.random.default_rng(13)
+    for _ in range(40):
+        IT = int(rng.integers(2000, 20000))
+        I1, I2 = (int(v) for v in rng.integers(1, IT // 4, size=2))
+        T1, T2 = (int(v) for v in rng.integers(1, IT // 4, size=2))
+        wstar = IT - T2 - I2
+        grid = sorted(set([0, wstar] + [int(v) for v in rng.integers(1, 2 * IT, size=20)]))
+        r = np.arange(12, dtype=np.int64) * IT
+        p = mk([[], [0]], [I1, I2], [T1, T2], r, grid, sla=I1 + I2)
+        o = OracleProblem(p)
+        best = None
+        for wi in range(len(grid)):
+            billed, lat = o.simulate([0, 0], [0, wi])
+            if lat.max() <= I1 + I2 and (best is None or billed[1] < best[1]):
+                best = (wi, billed[1])
+        assert grid[best[0]] == wstar
+        assert best[1] == 12 * (T2 + I2)
+
+
+# ---------------------------------------------------------------------------
+# Textbook reductions
+# ---------------------------------------------------------------------------
+
+def test_case_III_lindley_single_server():
+    """P:198 Fig. 5(c): a kept-alive function serves FIFO; waiting times follow
+    Lindley's recursion W_j = max(0, W_{j-1} + I - (r_j - r_{j-1}))."""
+    rng = np.random.default_rng(14)
+    for _ in range(300):
+        J = int(rng.integers(1, 60))
+        I = int(rng.integers(0, 5000))
+        T = int(rng.integers(0, 5000))
+        r = np.cumsum(rng.integers(0, 2 * I + 2, size=J)).astype(np.int64)
+        p = mk([[]], [I], [T], r, [0])
+        billed, lat = OracleProblem(p).simulate([0], [0])
+        w = 0
+        exp = []
+        for j in range(J):
+            if j:
+                w = max(0, w + I - int(r[j] - r[j - 1]))
+            exp.append(w + I)
+        assert lat.tolist() == exp
+        # keep-alive: loaded from x_0 - T to the last completion
+        assert int(billed[0]) == T + (int(r[-1]) + exp[-1]) - int(r[0])
+
+
+def test_keepalive_tandem_queue_recursion():
+    """Chain with keep-alive everywhere is a tandem of FIFO single servers:
+    D_j^k = max(D_j^{k-1}, D_{j-1}^k) + I_k (max-plus recursion)."""
+    rng = np.random.default_rng(15)
+    for _ in range(200):
+        n = int(rng.integers(1, 6))
+        J = int(rng.integers(1, 40))
+        I = rng.integers(0, 3000, size=n)
+        T = rng.integers(0, 3000, size=n)
+        r = np.cumsum(rng.integers(0, 4000, size=J)).astype(np.int64)
+        p = mk([[]] + [[k - 1] for k in range(1, n)], I, T, r, [0])
+        billed, lat = OracleProblem(p).simulate([0] * n, [0] * n)
+        D = np.zeros((n, J), np.int64)
+        for j in range(J):
+            for k in range(n):
+                up = r[j] if k == 0 else D[k - 1, j]
+                prev = D[k, j - 1] if j else up
+                D[k, j] = max(up, prev) + I[k]
+        assert lat.tolist() == (D[n - 1] - r).tolist()
+        first_start = [int(r[0])] + [int(D[k - 1, 0]) for k in range(1, n)]
+        assert billed.tolist() == [int(T[k] + D[k, -1] - first_start[k]) for k in range(n)]
+
+
+def _all_paths_longest(preds, I):
+    """Brute-force longest I-weighted source->sink path by enumerating paths."""
+    n = len(preds)
+    succ = [[] for _ in range(n)]
+    for k, ps in enumerate(preds):
+        for q in ps:
+            succ[q].append(k)
+    best = 0
+
+    def walk(k, acc):
+        nonlocal best
+        acc += int(I[k])
+        if not succ[k]:
+            best = max(best, acc)
+        for s in succ[k]:
+            walk(s, acc)
+
+    for k in range(n):
+        if not preds[k]:
+            walk(k, 0)
+    return best
+
+
+def test_dag_latency_is_longest_path_when_sparse():
+    """'sum along sequential stages, max over parallel branches':
+    with warm (keep-alive) functions and gaps larger than every path, each
+    request's latency is the longest I-weighted path of the DAG."""
+    rng = np.random.default_rng(16)
+    for _ in range(200):
+        n = int(rng.integers(1, 8))
+        p0 = W.random_problem(rng, n, 1, 1, int(rng.integers(1, 8)))
+        preds = [p0.preds(k) for k in range(n)]
+        I = rng.integers(0, 1000, size=n)
+        r = np.cumsum(rng.integers(int(I.sum()) + 1, int(I.sum()) + 5000, size=p0.arrivals_us.shape[0]))
+        p = mk(preds, I, rng.integers(0, 10**6, size=n), r.astype(np.int64), [0])
+        billed, lat = OracleProblem(p).simulate([0] * n, [0] * n)
+        assert (lat == _all_paths_longest(preds, I)).all()
+
+
+def test_mixed_radix_decode_matches_numpy():
+    """Index order: function 0 most significant, config-major digit
+    d_k = c_k * W + w_k; checked against numpy.unravel_index (C order)."""
+    rng = np.random.default_rng(17)
+    for _ in range(50):
+        n = int(rng.integers(1, 6))
+        p = W.random_problem(rng, n, 4, int(rng.integers(1, 4)), 2)
+        o = OracleProblem(p)
+        Wn = len(p.windows_us)
+        shape = tuple(int(p.n_configs[k]) * Wn for k in range(n))
+        assert o.space_size() == int(np.prod(shape))
+        for idx in rng.integers(0, o.space_size(), size=20):
+            c, w = o.decode(int(idx))
+            digits = np.unravel_index(int(idx), shape)
+            assert [int(d) // Wn for d in digits] == c.tolist()
+            assert [int(d) % Wn for d in digits] == w.tolist()
+
+
+def test_n_fixed_prefix_pins_leading_digits():
+    rng = np.random.default_rng(18)
+    p = W.random_problem(rng, 4, 3, 2, 5)
+    Wn = len(p.windows_us)
+    full = OracleProblem(p)
+    fixed = [int(rng.integers(0, p.n_configs[0] * Wn))]
+    sub = OracleProblem(p, n_fixed=1, fixed_digits=fixed)
+    S = sub.space_size()
+    assert full.space_size() == S * int(p.n_configs[0]) * Wn
+    for i in range(S):
+        assert np.array_equal(sub.evaluate([i])[0], full.evaluate([fixed[0] * S + i])[0])
+
+
+# ---------------------------------------------------------------------------
+# Independent implementation: the event-driven simulator (oracle/des.py)
+# ---------------------------------------------------------------------------
+
+def test_oracle_matches_event_driven_simulator():
+    """G3/G4/G5/G6/G7 are not fixed by the paper; two independent
+    implementations of the stated rule (case split vs explicit instance state
+    machine with loaded-time integration) must agree exactly."""
+    rng = np.random.default_rng(19)
+    for _ in range(3000):
+        n = int(rng.integers(1, 7))
+        p = W.random_problem(rng, n, 3, int(rng.integers(1, 5)), int(rng.integers(1, 13)))
+        o = OracleProblem(p)
+        c = [int(rng.integers(0, p.n_configs[k])) for k in range(n)]
+        w = [int(rng.integers(0, len(p.windows_us))) for k in range(n)]
+        billed, lat = o.simulate(c, w)
+        b2, l2 = des.simulate(p, c, w)
+        assert billed.tolist() == b2
+        assert lat.tolist() == l2
+
+
+def _des_cost(p, c, w):
+    billed, lat = des.simulate(p, c, w)
+    off = np.concatenate([[0], np.cumsum(p.n_configs)])
+    cost = 0.0
+    for k in range(p.n_funcs):
+        cost = cost + float(p.price_per_us[off[k] + c[k]]) * float(billed[k])
+    return cost, max(lat)
+
+
+def test_plan_equals_brute_force_through_des():
+    """OPT by brute force through the independent DES (P:305 'exhaustive
+    search'): lowest index among minimum-cost SLA-feasible candidates."""
+    rng = np.random.default_rng(20)
+    checked = 0
+    for _ in range(60):
+        n = int(rng.integers(1, 4))
+        p = W.random_problem(rng, n, 3, int(rng.integers(1, 4)), int(rng.integers(1, 8)))
+        o = OracleProblem(p)
+        S = o.space_size()
+        if S > 600:
+            continue
+        best = None
+        for i in range(S):
+            c, w = o.decode(i)
+            cost, ml = _des_cost(p, c.tolist(), w.tolist())
+            if ml <= p.sla_us and (best is None or cost < best[1]):
+                best = (i, cost, ml)
+        got = o.plan(n_threads=3)
+        assert got == best
+        checked += 1
+    assert checked > 20
+
+
+def test_cost_is_exact_sum_for_dyadic_prices():
+    """Eq. (3)/(4): cost = sum_k U_k * billed_k.  With dyadic prices every
+    product and partial sum is exact, so the oracle's cost equals the exact
+    rational sum (pins: no dropped/duplicated term, right price row)."""
+    rng = np.random.default_rng(21)
+    for _ in range(300):
+        n = int(rng.integers(1, 7))
+        p = W.random_problem(rng, n, 4, 2, int(rng.integers(1, 10)))
+        o = OracleProblem(p)
+        i = int(rng.integers(0, o.space_size()))
+        c, w = o.decode(i)
+        billed, _ = o.simulate(c, w)
+        off = np.concatenate([[0], np.cumsum(p.n_configs)])
+        exact = sum(Fraction(float(p.price_per_us[off[k] + c[k]])) * int(billed[k]) for k in range(n))
+        cost, _, _ = o.evaluate([i])
+        assert Fraction(float(cost[0])) == exact
+
+
+def test_plan_thread_count_invariant():
+    p = W.make_config("C1")
+    a = OracleProblem(p).plan(n_threads=1)
+    b = OracleProblem(p).plan(n_threads=7)
+    assert a == b and a is not None
+
+
+# ---------------------------------------------------------------------------
+# Invariants
+# ---------------------------------------------------------------------------
+
+def test_sla_nesting_and_monotone_opt():
+    """Eq. (4) constraint L <= SLA: the feasible set shrinks as the SLA
+    tightens and the optimal cost is non-increasing in the SLA."""
+    p = W.make_config("C1", n_arrivals=40)
+    o = OracleProblem(p)
+    idx = np.arange(o.space_size())
+    cost, lat, _ = o.evaluate(idx)
+    prev_set, prev_opt = None, None
+    for sla in [400_000, 800_000, 1_200_000, 1_600_000, 2_000_000, 3_000_000, 10**9]:
+        feas = set(np.nonzero(lat <= sla)[0].tolist())
+        if prev_set is not None:
+            assert prev_set <= feas
+        got = OracleProblem(p, sla_us=sla).plan()
+        opt = None if got is None else got[1]
+        if prev_opt is not None:
+            assert opt is not None and opt <= prev_opt
+        prev_set, prev_opt = feas, opt
+
+
+def test_price_power_of_two_scaling():
+    """Scaling every U by 2 scales every cost exactly by 2 and keeps the argmin."""
+    p = W.make_config("C1", n_arrivals=30)
+    a = OracleProblem(p).plan()
+    b = OracleProblem(p.replace(price_per_us=p.price_per_us * 2.0)).plan()
+    assert a[0] == b[0] and b[1] == 2.0 * a[1] and a[2] == b[2]
+
+
+def test_integer_time_scaling():
+    """Scaling all times (I, T, windows, arrivals) by k scales latencies and
+    billed times by k (the model is homogeneous of degree 1 in time)."""
+    rng = np.random.default_rng(22)
+    for _ in range(100):
+        n = int(rng.integers(1, 6))
+        p = W.random_problem(rng, n, 2, 3, int(rng.integers(1, 9)))
+        k = int(rng.integers(2, 6))
+        q = p.replace(exec_us=p.exec_us * k, init_us=p.init_us * k, windows_us=p.windows_us * k,
+                      arrivals_us=p.arrivals_us * k, sla_us=p.sla_us * k)
+        c = [int(rng.integers(0, p.n_configs[i])) for i in range(n)]
+        w = [int(rng.integers(0, len(p.windows_us))) for i in range(n)]
+        b1, l1 = OracleProblem(p).simulate(c, w)
+        b2, l2 = OracleProblem(q).simulate(c, w)
+        assert (b2 == k * b1).all() and (l2 == k * l1).all()
+
+
+def test_keepalive_is_latency_lower_bound():
+    """Keep-alive (all windows 0) never loads a cold instance, so every done
+    time -- hence every latency -- is a lower bound for any window choice
+    (basis of the exact keep-alive pre-pass prune)."""
+    rng = np.random.default_rng(23)
+    for _ in range(1000):
+        n = int(rng.integers(1, 7))
+        p = W.random_problem(rng, n, 2, 4, int(rng.integers(1, 12)))
+        if p.windows_us[0] != 0:
+            p = p.replace(windows_us=np.concatenate([[0], p.windows_us]).astype(np.int32))
+        o = OracleProblem(p)
+        c = [int(rng.integers(0, p.n_configs[i])) for i in range(n)]
+        w = [int(rng.integers(0, len(p.windows_us))) for i in range(n)]
+        _, l_any = o.simulate(c, w)
+        _, l_ka = o.simulate(c, [0] * n)
+        assert (l_ka <= l_any).all()
+
+
+def test_cost_monotone_in_keepalive_when_never_busy():
+    """North star invariant 'cost is monotone in keep-alive', in the form that
+    holds under the model (G20): for a function whose every gap
+    exceeds I + T, its billed time is non-increasing and its latency
+    non-decreasing as the window grows, and keep-alive (window 0) bills the most."""
+    rng = np.random.default_rng(24)
+    for _ in range(300):
+        I = int(rng.integers(0, 2000))
+        T = int(rng.integers(0, 2000))
+        J = int(rng.integers(2, 20))
+        r = np.cumsum(rng.integers(I + T + 1, 20000, size=J)).astype(np.int64)
+        grid = sorted(set([0] + rng.integers(1, 30000, size=12).tolist()))
+        p = mk([[]], [I], [T], r, grid)
+        o = OracleProblem(p)
+        res = [o.simulate([0], [wi]) for wi in range(len(grid))]
+        billed = [int(b[0]) for b, _ in res]
+        lat = [int(l.max()) for _, l in res]
+        assert all(billed[i] >= billed[i + 1] for i in range(len(grid) - 1))
+        assert all(lat[i] <= lat[i + 1] for i in range(1, len(grid) - 1))
+        assert billed[0] == max(billed)
+
+
+def test_oracle_rejects_bad_args():
+    p = mk([[]], [1], [1], [0], [0])
+    o = OracleProblem(p)
+    o.s.n_arrivals = 0
+    with pytest.raises(ValueError):
+        o.evaluate([0])
