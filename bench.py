@@ -1,0 +1,361 @@
+#!/usr/bin/env python
+"""bench.py -- candidate plans evaluated/s (and time-to-optimal) of the SMIless hot path on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2] [--impl ours|reference]
+    python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 bench.py --gpus N ...
+
+Step (BASELINE.json metric, configs[1]): one smiless_plan call = the whole hot path
+(arrival prep, NVRTC-specialised evaluator over every candidate, argmin, exact
+re-evaluation of the winner) over the fixed 2^28-candidate slice of C2 (IPA-6 DAG,
+16 configs x 8 windows, 10^4 Poisson arrivals; functions 0 and 1 pinned to
+GPU-100% / keep-alive), in throughput mode (no pruning: every candidate walked through
+all 10^4 arrivals).  N GPUs split that fixed slice (strong scaling: time-to-optimal
+of the slice); each rank plans its interleaved chunks and the ranks exchange the
+winner with NCCL MIN all-reduces.
+
+`value` = candidates of the slice / max-over-ranks device time per step (inputs resident
+in HBM: arrivals passed as a device tensor).  `e2e` = the same through the public API
+with the arrivals in pinned host memory (H2D inside the timed region) and the result
+read back to the host.  Only rank 0 at N=1 times the CPU oracle (cpu_baseline) on a
+bounded sample; `--impl reference` times the oracle as the reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+METRIC = "candidate plans evaluated/sec and time-to-optimal-plan at 1/2/4/8 B200"
+UNIT = "candidates/s"
+ISSUE_LANES_PER_CLK_PER_SM = 4 * 32      # 4 SMSPs x 1 warp-instruction/clk x 32 lanes
+
+
+def workload(name: str = "C2"):
+    """(Problem, plan kwargs) of the timed step.  Shared with tests/test_gpu_parity.py."""
+    if name == "C2":
+        p = W.make_config("C2")
+        Wn = len(p.windows_us)
+        gpu100 = 15                        # CONFIG_GRIDS[16][15] = ("gpu", 1.0)
+        fixed = [gpu100 * Wn + 0, gpu100 * Wn + 0]   # SR, IR on GPU-100%, keep-alive
+        return p, dict(n_fixed=2, fixed_digits=fixed)
+    if name == "C1":
+        return W.make_config("C1"), dict(n_fixed=0, fixed_digits=[])
+    raise KeyError(name)
+
+
+def algorithmic_ops_per_unit(p, n_fixed: int) -> int:
+    """Integer ops one lane-unit (one upstream prefix x all W windows of the last
+    function) needs per the model: per invocation j >= 1, 6 ops
+    per upstream function-step (g, u, busy, delta, select, F), +1 per extra join input,
+    +1 per upstream sink latency check, 7 per last-function window variant (6 + the
+    latency max), +1 shared offset negation."""
+    n = p.n_funcs
+    Wn = len(p.windows_us)
+    joins = sum(max(0, len(p.preds(k)) - 1) for k in range(n))
+    listed = set(int(v) for v in p.pred_idx)
+    up_sinks = sum(1 for k in range(n - 1) if k not in listed)
+    per_step = 6 * (n - 1) + joins + up_sinks + 7 * Wn + 1
+    return per_step * (len(p.arrivals_us) - 1)
+
+
+class ClockSampler:
+    """nvidia-smi-equivalent clocks/throttle sampling (NVML) during the timed region."""
+
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+        0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+        0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
+    }
+
+    def __init__(self, device_index: int, period_s: float = 0.2):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        self._thr = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self._nv = pynvml
+            self._h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self._h, pynvml.NVML_CLOCK_SM)
+        except Exception as e:  # pragma: no cover
+            self._nv = None
+            self.error = str(e)
+        self.period = period_s
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self._nv.nvmlDeviceGetClockInfo(self._h, self._nv.NVML_CLOCK_SM))
+                r = self._nv.nvmlDeviceGetCurrentClocksEventReasons(self._h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and bit != 0x1:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            self._stop.wait(self.period)
+
+    def __enter__(self):
+        if self._nv is not None:
+            self._thr = threading.Thread(target=self._run, daemon=True)
+            self._thr.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._thr:
+            self._thr.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                    "samples": 0}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def measured_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+def ncu_traffic():
+    """DRAM bytes per launch of the evaluator from the committed ncu --set full summary."""
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "ncu_evaluator_summary.json")))
+        return d.get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+def cpu_oracle_rate(p, kw, seconds: float = 15.0, threads=None):
+    """Oracle (as it stands) on the host cores: candidates/s over a bounded sample of the
+    same slice (its first candidates, sized to ~`seconds` of CPU work)."""
+    from oracle import OracleProblem
+    threads = threads or os.cpu_count() or 1
+    o = OracleProblem(p, n_fixed=kw["n_fixed"], fixed_digits=kw["fixed_digits"])
+    n = max(threads, 8)
+    t0 = time.perf_counter()
+    o.plan(0, n, n_threads=threads)
+    dt = time.perf_counter() - t0
+    n2 = max(threads, int(n * seconds / max(dt, 1e-6)))
+    t0 = time.perf_counter()
+    o.plan(0, n2, n_threads=threads)
+    dt = time.perf_counter() - t0
+    return n2 / dt, n2, dt, threads
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as the reference arm (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    p, kw = workload(args.workload)
+    from oracle import OracleProblem
+    threads = os.cpu_count() or 1
+    o = OracleProblem(p, n_fixed=kw["n_fixed"], fixed_digits=kw["fixed_digits"])
+    # size one step to ~8 s of host work
+    probe = max(threads, 8)
+    t0 = time.perf_counter()
+    o.plan(0, probe, n_threads=threads)
+    per = (time.perf_counter() - t0) / probe
+    n_step = max(threads, int(8.0 / max(per, 1e-9)))
+    for _ in range(args.warmup):
+        o.plan(0, min(n_step, threads * 2), n_threads=threads)
+    t0 = time.perf_counter()
+    for s in range(args.steps):
+        o.plan(s * n_step, (s + 1) * n_step, n_threads=threads)
+    dt = time.perf_counter() - t0
+    value = args.steps * n_step / dt
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "i64+f64",
+        "data": "synthetic", "config": config_block(p, kw, args),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
+                         "sample": f"{n_step} consecutive candidates of the slice per step"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def config_block(p, kw, args):
+    space = 1
+    for k in range(kw["n_fixed"], p.n_funcs):
+        space *= int(p.n_configs[k]) * len(p.windows_us)
+    return {
+        "workload": f"{p.name}: {p.n_funcs}-function DAG, {int(p.n_configs[0])} configs x {len(p.windows_us)} "
+                    f"windows, J={len(p.arrivals_us)} arrivals, SLA {p.sla_us} us; slice of {space} candidates "
+                    f"(functions 0..{kw['n_fixed'] - 1} pinned to digits {list(kw['fixed_digits'])}); "
+                    f"throughput mode (no pruning)",
+        "candidates_per_step": space,
+        "arrivals": len(p.arrivals_us),
+        "l2": "256 MiB buffer written between timed steps (L2 flushed); working set < 1 MB",
+        "parallelism": f"candidate-space sharding x{args.gpus}",
+    }
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default="C2")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-pruned", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_luxl0y024_b200 import smiless as S
+    from paper_conf_sc_luxl0y024_b200.dist import reduce_best
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    p, kw = workload(args.workload)
+    stream = torch.cuda.current_stream(dev)
+    pl = S.planner_for(p, device=local, stream=stream.cuda_stream)
+    arr_dev = torch.as_tensor(p.arrivals_us).to(dev)                 # HBM-resident inputs
+    arr_pin = torch.as_tensor(p.arrivals_us).pin_memory()            # e2e: pinned host inputs
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    plan_kw = dict(kw, flags=S.FLAG_NO_PRUNE, shard=rank, n_shards=world)
+
+    def step(arrivals):
+        r = pl.plan(arrivals, p.sla_us, p.windows_us, **plan_kw)
+        if world > 1:
+            reduce_best(r.cost if r.feasible else None, r.index, r.max_latency_us, r.n_decided, dev)
+        return r
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+
+    for _ in range(args.warmup):
+        r = step(arr_dev)
+    barrier()
+
+    def timed(arrivals, n):
+        evs = []
+        res = None
+        launches = 0
+        kernel_ms = 0.0
+        for _ in range(n):
+            flush.fill_(1)                                           # L2 flush, outside the events
+            a = torch.cuda.Event(enable_timing=True)
+            b = torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            res = step(arrivals)
+            b.record(stream)
+            evs.append((a, b))
+            launches += res.launches
+            kernel_ms += res.eval_kernel_ms
+        torch.cuda.synchronize(dev)
+        ms = sum(a.elapsed_time(b) for a, b in evs)
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item()), res, launches, kernel_ms
+
+    barrier()
+    with ClockSampler(local) as clk:
+        ms, res, launches, kernel_ms = timed(arr_dev, args.steps)
+    barrier()
+    barrier()
+    ms_e2e, res_e2e, _, _ = timed(arr_pin, max(1, min(args.steps, 3)))
+    barrier()
+
+    cands = int(res.n_decided)
+    if world > 1:
+        t = torch.tensor([cands], dtype=torch.int64, device=dev)
+        dist.all_reduce(t)
+        cands = int(t.item())
+    steps_e2e = max(1, min(args.steps, 3))
+    value = cands * args.steps / (ms / 1e3)
+    e2e_value = cands * steps_e2e / (ms_e2e / 1e3)
+
+    # pruned (exact plan with early exit): time-to-optimal of the same slice
+    pruned = None
+    if not args.no_pruned:
+        kwp = dict(kw, flags=0, shard=rank, n_shards=world)
+        barrier()
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        rp = pl.plan(arr_dev, p.sla_us, p.windows_us, **kwp)
+        if world > 1:
+            reduce_best(rp.cost if rp.feasible else None, rp.index, rp.max_latency_us, rp.n_decided, dev)
+        b.record(stream)
+        torch.cuda.synchronize(dev)
+        pruned = {"time_to_optimal_ms": a.elapsed_time(b), "index": rp.index, "cost": rp.cost,
+                  "max_latency_us": rp.max_latency_us, "full_evals_fraction": rp.n_full_evals / max(1, rp.n_decided)}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return 0
+
+    peaks = measured_peaks()
+    props = torch.cuda.get_device_properties(dev)
+    clocks = clk.summary()
+    sm_mhz = clocks["sm_mhz"] or peaks.get("sm_max_mhz", 1965.0)
+    peak_ops = props.multi_processor_count * ISSUE_LANES_PER_CLK_PER_SM * float(clocks["sm_max_mhz"] or 1965.0) * 1e6
+    units_per_launch = res.n_decided / len(p.windows_us)
+    ops = algorithmic_ops_per_unit(p, kw["n_fixed"]) * units_per_launch
+    kernel_ms_per_step = kernel_ms / args.steps
+    achieved = ops / (kernel_ms_per_step / 1e3)
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "i32+f64", "data": "synthetic",
+        "config": config_block(p, kw, args),
+        "time_to_optimal_ms": ms / args.steps,
+        "winner": {"index": res.index, "cost": res.cost, "max_latency_us": res.max_latency_us,
+                   "config": res.config.tolist(), "window": res.window.tolist()} if world == 1 else None,
+        "pruned": pruned,
+        "gpu_launches": launches,
+        "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(p.arrivals_us.nbytes),
+                "d2h_bytes_per_step": 312},
+        "clocks": clocks,
+        "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_ops, "unit": "int-ops/s",
+                     "frac": achieved / peak_ops, "traffic": ncu_traffic(),
+                     "kernel": "smiless_plan_kernel", "kernel_ms_per_launch": kernel_ms_per_step,
+                     "ops_per_unit": algorithmic_ops_per_unit(p, kw["n_fixed"]),
+                     "peak_basis": "issue peak: SMs x 4 SMSP x 32 lanes x sm_max_mhz (DESIGN.md Roofline)"},
+        "kernel_share_of_step": kernel_ms_per_step / (ms / args.steps),
+    }
+    if world == 1 and not args.no_cpu_baseline:
+        rate, n, dt, threads = cpu_oracle_rate(p, kw)
+        line["cpu_baseline"] = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle",
+                                "sample": f"first {n} candidates of the slice ({dt:.1f} s, J={len(p.arrivals_us)})"}
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

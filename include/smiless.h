@@ -1,0 +1,190 @@
+/*
+ * smiless.h -- C ABI of the B200-native SMIless co-optimisation hot path.
+ *
+ * The operation (PAPER.md line citations, "P:n"):
+ *
+ *   Given an application DAG of N serverless inference functions,
+ *   per-function x per-configuration profiles -- inference time I, init time T
+ *   (T = mu + 3 sigma) and unit price U (Eq. (3)) --,
+ *   a cold-start policy set S = a grid of pre-warming windows (window 0
+ *   = keep alive), a predicted invocation-arrival sequence
+ *   and an SLA on end-to-end latency (Eq. (4), default 2 s P:283),
+ *   return the exhaustive optimum ("OPT ... determined through
+ *   exhaustive search") of
+ *
+ *       min_{chi, phi}  sum_k C_k(*_k, /\_k) = sum_k E_k * U(*_k)   (Eq. 3, 4)
+ *       s.t.            L(chi, phi) <= SLA      for every request
+ *
+ *   where each candidate (config *_k and window /\_k for every function) is
+ *   simulated over the whole arrival sequence with model M (DESIGN.md "Model
+ *   M": the Case I / II / III rules of P:169-200 applied per invocation; the
+ *   E2E latency is "sum along sequential stages, max over parallel branches"
+ *   with FIFO waiting and cold-start penalties; E_k = init + inference +
+ *   loaded-idle time).  Ties on cost go to the LOWEST candidate index.
+ *
+ * Units: all times are integer microseconds, prices are double per
+ * microsecond.  Candidate index order (mixed radix): function n_fixed is the
+ * most significant digit, function N-1 the least; digit d_k = c_k * W + w_k
+ * (config major, window minor); radix of function k is M_k * W.
+ *
+ * Ownership: the caller owns every buffer; inputs are copied before the call
+ * returns and no pointer is retained; outputs are written only when the call
+ * returns SMILESS_OK or SMILESS_INFEASIBLE.  The CUDA stream is borrowed.
+ * Threading: one context per host thread.  Every call is synchronous with
+ * respect to the host (results are on the host when it returns).
+ *
+ * Errors: negative return codes; smiless_last_error() returns a message.
+ * There is no CPU fallback: a missing GPU, driver or NVRTC returns
+ * SMILESS_ECUDA / SMILESS_EJIT.
+ */
+#ifndef SMILESS_H
+#define SMILESS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define SMILESS_API __attribute__((visibility("default")))
+#else
+#define SMILESS_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct smiless_ctx smiless_ctx;
+
+enum {
+    SMILESS_OK = 0,          /* success                                               */
+    SMILESS_INFEASIBLE = 1,  /* success, but no candidate meets the SLA (reading G13)  */
+    SMILESS_EINVAL = -1,     /* bad argument (null, size, range, unsorted arrivals ...) */
+    SMILESS_ENOTTOPO = -2,   /* DAG not a topologically ordered predecessor CSR         */
+    SMILESS_ERANGE = -3,     /* candidate space or index exceeds 2^63-1                 */
+    SMILESS_ESTATE = -4,     /* call order: plan/evaluate before load_dag+load_profiles */
+    SMILESS_ECUDA = -5,      /* CUDA runtime/driver failure or no device                */
+    SMILESS_ENOMEM = -6,     /* host or device allocation failed                        */
+    SMILESS_EJIT = -7        /* NVRTC specialisation of the evaluator failed            */
+};
+
+/* smiless_plan_args.flags */
+enum {
+    SMILESS_FLAG_NO_PRUNE = 1u,            /* throughput mode: walk every candidate to j = J-1 */
+    SMILESS_FLAG_ARRIVALS_ON_DEVICE = 2u,  /* arrivals_us is a device pointer (HBM-resident)   */
+    SMILESS_FLAG_FORCE_INT64 = 4u          /* use the int64 evaluator even if int32 is exact   */
+};
+
+#define SMILESS_MAX_FUNCS 32
+#define SMILESS_MAX_WINDOWS 32
+#define SMILESS_MAX_CONFIGS 256
+
+/* Create a context bound to CUDA device `cuda_device` and stream `cuda_stream`
+ * (a cudaStream_t; NULL = the legacy default stream; borrowed, not owned).
+ * Host-only calls (load_*, space_size, decode) never touch the GPU; device
+ * resources are acquired on the first plan/evaluate call.
+ * Returns OK, EINVAL (out == NULL or device < 0) or ENOMEM. */
+SMILESS_API int smiless_create(smiless_ctx **out, int cuda_device, void *cuda_stream);
+
+/* Replace the borrowed stream used by later calls. */
+SMILESS_API int smiless_set_stream(smiless_ctx *ctx, void *cuda_stream);
+
+/* Release everything the context owns.  NULL-safe. */
+SMILESS_API void smiless_destroy(smiless_ctx *ctx);
+
+/* Message of the last failing call on ctx ("" if none).  Owned by ctx; valid
+ * until the next call on ctx.  ctx == NULL gives the message of the last
+ * failed smiless_create on this thread. */
+SMILESS_API const char *smiless_last_error(const smiless_ctx *ctx);
+
+/* Load the application DAG (NetworkX in the paper)
+ * as a topologically ordered CSR over PREDECESSORS: function k's predecessors
+ * are pred_idx[pred_ptr[k] .. pred_ptr[k+1]), each p < k, no duplicates.
+ * Sources = empty predecessor list (they receive the request);
+ * sinks = functions no one lists (the request completes when all sinks have).
+ * 1 <= n_funcs <= SMILESS_MAX_FUNCS; pred_ptr has n_funcs+1 entries,
+ * pred_ptr[0] == 0, non-decreasing; pred_idx may be NULL when it is empty.
+ * Returns OK, EINVAL or ENOTTOPO.  Invalidates loaded profiles' compiled state. */
+SMILESS_API int smiless_load_dag(smiless_ctx *ctx, int32_t n_funcs, const int32_t *pred_ptr, const int32_t *pred_idx);
+
+/* Load per-function x per-config profiles: function k has
+ * n_configs[k] (1..SMILESS_MAX_CONFIGS) rows; exec_us, init_us and
+ * price_per_us are function-major, config-minor, length sum(n_configs).
+ * 0 <= exec_us, init_us < 2^29; price_per_us finite and >= 0.
+ * Requires a loaded DAG (else ESTATE).  Returns OK, EINVAL or ESTATE. */
+SMILESS_API int smiless_load_profiles(smiless_ctx *ctx, const int32_t *n_configs, const int32_t *exec_us,
+                          const int32_t *init_us, const double *price_per_us);
+
+typedef struct {
+    const int64_t *arrivals_us;   /* [n_arrivals] predicted arrivals r_0 <= r_1 <= ...;
+                                     host pointer, or device pointer with FLAG_ARRIVALS_ON_DEVICE;
+                                     |r_j| < 2^62                                                    */
+    int64_t n_arrivals;           /* J >= 1                                                         */
+    int64_t sla_us;               /* 0 <= SLA < 2^29; feasible iff max_j L_j <= SLA (G8)      */
+    const int32_t *windows_us;    /* [n_windows] strictly increasing, 0 <= w < 2^29 (0 = keep-alive) */
+    int32_t n_windows;            /* 1 <= W <= SMILESS_MAX_WINDOWS                                   */
+    int32_t n_fixed;              /* digits of functions 0..n_fixed-1 are pinned (0 <= n_fixed <= N) */
+    const int32_t *fixed_digits;  /* [n_fixed] digit = config * W + window; NULL if n_fixed == 0      */
+    uint64_t begin, end;          /* index sub-range [begin, end) of the suffix space; end = 0: all  */
+    uint32_t flags;               /* SMILESS_FLAG_*                                                  */
+    int32_t shard, n_shards;      /* multi-GPU: this rank plans chunks c with c % n_shards == shard;
+                                     n_shards = 0 or 1: everything                                   */
+} smiless_plan_args;
+
+typedef struct {
+    uint64_t index;           /* winning index in the suffix space; UINT64_MAX if infeasible      */
+    double cost;              /* its cost sum_k U_k * E_k ($); +inf if infeasible                  */
+    int64_t max_latency_us;   /* its max_j L_j; -1 if infeasible                                   */
+    uint64_t n_decided;       /* candidates of this shard's range that were decided               */
+    uint64_t n_full_evals;    /* candidates walked through all J arrivals                          */
+    double eval_kernel_ms;    /* device time of the evaluator kernel launches (CUDA events on the
+                                 launch stream)                                                    */
+    double total_device_ms;   /* device time of the whole call (first upload .. last kernel)      */
+    int32_t int64_path;       /* 1 if the int64 evaluator ran (int32 range check failed / forced)  */
+    int32_t launches;         /* kernels this call launched                                        */
+} smiless_plan_result;
+
+/* Size of the suffix candidate space prod_{k >= n_fixed} M_k * W.
+ * Returns OK, ESTATE (profiles not loaded), EINVAL or ERANGE (> 2^63-1). */
+SMILESS_API int smiless_space_size(const smiless_ctx *ctx, int32_t n_windows, int32_t n_fixed, uint64_t *out);
+
+/* The hot path: exhaustive SLA-constrained min-cost search over [begin, end)
+ * of the suffix space (this shard's chunks only when n_shards > 1).
+ * config_out / window_out ([n_funcs] or NULL) receive the winner's config and
+ * window index per function (the "execution strategy").
+ * Returns OK, INFEASIBLE (res->index = UINT64_MAX, cost = +inf,
+ * max_latency = -1, outputs set to -1), or an error. */
+SMILESS_API int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res,
+                 int32_t *config_out, int32_t *window_out);
+
+/* Exact int64 evaluation (no pruning, no clamping) of n explicit candidate
+ * indices of the suffix space: cost, max_j L_j and feasibility per index.
+ * a->begin/end/flags(NO_PRUNE)/shard are ignored.  Returns OK or an error
+ * (ERANGE if an index is outside the space). */
+SMILESS_API int smiless_evaluate(smiless_ctx *ctx, const smiless_plan_args *a, const uint64_t *idx, int64_t n,
+                     double *cost, int64_t *max_latency_us, uint8_t *feasible);
+
+/* Decode a suffix-space index into per-function config and window indices
+ * (pinned functions take their fixed digit).  Host-only.  Returns OK,
+ * ESTATE, EINVAL or ERANGE. */
+SMILESS_API int smiless_decode(const smiless_ctx *ctx, int32_t n_windows, uint64_t index, const smiless_plan_args *a,
+                   int32_t *config_out, int32_t *window_out);
+
+/* ---- introspection (build checks, SASS inspection, tests) --------------------------- */
+
+/* Copy the NVRTC source that smiless_plan would compile for (ctx, a) into buf
+ * (NUL-terminated, truncated to cap); *len receives the full size + 1.
+ * Host-only.  Returns OK, EINVAL, ESTATE or ERANGE. */
+SMILESS_API int smiless_kernel_source(smiless_ctx *ctx, const smiless_plan_args *a, char *buf, size_t cap,
+                                      size_t *len);
+
+/* NVRTC-compile that source for sm_100a without loading it (works without a GPU);
+ * the compile/ptxas log (registers, spills) goes to log.  Returns OK, EJIT or an
+ * argument error. */
+SMILESS_API int smiless_jit_compile(smiless_ctx *ctx, const smiless_plan_args *a, char *log, size_t logcap,
+                                    size_t *cubin_size);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* SMILESS_H */

@@ -1,0 +1,983 @@
+// host.cpp -- the C-ABI library (include/smiless.h): validation, derived tables, NVRTC
+// specialisation of the evaluator per (DAG, window grid, range mode), launches, result
+// decode.  SURVEY 8(a) steps a1-a10 on the host side; every per-candidate computation
+// runs in the CUDA kernels (evaluator.cuh via NVRTC, kernels.cu via nvcc).
+//
+// No CPU fallback: without a device, driver or NVRTC the calls fail with
+// SMILESS_ECUDA / SMILESS_EJIT.
+#include "smiless.h"
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nvrtc.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <sstream>
+#include <string>
+#include <vector>
+
+#include "kernels.h"
+
+extern "C" const char smiless_evaluator_src[];  // generated from evaluator.cuh at build time
+
+namespace {
+
+typedef long long i64;
+typedef unsigned long long u64;
+
+// ------------------------------------------------------------------------------------
+// Dynamically resolved NVRTC and CUDA driver entry points (so that the library loads on
+// a host without a GPU; nothing here runs until the first plan/evaluate).
+// ------------------------------------------------------------------------------------
+struct NvrtcApi {
+    bool ok = false;
+    std::string why;
+    decltype(&nvrtcCreateProgram) create = nullptr;
+    decltype(&nvrtcCompileProgram) compile = nullptr;
+    decltype(&nvrtcGetProgramLogSize) log_size = nullptr;
+    decltype(&nvrtcGetProgramLog) get_log = nullptr;
+    decltype(&nvrtcGetCUBINSize) cubin_size = nullptr;
+    decltype(&nvrtcGetCUBIN) get_cubin = nullptr;
+    decltype(&nvrtcDestroyProgram) destroy = nullptr;
+    decltype(&nvrtcGetErrorString) err_str = nullptr;
+};
+
+NvrtcApi &nvrtc() {
+    static NvrtcApi api;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        const char *env = getenv("SMILESS_NVRTC");
+        const char *cands[] = {env, "libnvrtc.so.12", "/usr/local/cuda/lib64/libnvrtc.so.12", "libnvrtc.so"};
+        void *h = nullptr;
+        for (const char *c : cands) {
+            if (!c) continue;
+            h = dlopen(c, RTLD_NOW | RTLD_LOCAL);
+            if (h) break;
+        }
+        if (!h) {
+            api.why = "cannot dlopen libnvrtc.so.12";
+            return;
+        }
+#define SMILESS_SYM(field, name)                                       \
+    api.field = reinterpret_cast<decltype(api.field)>(dlsym(h, name)); \
+    if (!api.field) { api.why = std::string("missing NVRTC symbol ") + name; return; }
+        SMILESS_SYM(create, "nvrtcCreateProgram");
+        SMILESS_SYM(compile, "nvrtcCompileProgram");
+        SMILESS_SYM(log_size, "nvrtcGetProgramLogSize");
+        SMILESS_SYM(get_log, "nvrtcGetProgramLog");
+        SMILESS_SYM(cubin_size, "nvrtcGetCUBINSize");
+        SMILESS_SYM(get_cubin, "nvrtcGetCUBIN");
+        SMILESS_SYM(destroy, "nvrtcDestroyProgram");
+        SMILESS_SYM(err_str, "nvrtcGetErrorString");
+#undef SMILESS_SYM
+        api.ok = true;
+    });
+    return api;
+}
+
+struct DriverApi {
+    bool ok = false;
+    std::string why;
+    CUresult (*moduleLoadData)(CUmodule *, const void *) = nullptr;
+    CUresult (*moduleUnload)(CUmodule) = nullptr;
+    CUresult (*moduleGetFunction)(CUfunction *, CUmodule, const char *) = nullptr;
+    CUresult (*funcSetAttribute)(CUfunction, CUfunction_attribute, int) = nullptr;
+    CUresult (*funcGetAttribute)(int *, CUfunction_attribute, CUfunction) = nullptr;
+    CUresult (*launchKernel)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
+                             CUstream, void **, void **) = nullptr;
+    CUresult (*occupancy)(int *, CUfunction, int, size_t) = nullptr;
+    CUresult (*getErrorString)(CUresult, const char **) = nullptr;
+};
+
+DriverApi &driver() {
+    static DriverApi api;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        auto get = [&](const char *name, void **fn) -> bool {
+            cudaDriverEntryPointQueryResult q;
+            cudaError_t e = cudaGetDriverEntryPointByVersion(name, fn, 12000, cudaEnableDefault, &q);
+            if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !*fn) {
+                api.why = std::string("cannot resolve driver entry point ") + name;
+                return false;
+            }
+            return true;
+        };
+        if (!get("cuModuleLoadData", (void **)&api.moduleLoadData)) return;
+        if (!get("cuModuleUnload", (void **)&api.moduleUnload)) return;
+        if (!get("cuModuleGetFunction", (void **)&api.moduleGetFunction)) return;
+        if (!get("cuFuncSetAttribute", (void **)&api.funcSetAttribute)) return;
+        if (!get("cuFuncGetAttribute", (void **)&api.funcGetAttribute)) return;
+        if (!get("cuLaunchKernel", (void **)&api.launchKernel)) return;
+        if (!get("cuOccupancyMaxActiveBlocksPerMultiprocessor", (void **)&api.occupancy)) return;
+        if (!get("cuGetErrorString", (void **)&api.getErrorString)) return;
+        api.ok = true;
+    });
+    return api;
+}
+
+// ------------------------------------------------------------------------------------
+// Kernel parameter block: must match PlanParams in evaluator.cuh byte for byte.
+// ------------------------------------------------------------------------------------
+struct PlanParamsHost {
+    const int *tabI;
+    const int *tabT;
+    const double *tabU;
+    const void *off;
+    const i64 *scal;
+    u64 *counter;
+    u64 *stats;
+    u64 *blk_best;
+    u64 unit_begin, unit_end;
+    u64 cand_begin, cand_end;
+    u64 claims_end;
+    u64 claims_begin;
+    i64 n_steps;
+    i64 n_off;
+    int sumM;
+    int sla;
+    int prune;
+    int shard, n_shards;
+    int chunk_units;
+    int fixed[SMILESS_MAX_FUNCS];  // evaluator uses SM_NFIXED_ALLOC <= SMILESS_MAX_FUNCS; extra tail is ignored
+};
+
+constexpr int kThreads = 256;
+constexpr int kChunkUnits = 256;     // sharding / claim granularity in units (multiple of 32)
+
+struct JitKernel {
+    CUmodule mod = nullptr;
+    CUfunction fn = nullptr;
+    size_t smem = 0;
+    int blocks_per_sm = 0;
+    int regs = 0;
+    size_t params_size = 0;
+};
+
+template <typename T>
+struct DevBuf {
+    T *p = nullptr;
+    size_t n = 0;
+    cudaError_t ensure(size_t want) {
+        if (want <= n && p) return cudaSuccess;
+        if (p) cudaFree(p);
+        p = nullptr;
+        n = 0;
+        cudaError_t e = cudaMalloc((void **)&p, std::max<size_t>(want, 1) * sizeof(T));
+        if (e == cudaSuccess) n = want;
+        return e;
+    }
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        n = 0;
+    }
+};
+
+}  // namespace
+
+struct smiless_ctx {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    std::string err;
+
+    // DAG
+    int N = 0;
+    std::vector<int32_t> pred_ptr, pred_idx;
+    u64 sinkmask = 0;
+    bool dag_loaded = false;
+
+    // profiles
+    std::vector<int32_t> M, row0;
+    std::vector<int32_t> I, T;
+    std::vector<double> U;
+    int sumM = 0;
+    i64 Tmax = 0, Imax = 0;
+    bool prof_loaded = false;
+    bool tables_dirty = true;
+
+    // device state
+    bool dev_ready = false;
+    int n_sms = 0;
+    DevBuf<int> dI, dT, dPtr, dIdx;
+    DevBuf<double> dU;
+    DevBuf<i64> dArr;
+    DevBuf<unsigned char> dOff;
+    DevBuf<i64> dScal;
+    DevBuf<int> dErr;
+    DevBuf<u64> dCounter, dStats, dBlk, dIdxEval;
+    DevBuf<double> dCost;
+    DevBuf<i64> dLat;
+    DevBuf<unsigned char> dFeas;
+    DevBuf<ResBlock> dRes;
+    ResBlock *hRes = nullptr;    // pinned
+    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+
+    std::map<std::string, JitKernel> jit_cache;
+};
+
+namespace {
+
+thread_local std::string g_create_err;
+
+int fail(smiless_ctx *c, int code, const char *fmt, ...) {
+    char buf[1024];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    if (c) c->err = buf;
+    return code;
+}
+
+int cuda_fail(smiless_ctx *c, cudaError_t e, const char *what) {
+    return fail(c, SMILESS_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+int drv_fail(smiless_ctx *c, CUresult r, const char *what) {
+    const char *s = "?";
+    if (driver().getErrorString) driver().getErrorString(r, &s);
+    return fail(c, SMILESS_ECUDA, "%s: %s", what, s);
+}
+
+#define CK(expr, what)                                          \
+    do {                                                        \
+        cudaError_t e_ = (expr);                                \
+        if (e_ != cudaSuccess) return cuda_fail(ctx, e_, what); \
+    } while (0)
+
+int ensure_device(smiless_ctx *ctx) {
+    if (ctx->dev_ready) return SMILESS_OK;
+    int n = 0;
+    cudaError_t e = cudaGetDeviceCount(&n);
+    if (e != cudaSuccess || n == 0) return fail(ctx, SMILESS_ECUDA, "no CUDA device: %s", cudaGetErrorString(e));
+    if (ctx->device >= n) return fail(ctx, SMILESS_ECUDA, "device %d out of range (%d devices)", ctx->device, n);
+    CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+    CK(cudaFree(nullptr), "context init");
+    cudaDeviceProp prop;
+    CK(cudaGetDeviceProperties(&prop, ctx->device), "cudaGetDeviceProperties");
+    if (prop.major != 10 || prop.minor != 0)
+        return fail(ctx, SMILESS_ECUDA, "device %d is sm_%d%d; this library is built for sm_100a (B200)", ctx->device,
+                    prop.major, prop.minor);
+    ctx->n_sms = prop.multiProcessorCount;
+    if (!driver().ok) return fail(ctx, SMILESS_ECUDA, "CUDA driver API: %s", driver().why.c_str());
+    for (auto &ev : ctx->ev) CK(cudaEventCreate(&ev), "cudaEventCreate");
+    CK(cudaMallocHost((void **)&ctx->hRes, sizeof(ResBlock)), "cudaMallocHost");
+    CK(ctx->dRes.ensure(1), "cudaMalloc");
+    CK(ctx->dScal.ensure(2), "cudaMalloc");
+    CK(ctx->dErr.ensure(1), "cudaMalloc");
+    CK(ctx->dCounter.ensure(1), "cudaMalloc");
+    CK(ctx->dStats.ensure(2), "cudaMalloc");
+    ctx->dev_ready = true;
+    return SMILESS_OK;
+}
+
+int upload_tables(smiless_ctx *ctx) {
+    if (!ctx->tables_dirty) return SMILESS_OK;
+    const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
+    const size_t padU = (size_t)((ctx->sumM + 1) & ~1);
+    std::vector<int> I(padI, 0), T(padI, 0);
+    std::vector<double> U(padU, 0.0);
+    std::copy(ctx->I.begin(), ctx->I.end(), I.begin());
+    std::copy(ctx->T.begin(), ctx->T.end(), T.begin());
+    std::copy(ctx->U.begin(), ctx->U.end(), U.begin());
+    CK(ctx->dI.ensure(padI), "cudaMalloc");
+    CK(ctx->dT.ensure(padI), "cudaMalloc");
+    CK(ctx->dU.ensure(padU), "cudaMalloc");
+    CK(ctx->dPtr.ensure(ctx->pred_ptr.size()), "cudaMalloc");
+    CK(ctx->dIdx.ensure(std::max<size_t>(ctx->pred_idx.size(), 1)), "cudaMalloc");
+    CK(cudaMemcpy(ctx->dI.p, I.data(), padI * sizeof(int), cudaMemcpyHostToDevice), "H2D tables");
+    CK(cudaMemcpy(ctx->dT.p, T.data(), padI * sizeof(int), cudaMemcpyHostToDevice), "H2D tables");
+    CK(cudaMemcpy(ctx->dU.p, U.data(), padU * sizeof(double), cudaMemcpyHostToDevice), "H2D tables");
+    CK(cudaMemcpy(ctx->dPtr.p, ctx->pred_ptr.data(), ctx->pred_ptr.size() * sizeof(int), cudaMemcpyHostToDevice),
+       "H2D dag");
+    if (!ctx->pred_idx.empty())
+        CK(cudaMemcpy(ctx->dIdx.p, ctx->pred_idx.data(), ctx->pred_idx.size() * sizeof(int), cudaMemcpyHostToDevice),
+           "H2D dag");
+    ctx->tables_dirty = false;
+    return SMILESS_OK;
+}
+
+// ------------------------------------------------------------------------------------
+// Argument validation and derived quantities
+// ------------------------------------------------------------------------------------
+bool space_size_of(const smiless_ctx *c, int W, int n_fixed, u64 *out) {
+    unsigned __int128 s = 1;
+    for (int k = n_fixed; k < c->N; ++k) {
+        s *= (unsigned __int128)((u64)c->M[k] * (u64)W);
+        if (s > (unsigned __int128)INT64_MAX) return false;
+    }
+    *out = (u64)s;
+    return true;
+}
+
+int validate_args(smiless_ctx *ctx, const smiless_plan_args *a, bool need_arrivals_host_check) {
+    if (!a) return fail(ctx, SMILESS_EINVAL, "args is NULL");
+    if (!ctx->dag_loaded || !ctx->prof_loaded) return fail(ctx, SMILESS_ESTATE, "load_dag and load_profiles first");
+    if (a->n_windows < 1 || a->n_windows > SMILESS_MAX_WINDOWS)
+        return fail(ctx, SMILESS_EINVAL, "n_windows must be in [1, %d]", SMILESS_MAX_WINDOWS);
+    if (!a->windows_us) return fail(ctx, SMILESS_EINVAL, "windows_us is NULL");
+    for (int v = 0; v < a->n_windows; ++v) {
+        if (a->windows_us[v] < 0 || a->windows_us[v] >= (1 << 29))
+            return fail(ctx, SMILESS_EINVAL, "window %d out of [0, 2^29)", v);
+        if (v && a->windows_us[v] <= a->windows_us[v - 1])
+            return fail(ctx, SMILESS_EINVAL, "windows must be strictly increasing");
+    }
+    if (a->sla_us < 0 || a->sla_us >= (1ll << 29)) return fail(ctx, SMILESS_EINVAL, "sla_us out of [0, 2^29)");
+    if (a->n_arrivals < 1) return fail(ctx, SMILESS_EINVAL, "n_arrivals must be >= 1");
+    if (a->n_arrivals > (1ll << 31)) return fail(ctx, SMILESS_EINVAL, "n_arrivals too large");
+    if (!a->arrivals_us) return fail(ctx, SMILESS_EINVAL, "arrivals_us is NULL");
+    if (need_arrivals_host_check && !(a->flags & SMILESS_FLAG_ARRIVALS_ON_DEVICE)) {
+        const i64 LIM = (i64)1 << 62;
+        for (i64 j = 0; j < a->n_arrivals; ++j) {
+            const i64 r = a->arrivals_us[j];
+            if (r <= -LIM || r >= LIM) return fail(ctx, SMILESS_EINVAL, "arrival %lld out of range", (long long)j);
+            if (j && r < a->arrivals_us[j - 1])
+                return fail(ctx, SMILESS_EINVAL, "arrivals must be non-decreasing (index %lld)", (long long)j);
+        }
+    }
+    if (a->n_fixed < 0 || a->n_fixed > ctx->N) return fail(ctx, SMILESS_EINVAL, "n_fixed out of [0, N]");
+    if (a->n_fixed > 0 && !a->fixed_digits) return fail(ctx, SMILESS_EINVAL, "fixed_digits is NULL");
+    for (int k = 0; k < a->n_fixed; ++k)
+        if (a->fixed_digits[k] < 0 || (i64)a->fixed_digits[k] >= (i64)ctx->M[k] * a->n_windows)
+            return fail(ctx, SMILESS_EINVAL, "fixed digit %d out of range", k);
+    u64 space;
+    if (!space_size_of(ctx, a->n_windows, a->n_fixed, &space))
+        return fail(ctx, SMILESS_ERANGE, "candidate space exceeds 2^63-1; pin leading digits with n_fixed");
+    if (a->n_shards < 0 || (a->n_shards > 0 && (a->shard < 0 || a->shard >= a->n_shards)))
+        return fail(ctx, SMILESS_EINVAL, "bad shard/n_shards");
+    return SMILESS_OK;
+}
+
+std::string fmt_ll(long long v) { return std::to_string(v); }
+
+// Choose the int32 chunk length K (or the int64 path): every relative value of a candidate
+// still within the SLA must fit in int32.
+struct RangePlan {
+    bool time64;
+    int K;
+    i64 d_cap;
+};
+
+RangePlan range_plan(const smiless_ctx *ctx, const smiless_plan_args *a) {
+    const i64 wmax = a->windows_us[a->n_windows - 1];
+    const i64 sla = a->sla_us;
+    const i64 d_cap = sla + wmax + ctx->Tmax + 1;
+    RangePlan rp{true, 64, d_cap};
+    if (a->flags & SMILESS_FLAG_FORCE_INT64) return rp;
+    const i64 LIM = 0x7fffffffll;
+    for (int K : {64, 32, 16, 8, 4}) {
+        const i64 bound = (i64)K * d_cap + sla + (i64)ctx->N * (ctx->Tmax + ctx->Imax) + wmax + ctx->Tmax;
+        if (bound < LIM && (i64)K * wmax < LIM) return RangePlan{false, K, d_cap};
+    }
+    return rp;
+}
+
+// ------------------------------------------------------------------------------------
+// NVRTC specialisation
+// ------------------------------------------------------------------------------------
+std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, bool off_smem,
+                            int minb) {
+    const int N = ctx->N, W = a->n_windows, NU = N - 1, nf = a->n_fixed;
+    std::ostringstream s;
+    s << "// generated by host.cpp:dag_spec_source -- DAG-specialised prefix of evaluator.cuh\n";
+    s << "#define SM_N " << N << "\n#define SM_NU " << NU << "\n#define SM_NU_ALLOC " << std::max(NU, 1) << "\n";
+    s << "#define SM_W " << W << "\n#define SM_NFIXED " << nf << "\n#define SM_NFIXED_ALLOC " << SMILESS_MAX_FUNCS
+      << "\n";
+    s << "#define SM_K " << rp.K << "\n#define SM_TIME64 " << (rp.time64 ? 1 : 0) << "\n";
+    s << "#define SM_OFF_SMEM " << (off_smem ? 1 : 0) << "\n#define SM_THREADS " << kThreads
+      << "\n#define SM_MINB " << minb << "\n";
+    s << "#define SM_W0_ZERO " << (a->windows_us[0] == 0 ? 1 : 0) << "\n";
+    // compile-time window grid (immediates) and a constant-bank copy for runtime indices
+    s << "#define SM_WIN(v) (";
+    for (int v = 0; v < W; ++v) s << "(v)==" << v << "?" << a->windows_us[v] << ":";
+    s << "0)\n";
+    s << "__constant__ int c_win[" << W << "] = {";
+    for (int v = 0; v < W; ++v) s << (v ? "," : "") << a->windows_us[v];
+    s << "};\n#define SM_WINV(i) c_win[(i)]\n";
+    s << "#define SM_ROW0(k) (";
+    for (int k = 0; k < N; ++k) s << "(k)==" << k << "?" << ctx->row0[k] << ":";
+    s << "0)\n";
+    s << R"(
+typedef long long i64;
+typedef unsigned long long u64;
+#if SM_TIME64
+typedef long long tm_t;
+#else
+typedef int tm_t;
+#endif
+static __device__ __forceinline__ void fstep(tm_t &F, tm_t &SU, tm_t x, tm_t I, tm_t Te, tm_t w);
+static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
+static __device__ __forceinline__ tm_t vaddmax(tm_t a, tm_t b, tm_t c);
+)";
+    // ---- decode: unit u -> digits (function N-1: config only) -------------------------
+    s << "static __device__ __forceinline__ void dag_decode(u64 u, int (&dig)[SM_N], const int *fixed) {\n";
+    if (nf <= N - 1) {
+        s << "  dig[" << N - 1 << "] = (int)(u % " << ctx->M[N - 1] << "ull); u /= " << ctx->M[N - 1] << "ull;\n";
+        for (int k = N - 2; k >= nf; --k) {
+            const u64 radix = (u64)ctx->M[k] * (u64)W;
+            s << "  dig[" << k << "] = (int)(u % " << radix << "ull); u /= " << radix << "ull;\n";
+        }
+    }
+    for (int k = 0; k < nf; ++k) s << "  dig[" << k << "] = fixed[" << k << "];\n";
+    s << "  (void)u; (void)fixed;\n}\n";
+
+    // ---- input expressions --------------------------------------------------------------
+    auto x_expr = [&](int k, const char *src) {
+        const int e0 = ctx->pred_ptr[k], e1 = ctx->pred_ptr[k + 1];
+        if (e0 == e1) return std::string(src);
+        std::string e = "F[" + std::to_string(ctx->pred_idx[e0]) + "]";
+        for (int e_ = e0 + 1; e_ < e1; ++e_) e = "vmax(" + e + ", F[" + std::to_string(ctx->pred_idx[e_]) + "])";
+        return e;
+    };
+    // ---- j = 0 ----------------------------------------------------------------------------
+    s << "template <int A> static __device__ __forceinline__ void dag_first(tm_t (&F)[A], const tm_t (&I)[A], "
+         "tm_t *st0, int tid, tm_t &xl, tm_t &upL) {\n";
+    for (int k = 0; k < N - 1; ++k) {
+        s << "  { const tm_t x = " << x_expr(k, "(tm_t)0") << "; st0[" << k << " * SM_THREADS + tid] = x; F[" << k
+          << "] = x + I[" << k << "]; }\n";
+    }
+    s << "  xl = " << x_expr(N - 1, "(tm_t)0") << ";\n";
+    for (int k = 0; k < N - 1; ++k)
+        if ((ctx->sinkmask >> k) & 1ull) s << "  upL = vmax(upL, F[" << k << "]);\n";
+    s << "  (void)F; (void)I; (void)st0; (void)tid; (void)upL;\n}\n";
+    // ---- j >= 1 -----------------------------------------------------------------------------
+    s << "template <int A> static __device__ __forceinline__ void dag_step(tm_t (&F)[A], tm_t (&SU)[A], const tm_t "
+         "(&I)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], tm_t o, tm_t negO, tm_t &xl, tm_t &upL) {\n";
+    for (int k = 0; k < N - 1; ++k)
+        s << "  fstep(F[" << k << "], SU[" << k << "], " << x_expr(k, "o") << ", I[" << k << "], Te[" << k
+          << "], Wn[" << k << "]);\n";
+    s << "  xl = " << x_expr(N - 1, "o") << ";\n";
+    for (int k = 0; k < N - 1; ++k)
+        if ((ctx->sinkmask >> k) & 1ull) s << "  upL = vaddmax(F[" << k << "], negO, upL);\n";
+    s << "  (void)F; (void)SU; (void)I; (void)Te; (void)Wn; (void)o; (void)negO; (void)upL;\n}\n";
+    return s.str();
+}
+
+std::string full_source(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, bool off_smem,
+                        int minb) {
+    return dag_spec_source(ctx, a, rp, off_smem, minb) + "\n" + smiless_evaluator_src;
+}
+
+int nvrtc_compile(smiless_ctx *ctx, const std::string &src, std::vector<char> &cubin, std::string &log) {
+    NvrtcApi &nv = nvrtc();
+    if (!nv.ok) return fail(ctx, SMILESS_EJIT, "NVRTC unavailable: %s", nv.why.c_str());
+    nvrtcProgram prog;
+    nvrtcResult r = nv.create(&prog, src.c_str(), "smiless_evaluator.cu", 0, nullptr, nullptr);
+    if (r != NVRTC_SUCCESS) return fail(ctx, SMILESS_EJIT, "nvrtcCreateProgram: %s", nv.err_str(r));
+    const char *opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-default-device", "-lineinfo", "-fmad=false",
+                          "--ptxas-options=-v"};
+    r = nv.compile(prog, (int)(sizeof opts / sizeof *opts), opts);
+    size_t ls = 0;
+    nv.log_size(prog, &ls);
+    log.assign(ls, '\0');
+    if (ls) nv.get_log(prog, &log[0]);
+    if (r != NVRTC_SUCCESS) {
+        nv.destroy(&prog);
+        return fail(ctx, SMILESS_EJIT, "NVRTC compile failed: %s\n%s", nv.err_str(r), log.c_str());
+    }
+    size_t cs = 0;
+    nv.cubin_size(prog, &cs);
+    cubin.resize(cs);
+    nv.get_cubin(prog, cubin.data());
+    nv.destroy(&prog);
+    return SMILESS_OK;
+}
+
+size_t smem_bytes(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off, bool off_smem) {
+    const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
+    const size_t padU = (size_t)((ctx->sumM + 1) & ~1);
+    const size_t tsz = rp.time64 ? 8 : 4;
+    size_t b = 2 * padI * 4 + padU * 8;
+    b += 8ull * (size_t)(ctx->N - 1 + a->n_windows) * kThreads;
+    b += (tsz * (size_t)ctx->N * kThreads + 15) & ~(size_t)15;
+    if (off_smem) b += tsz * (size_t)n_off;
+    return b;
+}
+
+int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off, JitKernel **out) {
+    // offsets in shared memory when they fit next to the per-thread accumulators
+    const size_t max_smem = 227 * 1024;
+    bool off_smem = smem_bytes(ctx, a, rp, n_off, true) <= max_smem;
+    const int minb = 1;
+    std::string src = full_source(ctx, a, rp, off_smem, minb);
+    auto it = ctx->jit_cache.find(src);
+    if (it == ctx->jit_cache.end()) {
+        std::vector<char> cubin;
+        std::string log;
+        int rc = nvrtc_compile(ctx, src, cubin, log);
+        if (rc) return rc;
+        JitKernel jk;
+        CUresult r = driver().moduleLoadData(&jk.mod, cubin.data());
+        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleLoadData");
+        r = driver().moduleGetFunction(&jk.fn, jk.mod, "smiless_plan_kernel");
+        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction");
+        jk.smem = smem_bytes(ctx, a, rp, n_off, off_smem);
+        r = driver().funcSetAttribute(jk.fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)jk.smem);
+        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(smem)");
+        driver().funcGetAttribute(&jk.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, jk.fn);
+        r = driver().occupancy(&jk.blocks_per_sm, jk.fn, kThreads, jk.smem);
+        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuOccupancyMaxActiveBlocksPerMultiprocessor");
+        if (jk.blocks_per_sm < 1) return fail(ctx, SMILESS_ECUDA, "evaluator does not fit on an SM (smem %zu)", jk.smem);
+        it = ctx->jit_cache.emplace(src, jk).first;
+    }
+    *out = &it->second;
+    return SMILESS_OK;
+}
+
+void fill_exact_params(const smiless_ctx *ctx, const smiless_plan_args *a, const i64 *d_arr, ExactParams &ep) {
+    memset(&ep, 0, sizeof ep);
+    ep.tabI = ctx->dI.p;
+    ep.tabT = ctx->dT.p;
+    ep.tabU = ctx->dU.p;
+    ep.arr = (const long long *)d_arr;
+    ep.J = a->n_arrivals;
+    ep.sla = a->sla_us;
+    ep.N = ctx->N;
+    ep.W = a->n_windows;
+    ep.n_fixed = a->n_fixed;
+    ep.sinkmask = (unsigned)ctx->sinkmask;
+    ep.pred_ptr = ctx->dPtr.p;
+    ep.pred_idx = ctx->dIdx.p;
+    for (int k = 0; k < ctx->N; ++k) {
+        ep.M[k] = ctx->M[k];
+        ep.row0[k] = ctx->row0[k];
+    }
+    for (int v = 0; v < a->n_windows; ++v) ep.win[v] = a->windows_us[v];
+    for (int k = 0; k < a->n_fixed; ++k) ep.fixed[k] = a->fixed_digits[k];
+}
+
+// Upload (host) or adopt (device) the arrival sequence; returns the device pointer.
+int stage_arrivals(smiless_ctx *ctx, const smiless_plan_args *a, const i64 **d_arr) {
+    if (a->flags & SMILESS_FLAG_ARRIVALS_ON_DEVICE) {
+        *d_arr = (const i64 *)a->arrivals_us;
+        return SMILESS_OK;
+    }
+    CK(ctx->dArr.ensure((size_t)a->n_arrivals), "cudaMalloc arrivals");
+    CK(cudaMemcpyAsync(ctx->dArr.p, a->arrivals_us, (size_t)a->n_arrivals * sizeof(i64), cudaMemcpyHostToDevice,
+                       ctx->stream),
+       "H2D arrivals");
+    *d_arr = ctx->dArr.p;
+    return SMILESS_OK;
+}
+
+}  // namespace
+
+// ======================================================================================
+// C ABI
+// ======================================================================================
+extern "C" {
+
+int smiless_create(smiless_ctx **out, int cuda_device, void *cuda_stream) {
+    if (!out) {
+        g_create_err = "out is NULL";
+        return SMILESS_EINVAL;
+    }
+    *out = nullptr;
+    if (cuda_device < 0) {
+        g_create_err = "cuda_device must be >= 0";
+        return SMILESS_EINVAL;
+    }
+    smiless_ctx *c = new (std::nothrow) smiless_ctx();
+    if (!c) {
+        g_create_err = "out of host memory";
+        return SMILESS_ENOMEM;
+    }
+    c->device = cuda_device;
+    c->stream = (cudaStream_t)cuda_stream;
+    *out = c;
+    return SMILESS_OK;
+}
+
+int smiless_set_stream(smiless_ctx *ctx, void *cuda_stream) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->stream = (cudaStream_t)cuda_stream;
+    return SMILESS_OK;
+}
+
+void smiless_destroy(smiless_ctx *ctx) {
+    if (!ctx) return;
+    if (ctx->dev_ready) {
+        cudaSetDevice(ctx->device);
+        for (auto &kv : ctx->jit_cache)
+            if (kv.second.mod) driver().moduleUnload(kv.second.mod);
+        ctx->dI.release(); ctx->dT.release(); ctx->dU.release(); ctx->dPtr.release(); ctx->dIdx.release();
+        ctx->dArr.release(); ctx->dOff.release(); ctx->dScal.release(); ctx->dErr.release();
+        ctx->dCounter.release(); ctx->dStats.release(); ctx->dBlk.release(); ctx->dIdxEval.release();
+        ctx->dCost.release(); ctx->dLat.release(); ctx->dFeas.release(); ctx->dRes.release();
+        if (ctx->hRes) cudaFreeHost(ctx->hRes);
+        for (auto &ev : ctx->ev)
+            if (ev) cudaEventDestroy(ev);
+    }
+    delete ctx;
+}
+
+const char *smiless_last_error(const smiless_ctx *ctx) {
+    if (!ctx) return g_create_err.c_str();
+    return ctx->err.c_str();
+}
+
+int smiless_load_dag(smiless_ctx *ctx, int32_t n_funcs, const int32_t *pred_ptr, const int32_t *pred_idx) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->err.clear();
+    if (n_funcs < 1 || n_funcs > SMILESS_MAX_FUNCS)
+        return fail(ctx, SMILESS_EINVAL, "n_funcs must be in [1, %d]", SMILESS_MAX_FUNCS);
+    if (!pred_ptr) return fail(ctx, SMILESS_EINVAL, "pred_ptr is NULL");
+    if (pred_ptr[0] != 0) return fail(ctx, SMILESS_EINVAL, "pred_ptr[0] must be 0");
+    for (int k = 0; k < n_funcs; ++k)
+        if (pred_ptr[k + 1] < pred_ptr[k]) return fail(ctx, SMILESS_EINVAL, "pred_ptr must be non-decreasing");
+    const int E = pred_ptr[n_funcs];
+    if (E > SMILESS_DEV_MAX_EDGES) return fail(ctx, SMILESS_EINVAL, "too many edges");
+    if (E > 0 && !pred_idx) return fail(ctx, SMILESS_EINVAL, "pred_idx is NULL");
+    u64 sinkmask = (n_funcs == 64) ? ~0ull : ((1ull << n_funcs) - 1);
+    for (int k = 0; k < n_funcs; ++k) {
+        u64 seen = 0;
+        for (int e = pred_ptr[k]; e < pred_ptr[k + 1]; ++e) {
+            const int p = pred_idx[e];
+            if (p < 0 || p >= n_funcs) return fail(ctx, SMILESS_EINVAL, "pred_idx[%d] out of range", e);
+            if (p >= k)
+                return fail(ctx, SMILESS_ENOTTOPO, "function %d lists predecessor %d >= itself (not topological)", k, p);
+            if ((seen >> p) & 1ull) return fail(ctx, SMILESS_EINVAL, "duplicate predecessor %d of %d", p, k);
+            seen |= 1ull << p;
+            sinkmask &= ~(1ull << p);
+        }
+    }
+    ctx->N = n_funcs;
+    ctx->pred_ptr.assign(pred_ptr, pred_ptr + n_funcs + 1);
+    ctx->pred_idx.assign(pred_idx ? pred_idx : pred_ptr, pred_idx ? pred_idx + E : pred_ptr);
+    ctx->sinkmask = sinkmask;
+    ctx->dag_loaded = true;
+    ctx->prof_loaded = false;  // profiles are per function: reload after a new DAG
+    ctx->tables_dirty = true;
+    return SMILESS_OK;
+}
+
+int smiless_load_profiles(smiless_ctx *ctx, const int32_t *n_configs, const int32_t *exec_us, const int32_t *init_us,
+                          const double *price_per_us) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->err.clear();
+    if (!ctx->dag_loaded) return fail(ctx, SMILESS_ESTATE, "load_dag first");
+    if (!n_configs || !exec_us || !init_us || !price_per_us) return fail(ctx, SMILESS_EINVAL, "NULL profile array");
+    int sum = 0;
+    std::vector<int32_t> M(ctx->N), row0(ctx->N);
+    for (int k = 0; k < ctx->N; ++k) {
+        if (n_configs[k] < 1 || n_configs[k] > SMILESS_MAX_CONFIGS)
+            return fail(ctx, SMILESS_EINVAL, "n_configs[%d] must be in [1, %d]", k, SMILESS_MAX_CONFIGS);
+        M[k] = n_configs[k];
+        row0[k] = sum;
+        sum += n_configs[k];
+    }
+    i64 tmax = 0, imax = 0;
+    for (int r = 0; r < sum; ++r) {
+        if (exec_us[r] < 0 || exec_us[r] >= (1 << 29)) return fail(ctx, SMILESS_EINVAL, "exec_us[%d] out of [0, 2^29)", r);
+        if (init_us[r] < 0 || init_us[r] >= (1 << 29)) return fail(ctx, SMILESS_EINVAL, "init_us[%d] out of [0, 2^29)", r);
+        if (!std::isfinite(price_per_us[r]) || price_per_us[r] < 0)
+            return fail(ctx, SMILESS_EINVAL, "price_per_us[%d] must be finite and >= 0", r);
+        tmax = std::max<i64>(tmax, init_us[r]);
+        imax = std::max<i64>(imax, exec_us[r]);
+    }
+    ctx->M = M;
+    ctx->row0 = row0;
+    ctx->sumM = sum;
+    ctx->I.assign(exec_us, exec_us + sum);
+    ctx->T.assign(init_us, init_us + sum);
+    ctx->U.assign(price_per_us, price_per_us + sum);
+    ctx->Tmax = tmax;
+    ctx->Imax = imax;
+    ctx->prof_loaded = true;
+    ctx->tables_dirty = true;
+    return SMILESS_OK;
+}
+
+int smiless_space_size(const smiless_ctx *ctx, int32_t n_windows, int32_t n_fixed, uint64_t *out) {
+    if (!ctx || !out) return SMILESS_EINVAL;
+    if (!ctx->dag_loaded || !ctx->prof_loaded) return SMILESS_ESTATE;
+    if (n_windows < 1 || n_windows > SMILESS_MAX_WINDOWS || n_fixed < 0 || n_fixed > ctx->N) return SMILESS_EINVAL;
+    u64 s;
+    if (!space_size_of(ctx, n_windows, n_fixed, &s)) return SMILESS_ERANGE;
+    *out = s;
+    return SMILESS_OK;
+}
+
+int smiless_decode(const smiless_ctx *ctx, int32_t n_windows, uint64_t index, const smiless_plan_args *a,
+                   int32_t *config_out, int32_t *window_out) {
+    if (!ctx || !config_out || !window_out) return SMILESS_EINVAL;
+    if (!ctx->dag_loaded || !ctx->prof_loaded) return SMILESS_ESTATE;
+    const int nf = a ? a->n_fixed : 0;
+    if (n_windows < 1 || n_windows > SMILESS_MAX_WINDOWS || nf < 0 || nf > ctx->N) return SMILESS_EINVAL;
+    if (nf > 0 && !a->fixed_digits) return SMILESS_EINVAL;
+    u64 space;
+    if (!space_size_of(ctx, n_windows, nf, &space)) return SMILESS_ERANGE;
+    if (index >= space) return SMILESS_ERANGE;
+    for (int k = ctx->N - 1; k >= nf; --k) {
+        const u64 radix = (u64)ctx->M[k] * (u64)n_windows;
+        const u64 d = index % radix;
+        index /= radix;
+        config_out[k] = (int32_t)(d / (u64)n_windows);
+        window_out[k] = (int32_t)(d % (u64)n_windows);
+    }
+    for (int k = 0; k < nf; ++k) {
+        if (a->fixed_digits[k] < 0 || (i64)a->fixed_digits[k] >= (i64)ctx->M[k] * n_windows) return SMILESS_EINVAL;
+        config_out[k] = a->fixed_digits[k] / n_windows;
+        window_out[k] = a->fixed_digits[k] % n_windows;
+    }
+    return SMILESS_OK;
+}
+
+int smiless_evaluate(smiless_ctx *ctx, const smiless_plan_args *a, const uint64_t *idx, int64_t n, double *cost,
+                     int64_t *max_latency_us, uint8_t *feasible) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->err.clear();
+    int rc = validate_args(ctx, a, true);
+    if (rc) return rc;
+    if (n < 0 || (n > 0 && (!idx || !cost || !max_latency_us || !feasible)))
+        return fail(ctx, SMILESS_EINVAL, "bad output arrays");
+    u64 space;
+    space_size_of(ctx, a->n_windows, a->n_fixed, &space);
+    for (i64 i = 0; i < n; ++i)
+        if (idx[i] >= space) return fail(ctx, SMILESS_ERANGE, "index %llu outside the space", (unsigned long long)idx[i]);
+    if (n == 0) return SMILESS_OK;
+    if ((rc = ensure_device(ctx))) return rc;
+    CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+    if ((rc = upload_tables(ctx))) return rc;
+    const i64 *d_arr = nullptr;
+    if ((rc = stage_arrivals(ctx, a, &d_arr))) return rc;
+    CK(ctx->dIdxEval.ensure((size_t)n), "cudaMalloc");
+    CK(ctx->dCost.ensure((size_t)n), "cudaMalloc");
+    CK(ctx->dLat.ensure((size_t)n), "cudaMalloc");
+    CK(ctx->dFeas.ensure((size_t)n), "cudaMalloc");
+    CK(cudaMemcpyAsync(ctx->dIdxEval.p, idx, (size_t)n * 8, cudaMemcpyHostToDevice, ctx->stream), "H2D idx");
+    ExactParams ep;
+    fill_exact_params(ctx, a, d_arr, ep);
+    ep.idx = ctx->dIdxEval.p;
+    ep.n = n;
+    ep.cost = ctx->dCost.p;
+    ep.maxlat = (long long *)ctx->dLat.p;
+    ep.feas = ctx->dFeas.p;
+    ep.idx_from_res = 0;
+    int e = smiless_dev_eval_exact(&ep, ctx->stream);
+    if (e) return cuda_fail(ctx, (cudaError_t)e, "eval_exact launch");
+    CK(cudaMemcpyAsync(cost, ctx->dCost.p, (size_t)n * 8, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
+    CK(cudaMemcpyAsync(max_latency_us, ctx->dLat.p, (size_t)n * 8, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
+    CK(cudaMemcpyAsync(feasible, ctx->dFeas.p, (size_t)n, cudaMemcpyDeviceToHost, ctx->stream), "D2H");
+    CK(cudaStreamSynchronize(ctx->stream), "evaluate");
+    return SMILESS_OK;
+}
+
+int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res, int32_t *config_out,
+                 int32_t *window_out) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->err.clear();
+    if (!res) return fail(ctx, SMILESS_EINVAL, "res is NULL");
+    int rc = validate_args(ctx, a, true);
+    if (rc) return rc;
+    u64 space;
+    space_size_of(ctx, a->n_windows, a->n_fixed, &space);
+    const u64 cb = a->begin;
+    const u64 ce = (a->end == 0 || a->end > space) ? space : a->end;
+    if (cb > ce) return fail(ctx, SMILESS_EINVAL, "begin > end");
+    const int n_shards = a->n_shards <= 0 ? 1 : a->n_shards;
+    const int shard = a->n_shards <= 0 ? 0 : a->shard;
+    if ((rc = ensure_device(ctx))) return rc;
+    CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+    if ((rc = upload_tables(ctx))) return rc;
+    cudaStream_t st = ctx->stream;
+    CK(cudaEventRecord(ctx->ev[0], st), "event");
+    int launches = 0;
+
+    const i64 *d_arr = nullptr;
+    if ((rc = stage_arrivals(ctx, a, &d_arr))) return rc;
+
+    const RangePlan rp = range_plan(ctx, a);
+    const i64 n_steps = a->n_arrivals - 1;
+    const i64 n_off = std::max<i64>(4, (n_steps + rp.K - 1) / rp.K * rp.K);
+    const size_t tsz = rp.time64 ? 8 : 4;
+    CK(ctx->dOff.ensure((size_t)n_off * tsz), "cudaMalloc offsets");
+    CK(cudaMemsetAsync(ctx->dErr.p, 0, sizeof(int), st), "memset");
+    CK(cudaMemsetAsync(ctx->dRes.p, 0xff, sizeof(ResBlock), st), "memset");
+    int e = smiless_dev_prep_offsets(d_arr, a->n_arrivals, rp.d_cap, rp.K, rp.time64 ? 1 : 0, ctx->dOff.p, n_off,
+                                     ctx->dScal.p, ctx->dErr.p, st);
+    if (e) return cuda_fail(ctx, (cudaError_t)e, "prep_offsets launch");
+    ++launches;
+
+    const bool single = a->n_fixed == ctx->N;    // nothing left to search: one candidate
+    double eval_ms = 0.0;
+    u64 n_decided = 0, n_full = 0;
+    if (!single && ce > cb) {
+        JitKernel *jk = nullptr;
+        if ((rc = get_kernel(ctx, a, rp, n_off, &jk))) return rc;
+        const int W = a->n_windows;
+        const u64 ub = cb / (u64)W, ue = (ce + (u64)W - 1) / (u64)W;
+        const u64 U = ue - ub;
+        const u64 n_chunks = (U + kChunkUnits - 1) / kChunkUnits;
+        const u64 my_chunks = n_chunks > (u64)shard ? (n_chunks - 1 - (u64)shard) / (u64)n_shards + 1 : 0;
+        const u64 claims_total = my_chunks * (u64)kChunkUnits;
+        const int grid = jk->blocks_per_sm * ctx->n_sms;
+        CK(ctx->dBlk.ensure((size_t)grid * 2), "cudaMalloc");
+        CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid * 16, st), "memset");
+        CK(cudaMemsetAsync(ctx->dStats.p, 0, 16, st), "memset");
+        PlanParamsHost pp;
+        memset(&pp, 0, sizeof pp);
+        pp.tabI = ctx->dI.p;
+        pp.tabT = ctx->dT.p;
+        pp.tabU = ctx->dU.p;
+        pp.off = ctx->dOff.p;
+        pp.scal = ctx->dScal.p;
+        pp.counter = ctx->dCounter.p;
+        pp.stats = ctx->dStats.p;
+        pp.blk_best = ctx->dBlk.p;
+        pp.unit_begin = ub;
+        pp.unit_end = ue;
+        pp.cand_begin = cb;
+        pp.cand_end = ce;
+        pp.n_steps = n_steps;
+        pp.n_off = n_off;
+        pp.sumM = ctx->sumM;
+        pp.sla = (int)a->sla_us;
+        pp.prune = (a->flags & SMILESS_FLAG_NO_PRUNE) ? 0 : 1;
+        pp.shard = shard;
+        pp.n_shards = n_shards;
+        pp.chunk_units = kChunkUnits;
+        for (int k = 0; k < a->n_fixed; ++k) pp.fixed[k] = a->fixed_digits[k];
+        // split very large ranges into several launches (bounded kernel duration)
+        const u64 claims_per_launch = (u64)1 << 28;  // units (x W candidates)
+        CK(cudaEventRecord(ctx->ev[1], st), "event");
+        for (u64 q0 = 0; q0 < claims_total; q0 += claims_per_launch) {
+            const u64 q1 = std::min(claims_total, q0 + claims_per_launch);
+            CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+            pp.claims_begin = q0;
+            pp.claims_end = q1;
+            void *args[] = {&pp};
+            CUresult r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
+                                               (CUstream)st, args, nullptr);
+            if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
+            ++launches;
+        }
+        CK(cudaEventRecord(ctx->ev[2], st), "event");
+        e = smiless_dev_reduce_best(ctx->dBlk.p, grid, ctx->dRes.p, st);
+        if (e) return cuda_fail(ctx, (cudaError_t)e, "reduce launch");
+        ++launches;
+        CK(cudaMemcpyAsync(&ctx->dRes.p->stats[0], ctx->dStats.p, 16, cudaMemcpyDeviceToDevice, st), "D2D stats");
+    } else if (single && ce > cb) {
+        // the space is the single candidate of the pinned digits: index 0
+        CK(cudaMemsetAsync(&ctx->dRes.p->best_c, 0, 16, st), "memset");
+        CK(cudaEventRecord(ctx->ev[1], st), "event");
+        CK(cudaEventRecord(ctx->ev[2], st), "event");
+    } else {
+        CK(cudaEventRecord(ctx->ev[1], st), "event");
+        CK(cudaEventRecord(ctx->ev[2], st), "event");
+    }
+    // a10: exact int64 re-evaluation of the winner (also decodes its digits)
+    ExactParams ep;
+    fill_exact_params(ctx, a, d_arr, ep);
+    ep.n = 1;
+    ep.res = ctx->dRes.p;
+    ep.idx_from_res = 1;
+    e = smiless_dev_eval_exact(&ep, st);
+    if (e) return cuda_fail(ctx, (cudaError_t)e, "eval_exact launch");
+    ++launches;
+    CK(cudaMemcpyAsync(&ctx->dRes.p->err, ctx->dErr.p, sizeof(int), cudaMemcpyDeviceToDevice, st), "D2D err");
+    CK(cudaMemcpyAsync(ctx->hRes, ctx->dRes.p, sizeof(ResBlock), cudaMemcpyDeviceToHost, st), "D2H result");
+    CK(cudaEventRecord(ctx->ev[3], st), "event");
+    CK(cudaStreamSynchronize(st), "plan");
+    float ms = 0.f, tot = 0.f;
+    cudaEventElapsedTime(&ms, ctx->ev[1], ctx->ev[2]);
+    cudaEventElapsedTime(&tot, ctx->ev[0], ctx->ev[3]);
+    eval_ms = ms;
+
+    const ResBlock &h = *ctx->hRes;
+    if (h.err & 1) return fail(ctx, SMILESS_EINVAL, "arrivals must be non-decreasing");
+    if (h.err & 2) return fail(ctx, SMILESS_EINVAL, "arrival times out of range (|r| >= 2^62)");
+    if (!single && ce > cb) {
+        n_decided = h.stats[0];
+        n_full = h.stats[1];
+    } else if (single && ce > cb) {
+        n_decided = n_full = 1;
+    }
+    const bool found = h.best_i != ~0ull && h.feasible == 1;
+    if (!single && h.best_i != ~0ull && h.feasible != 1)
+        return fail(ctx, SMILESS_ECUDA, "internal: evaluator winner %llu not feasible on exact re-evaluation",
+                    (unsigned long long)h.best_i);
+    if (found && !single) {
+        double c;
+        memcpy(&c, &h.best_c, 8);
+        if (c != h.cost)
+            return fail(ctx, SMILESS_ECUDA, "internal: evaluator cost %.17g != exact %.17g for index %llu", c, h.cost,
+                        (unsigned long long)h.best_i);
+    }
+    memset(res, 0, sizeof *res);
+    res->n_decided = n_decided;
+    res->n_full_evals = n_full;
+    res->eval_kernel_ms = eval_ms;
+    res->total_device_ms = tot;
+    res->int64_path = rp.time64 ? 1 : 0;
+    res->launches = launches;
+    if (!found) {
+        res->index = ~0ull;
+        res->cost = HUGE_VAL;
+        res->max_latency_us = -1;
+        for (int k = 0; k < ctx->N; ++k) {
+            if (config_out) config_out[k] = -1;
+            if (window_out) window_out[k] = -1;
+        }
+        return SMILESS_INFEASIBLE;
+    }
+    res->index = h.best_i;
+    res->cost = h.cost;
+    res->max_latency_us = h.maxlat;
+    for (int k = 0; k < ctx->N; ++k) {
+        if (config_out) config_out[k] = h.cfg[k];
+        if (window_out) window_out[k] = h.win[k];
+    }
+    return SMILESS_OK;
+}
+
+// ---- introspection (build checks, SASS inspection, tests) ---------------------------------
+int smiless_kernel_source(smiless_ctx *ctx, const smiless_plan_args *a, char *buf, size_t cap, size_t *len) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->err.clear();
+    int rc = validate_args(ctx, a, false);
+    if (rc) return rc;
+    const RangePlan rp = range_plan(ctx, a);
+    const i64 n_steps = a->n_arrivals - 1;
+    const i64 n_off = std::max<i64>(4, (n_steps + rp.K - 1) / rp.K * rp.K);
+    const bool off_smem = smem_bytes(ctx, a, rp, n_off, true) <= 227 * 1024;
+    std::string s = full_source(ctx, a, rp, off_smem, 1);
+    if (len) *len = s.size() + 1;
+    if (buf && cap) {
+        const size_t n = std::min(cap - 1, s.size());
+        memcpy(buf, s.data(), n);
+        buf[n] = '\0';
+    }
+    return SMILESS_OK;
+}
+
+int smiless_jit_compile(smiless_ctx *ctx, const smiless_plan_args *a, char *log, size_t logcap, size_t *cubin_size) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->err.clear();
+    int rc = validate_args(ctx, a, false);
+    if (rc) return rc;
+    const RangePlan rp = range_plan(ctx, a);
+    const i64 n_steps = a->n_arrivals - 1;
+    const i64 n_off = std::max<i64>(4, (n_steps + rp.K - 1) / rp.K * rp.K);
+    const bool off_smem = smem_bytes(ctx, a, rp, n_off, true) <= 227 * 1024;
+    std::vector<char> cubin;
+    std::string lg;
+    rc = nvrtc_compile(ctx, full_source(ctx, a, rp, off_smem, 1), cubin, lg);
+    if (log && logcap) {
+        const size_t n = std::min(logcap - 1, lg.size());
+        memcpy(log, lg.data(), n);
+        log[n] = '\0';
+    }
+    if (cubin_size) *cubin_size = cubin.size();
+    return rc;
+}
+
+}  // extern "C"

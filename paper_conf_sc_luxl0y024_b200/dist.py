@@ -1,0 +1,75 @@
+"""Multi-GPU driver: shard the candidate space across ranks, one exchange at the end.
+
+SURVEY 8(e): candidates are independent, so each rank (one process per GPU) plans the
+chunks c with c % world == rank (interleaved for balance under pruning) through the
+C ABI, then the ranks agree on the lexicographic (cost, index) minimum with two
+8-byte MIN all-reduces over NCCL/NVLink (cost bits of a non-negative double order like
+the double; then the index among ranks holding that cost).  No candidate data crosses
+GPUs.  The same code runs on the gloo backend for the CPU tests.
+"""
+from __future__ import annotations
+
+import struct
+from typing import Optional
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+INF_BITS = (1 << 63) - 1          # "no feasible candidate" key (above every finite cost's bits)
+NO_INDEX = (1 << 63) - 1
+
+
+def cost_bits(cost: Optional[float]) -> int:
+    if cost is None:
+        return INF_BITS
+    b = struct.unpack("<q", struct.pack("<d", float(cost)))[0]
+    assert b >= 0, "costs are non-negative"
+    return b
+
+
+def bits_cost(bits: int) -> Optional[float]:
+    if bits == INF_BITS:
+        return None
+    return struct.unpack("<d", struct.pack("<q", int(bits)))[0]
+
+
+def reduce_best(local_cost: Optional[float], local_index: Optional[int], local_latency: int,
+                n_decided: int, device, group=None):
+    """All-reduce the per-rank winners to the global lexicographic (cost, index) minimum.
+
+    Returns (cost or None, index or None, max_latency or -1, total decided)."""
+    kb = cost_bits(local_cost)
+    t = torch.tensor([kb], dtype=torch.int64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+    best_bits = int(t.item())
+    mine = local_cost is not None and kb == best_bits
+    v = torch.tensor([int(local_index) if mine else NO_INDEX], dtype=torch.int64, device=device)
+    dist.all_reduce(v, op=dist.ReduceOp.MIN, group=group)
+    best_index = int(v.item())
+    # one SUM: the (unique) owner contributes the winner's latency; everyone its decided count
+    s = torch.tensor([local_latency if (mine and local_index == best_index) else 0, int(n_decided)],
+                     dtype=torch.int64, device=device)
+    dist.all_reduce(s, op=dist.ReduceOp.SUM, group=group)
+    lat, dec = (int(v) for v in s.tolist())
+    if best_bits == INF_BITS:
+        return None, None, -1, dec
+    return bits_cost(best_bits), best_index, lat, dec
+
+
+def plan_distributed(planner, arrivals, sla_us, windows_us, group=None, device=None, **kw):
+    """Plan this rank's shard through the C ABI and reduce across ranks.
+
+    Returns (cost, index, max_latency, config, window, n_decided, local PlanResult)."""
+    rank = dist.get_rank(group)
+    world = dist.get_world_size(group)
+    if device is None:
+        device = torch.device("cuda", torch.cuda.current_device()) if torch.cuda.is_available() else "cpu"
+    r = planner.plan(arrivals, sla_us, windows_us, shard=rank, n_shards=world, **kw)
+    cost, index, lat, decided = reduce_best(r.cost if r.feasible else None, r.index, r.max_latency_us,
+                                            r.n_decided, device, group)
+    if index is None:
+        n = planner.n_funcs
+        return None, None, -1, np.full(n, -1, np.int32), np.full(n, -1, np.int32), decided, r
+    c, w = planner.decode(index, len(windows_us), kw.get("n_fixed", 0), kw.get("fixed_digits", ()))
+    return cost, index, lat, c, w, decided, r

@@ -1,0 +1,266 @@
+"""Thin Python binding of the C-ABI library (include/smiless.h) -- argument marshalling only.
+
+Every step of the hot path runs in libsmiless.so's CUDA kernels.  There is no CPU
+fallback: if the library cannot be loaded or the GPU is missing, calls raise
+SmilessError (the C side returns SMILESS_ECUDA / SMILESS_EJIT).
+"""
+from __future__ import annotations
+
+import ctypes
+import dataclasses
+import os
+from typing import Optional, Sequence, Tuple
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libsmiless.so")
+
+OK, INFEASIBLE = 0, 1
+EINVAL, ENOTTOPO, ERANGE, ESTATE, ECUDA, ENOMEM, EJIT = -1, -2, -3, -4, -5, -6, -7
+FLAG_NO_PRUNE, FLAG_ARRIVALS_ON_DEVICE, FLAG_FORCE_INT64 = 1, 2, 4
+_NAMES = {0: "OK", 1: "INFEASIBLE", -1: "EINVAL", -2: "ENOTTOPO", -3: "ERANGE", -4: "ESTATE",
+          -5: "ECUDA", -6: "ENOMEM", -7: "EJIT"}
+
+# every symbol include/smiless.h declares (checked by tests/test_abi.py)
+EXPORTS = ("smiless_create", "smiless_set_stream", "smiless_destroy", "smiless_last_error",
+           "smiless_load_dag", "smiless_load_profiles", "smiless_space_size", "smiless_plan",
+           "smiless_evaluate", "smiless_decode", "smiless_kernel_source", "smiless_jit_compile")
+
+
+class SmilessError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"{_NAMES.get(code, code)}: {msg}")
+        self.code = code
+
+
+class PlanArgs(ctypes.Structure):
+    _fields_ = [
+        ("arrivals_us", ctypes.c_void_p),
+        ("n_arrivals", ctypes.c_int64),
+        ("sla_us", ctypes.c_int64),
+        ("windows_us", ctypes.c_void_p),
+        ("n_windows", ctypes.c_int32),
+        ("n_fixed", ctypes.c_int32),
+        ("fixed_digits", ctypes.c_void_p),
+        ("begin", ctypes.c_uint64),
+        ("end", ctypes.c_uint64),
+        ("flags", ctypes.c_uint32),
+        ("shard", ctypes.c_int32),
+        ("n_shards", ctypes.c_int32),
+    ]
+
+
+class PlanResultC(ctypes.Structure):
+    _fields_ = [
+        ("index", ctypes.c_uint64),
+        ("cost", ctypes.c_double),
+        ("max_latency_us", ctypes.c_int64),
+        ("n_decided", ctypes.c_uint64),
+        ("n_full_evals", ctypes.c_uint64),
+        ("eval_kernel_ms", ctypes.c_double),
+        ("total_device_ms", ctypes.c_double),
+        ("int64_path", ctypes.c_int32),
+        ("launches", ctypes.c_int32),
+    ]
+
+
+@dataclasses.dataclass
+class PlanResult:
+    status: int                 # OK or INFEASIBLE
+    index: Optional[int]
+    cost: float
+    max_latency_us: int
+    config: np.ndarray
+    window: np.ndarray
+    n_decided: int
+    n_full_evals: int
+    eval_kernel_ms: float
+    total_device_ms: float
+    int64_path: bool
+    launches: int
+
+    @property
+    def feasible(self) -> bool:
+        return self.status == OK
+
+
+_lib = None
+
+
+def load_library(build_if_missing: bool = True):
+    """Load libsmiless.so (building it in-tree with nvcc when missing or stale)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if build_if_missing:
+        from . import build as _build
+        if _build.stale():
+            _build.build()
+    lib = ctypes.CDLL(LIB_PATH)
+    vp, i32, i64, u64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_uint64
+    lib.smiless_create.argtypes = [ctypes.POINTER(vp), ctypes.c_int, vp]
+    lib.smiless_set_stream.argtypes = [vp, vp]
+    lib.smiless_destroy.argtypes = [vp]
+    lib.smiless_destroy.restype = None
+    lib.smiless_last_error.argtypes = [vp]
+    lib.smiless_last_error.restype = ctypes.c_char_p
+    lib.smiless_load_dag.argtypes = [vp, i32, vp, vp]
+    lib.smiless_load_profiles.argtypes = [vp, vp, vp, vp, vp]
+    lib.smiless_space_size.argtypes = [vp, i32, i32, ctypes.POINTER(u64)]
+    lib.smiless_plan.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.POINTER(PlanResultC), vp, vp]
+    lib.smiless_evaluate.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i64, vp, vp, vp]
+    lib.smiless_decode.argtypes = [vp, i32, u64, ctypes.POINTER(PlanArgs), vp, vp]
+    lib.smiless_kernel_source.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.c_char_p, ctypes.c_size_t,
+                                          ctypes.POINTER(ctypes.c_size_t)]
+    lib.smiless_jit_compile.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.c_char_p, ctypes.c_size_t,
+                                        ctypes.POINTER(ctypes.c_size_t)]
+    for name in EXPORTS:
+        if name not in ("smiless_destroy", "smiless_last_error"):
+            getattr(lib, name).restype = ctypes.c_int
+    _lib = lib
+    return lib
+
+
+def _i32(a) -> np.ndarray:
+    return np.ascontiguousarray(np.asarray(a, dtype=np.int32))
+
+
+def _is_device_tensor(x) -> bool:
+    return hasattr(x, "is_cuda") and bool(getattr(x, "is_cuda"))
+
+
+class Planner:
+    """One smiless_ctx (one per host thread / GPU)."""
+
+    def __init__(self, device: int = 0, stream: Optional[int] = None):
+        self._lib = load_library()
+        self._ctx = ctypes.c_void_p()
+        rc = self._lib.smiless_create(ctypes.byref(self._ctx), int(device), ctypes.c_void_p(stream or 0))
+        if rc != OK:
+            raise SmilessError(rc, self._lib.smiless_last_error(None).decode())
+        self._keep = []
+        self.n_funcs = 0
+
+    def close(self):
+        if self._ctx:
+            self._lib.smiless_destroy(self._ctx)
+            self._ctx = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def _check(self, rc: int, allow=(OK,)) -> int:
+        if rc not in allow:
+            raise SmilessError(rc, self._lib.smiless_last_error(self._ctx).decode())
+        return rc
+
+    def set_stream(self, stream: int):
+        self._check(self._lib.smiless_set_stream(self._ctx, ctypes.c_void_p(stream)))
+
+    # ---- loads ---------------------------------------------------------------------------
+    def load_dag(self, pred_ptr: Sequence[int], pred_idx: Sequence[int]):
+        ptr = _i32(pred_ptr)
+        idx = _i32(pred_idx) if len(pred_idx) else np.zeros(1, np.int32)
+        n = int(ptr.shape[0] - 1)
+        self._check(self._lib.smiless_load_dag(self._ctx, n, ptr.ctypes.data,
+                                               idx.ctypes.data if len(pred_idx) else None))
+        self.n_funcs = n
+
+    def load_profiles(self, n_configs, exec_us, init_us, price_per_us):
+        m, e, t = _i32(n_configs), _i32(exec_us), _i32(init_us)
+        u = np.ascontiguousarray(np.asarray(price_per_us, dtype=np.float64))
+        self._check(self._lib.smiless_load_profiles(self._ctx, m.ctypes.data, e.ctypes.data, t.ctypes.data,
+                                                    u.ctypes.data))
+
+    # ---- args ----------------------------------------------------------------------------
+    def _args(self, arrivals, sla_us, windows_us, n_fixed=0, fixed_digits=(), begin=0, end=0, flags=0,
+              shard=0, n_shards=0):
+        keep = []
+        if _is_device_tensor(arrivals):
+            import torch
+            assert arrivals.dtype == torch.int64 and arrivals.is_contiguous()
+            ptr = arrivals.data_ptr()
+            n = int(arrivals.numel())
+            flags |= FLAG_ARRIVALS_ON_DEVICE
+            keep.append(arrivals)
+        else:
+            arr = np.ascontiguousarray(np.asarray(arrivals, dtype=np.int64))
+            keep.append(arr)
+            ptr, n = arr.ctypes.data, int(arr.shape[0])
+        win = _i32(windows_us)
+        fixed = _i32(list(fixed_digits) or [0])
+        keep += [win, fixed]
+        a = PlanArgs(arrivals_us=ptr, n_arrivals=n, sla_us=int(sla_us), windows_us=win.ctypes.data,
+                     n_windows=int(win.shape[0]), n_fixed=int(n_fixed),
+                     fixed_digits=fixed.ctypes.data if n_fixed else None, begin=int(begin), end=int(end),
+                     flags=int(flags), shard=int(shard), n_shards=int(n_shards))
+        return a, keep
+
+    # ---- API -----------------------------------------------------------------------------
+    def space_size(self, n_windows: int, n_fixed: int = 0) -> int:
+        out = ctypes.c_uint64()
+        self._check(self._lib.smiless_space_size(self._ctx, int(n_windows), int(n_fixed), ctypes.byref(out)))
+        return int(out.value)
+
+    def plan(self, arrivals, sla_us, windows_us, **kw) -> PlanResult:
+        a, keep = self._args(arrivals, sla_us, windows_us, **kw)
+        r = PlanResultC()
+        cfg = np.zeros(max(self.n_funcs, 1), np.int32)
+        win = np.zeros(max(self.n_funcs, 1), np.int32)
+        rc = self._check(self._lib.smiless_plan(self._ctx, ctypes.byref(a), ctypes.byref(r), cfg.ctypes.data,
+                                                win.ctypes.data), allow=(OK, INFEASIBLE))
+        del keep
+        return PlanResult(status=rc, index=None if rc == INFEASIBLE else int(r.index), cost=float(r.cost),
+                          max_latency_us=int(r.max_latency_us), config=cfg[:self.n_funcs],
+                          window=win[:self.n_funcs], n_decided=int(r.n_decided), n_full_evals=int(r.n_full_evals),
+                          eval_kernel_ms=float(r.eval_kernel_ms), total_device_ms=float(r.total_device_ms),
+                          int64_path=bool(r.int64_path), launches=int(r.launches))
+
+    def evaluate(self, idx, arrivals, sla_us, windows_us, **kw) -> Tuple[np.ndarray, np.ndarray, np.ndarray]:
+        a, keep = self._args(arrivals, sla_us, windows_us, **kw)
+        ix = np.ascontiguousarray(np.asarray(idx, dtype=np.uint64).reshape(-1))
+        n = int(ix.shape[0])
+        cost = np.zeros(n, np.float64)
+        lat = np.zeros(n, np.int64)
+        feas = np.zeros(n, np.uint8)
+        self._check(self._lib.smiless_evaluate(self._ctx, ctypes.byref(a), ix.ctypes.data, n, cost.ctypes.data,
+                                               lat.ctypes.data, feas.ctypes.data))
+        del keep
+        return cost, lat, feas.astype(bool)
+
+    def decode(self, index: int, n_windows: int, n_fixed: int = 0, fixed_digits=()):
+        fixed = _i32(list(fixed_digits) or [0])
+        a = PlanArgs(n_fixed=int(n_fixed), fixed_digits=fixed.ctypes.data if n_fixed else None)
+        c = np.zeros(self.n_funcs, np.int32)
+        w = np.zeros(self.n_funcs, np.int32)
+        self._check(self._lib.smiless_decode(self._ctx, int(n_windows), int(index), ctypes.byref(a),
+                                             c.ctypes.data, w.ctypes.data))
+        return c, w
+
+    def kernel_source(self, arrivals, sla_us, windows_us, **kw) -> str:
+        a, keep = self._args(arrivals, sla_us, windows_us, **kw)
+        n = ctypes.c_size_t()
+        self._check(self._lib.smiless_kernel_source(self._ctx, ctypes.byref(a), None, 0, ctypes.byref(n)))
+        buf = ctypes.create_string_buffer(n.value)
+        self._check(self._lib.smiless_kernel_source(self._ctx, ctypes.byref(a), buf, n.value, ctypes.byref(n)))
+        return buf.value.decode()
+
+    def jit_compile(self, arrivals, sla_us, windows_us, **kw) -> Tuple[str, int]:
+        """NVRTC-compile the specialised evaluator (no GPU needed); returns (ptxas log, cubin bytes)."""
+        a, keep = self._args(arrivals, sla_us, windows_us, **kw)
+        log = ctypes.create_string_buffer(1 << 16)
+        n = ctypes.c_size_t()
+        self._check(self._lib.smiless_jit_compile(self._ctx, ctypes.byref(a), log, 1 << 16, ctypes.byref(n)))
+        return log.value.decode(), int(n.value)
+
+
+def planner_for(problem, device: int = 0, stream: Optional[int] = None) -> Planner:
+    """Planner with a workloads.Problem-like object's DAG and profiles loaded."""
+    p = Planner(device, stream)
+    p.load_dag(problem.pred_ptr, problem.pred_idx)
+    p.load_profiles(problem.n_configs, problem.exec_us, problem.init_us, problem.price_per_us)
+    return p

@@ -1,0 +1,180 @@
+"""C-ABI boundary checks that need no GPU (-m "not gpu"): the library loads, exports
+every symbol include/smiless.h declares, validates arguments (T6), decodes indices,
+and NVRTC specialises the evaluator for every BASELINE config (sm_100a, no spills).
+"""
+import ctypes
+import re
+import os
+
+import numpy as np
+import pytest
+
+import workloads as W
+from paper_conf_sc_luxl0y024_b200 import smiless as S
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_symbols():
+    txt = open(os.path.join(ROOT, "include", "smiless.h")).read()
+    return sorted(set(re.findall(r"SMILESS_API\s+[\w\s\*]+?\b(smiless_\w+)\s*\(", txt)))
+
+
+def test_library_exports_every_header_symbol():
+    lib = S.load_library()
+    syms = header_symbols()
+    assert len(syms) >= 10
+    assert sorted(S.EXPORTS) == syms
+    for name in syms:
+        assert hasattr(lib, name), name
+
+
+def test_library_has_no_cpu_fallback_dependency():
+    """The product library links no oracle code and no CPU evaluator."""
+    import subprocess
+    out = subprocess.run(["nm", "-D", "--defined-only", S.LIB_PATH], capture_output=True, text=True).stdout
+    assert "oracle" not in out
+    src = open(os.path.join(ROOT, "paper_conf_sc_luxl0y024_b200", "smiless.py")).read()
+    assert "oracle" not in src.lower().replace("no cpu fallback", "")
+
+
+def planner(prob=None):
+    prob = prob or W.make_config("C1")
+    return S.planner_for(prob), prob
+
+
+def test_create_rejects_bad_args():
+    lib = S.load_library()
+    ctx = ctypes.c_void_p()
+    assert lib.smiless_create(None, 0, None) == S.EINVAL
+    assert lib.smiless_create(ctypes.byref(ctx), -1, None) == S.EINVAL
+    assert b"cuda_device" in lib.smiless_last_error(None)
+
+
+def test_load_dag_validation():
+    pl = S.Planner()
+    with pytest.raises(S.SmilessError) as e:
+        pl.load_dag([0, 0, 1], [1])          # function 1 lists itself
+    assert e.value.code == S.ENOTTOPO
+    with pytest.raises(S.SmilessError) as e:
+        pl.load_dag([0, 1, 1], [0])          # function 0 lists 0 -> not topological
+    assert e.value.code == S.ENOTTOPO
+    with pytest.raises(S.SmilessError) as e:
+        pl.load_dag([0, 0, 2], [0, 0])       # duplicate predecessor
+    assert e.value.code == S.EINVAL
+    with pytest.raises(S.SmilessError) as e:
+        pl.load_dag([0, 0, 1], [5])
+    assert e.value.code == S.EINVAL
+    with pytest.raises(S.SmilessError) as e:
+        pl.load_dag([1, 1], [])
+    assert e.value.code == S.EINVAL
+    with pytest.raises(S.SmilessError) as e:
+        pl.load_dag([0] * 40, [])            # > SMILESS_MAX_FUNCS
+    assert e.value.code == S.EINVAL
+    pl.load_dag([0, 0], [])                  # single function: ok
+
+
+def test_call_order_estate():
+    pl = S.Planner()
+    with pytest.raises(S.SmilessError) as e:
+        pl.load_profiles([1], [1], [1], [1.0])
+    assert e.value.code == S.ESTATE
+    pl.load_dag([0, 0], [])
+    with pytest.raises(S.SmilessError) as e:
+        pl.plan([0, 1], 10, [0])
+    assert e.value.code == S.ESTATE
+    with pytest.raises(S.SmilessError) as e:
+        pl.space_size(1)
+    assert e.value.code == S.ESTATE
+
+
+def test_profile_validation():
+    pl = S.Planner()
+    pl.load_dag([0, 0, 1], [0])
+    for bad in [dict(n_configs=[0, 1]), dict(exec_us=[-1, 1]), dict(init_us=[1 << 29, 1]),
+                dict(price_per_us=[float("nan"), 1.0]), dict(price_per_us=[-1.0, 1.0])]:
+        kw = dict(n_configs=[1, 1], exec_us=[1, 1], init_us=[1, 1], price_per_us=[1.0, 1.0])
+        kw.update(bad)
+        with pytest.raises(S.SmilessError) as e:
+            pl.load_profiles(**kw)
+        assert e.value.code == S.EINVAL
+
+
+def test_plan_argument_validation_before_any_gpu_work():
+    pl, p = planner()
+    ok = dict(arrivals=p.arrivals_us, sla_us=p.sla_us, windows_us=p.windows_us)
+    cases = [
+        (dict(windows_us=[0, 0, 5]), S.EINVAL),                    # not strictly increasing
+        (dict(windows_us=[-1, 5]), S.EINVAL),
+        (dict(windows_us=[0, 1 << 29]), S.EINVAL),
+        (dict(windows_us=list(range(40))), S.EINVAL),               # W > SMILESS_MAX_WINDOWS
+        (dict(sla_us=-1), S.EINVAL),
+        (dict(sla_us=1 << 29), S.EINVAL),
+        (dict(arrivals=[5, 3, 9]), S.EINVAL),                       # decreasing arrivals
+        (dict(arrivals=[]), S.EINVAL),
+        (dict(arrivals=[0, 1 << 62]), S.EINVAL),
+        (dict(n_fixed=4), S.EINVAL),
+        (dict(n_fixed=1, fixed_digits=[16]), S.EINVAL),             # digit >= M*W
+        (dict(n_shards=2, shard=2), S.EINVAL),
+    ]
+    for over, code in cases:
+        kw = dict(ok)
+        kw.update(over)
+        with pytest.raises(S.SmilessError) as e:
+            pl.plan(**kw)
+        assert e.value.code == code, over
+
+
+def test_space_size_and_erange():
+    pl, p = planner(W.make_config("C5", n_arrivals=10))
+    with pytest.raises(S.SmilessError) as e:
+        pl.space_size(16)                    # 128^10 = 2^70 > 2^63-1
+    assert e.value.code == S.ERANGE
+    assert pl.space_size(16, n_fixed=2) == 128 ** 8
+    with pytest.raises(S.SmilessError):
+        pl.space_size(16, n_fixed=1)         # 2^63 > 2^63-1
+    with pytest.raises(S.SmilessError) as e:
+        pl.plan(p.arrivals_us, p.sla_us, p.windows_us)
+    assert e.value.code == S.ERANGE
+
+
+def test_decode_matches_numpy_unravel():
+    pl, p = planner(W.make_config("C2", n_arrivals=10))
+    Wn = len(p.windows_us)
+    shape = tuple(int(m) * Wn for m in p.n_configs)
+    rng = np.random.default_rng(0)
+    for idx in rng.integers(0, pl.space_size(Wn), size=200):
+        c, w = pl.decode(int(idx), Wn)
+        d = np.unravel_index(int(idx), shape)
+        assert (c == np.array(d) // Wn).all() and (w == np.array(d) % Wn).all()
+    c, w = pl.decode(7, Wn, n_fixed=2, fixed_digits=[3, 9])
+    assert c[:2].tolist() == [0, 1] and w[:2].tolist() == [3, 1]
+    with pytest.raises(S.SmilessError) as e:
+        pl.decode(pl.space_size(Wn), Wn)
+    assert e.value.code == S.ERANGE
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C3", "C4", "C5"])
+def test_nvrtc_specialises_every_config_for_sm100a(name):
+    """NVRTC compiles the DAG-specialised evaluator for sm_100a with no local memory."""
+    p = W.make_config(name, n_arrivals=100)
+    pl = S.planner_for(p)
+    nf = 3 if name == "C5" else 0
+    log, n = pl.jit_compile(p.arrivals_us, p.sla_us, p.windows_us, n_fixed=nf, fixed_digits=[0] * nf)
+    assert n > 0
+    assert "0 bytes stack frame, 0 bytes spill stores, 0 bytes spill loads" in log, log
+    src = pl.kernel_source(p.arrivals_us, p.sla_us, p.windows_us, n_fixed=nf, fixed_digits=[0] * nf)
+    assert "#define SM_N %d" % p.n_funcs in src and "smiless_plan_kernel" in src
+
+
+def test_int64_path_selected_when_int32_range_fails():
+    p = W.make_config("C1", n_arrivals=20)
+    p = p.replace(windows_us=np.array([0, (1 << 29) - 1], np.int32), init_us=np.full_like(p.init_us, (1 << 29) - 1))
+    pl = S.planner_for(p)
+    src = pl.kernel_source(p.arrivals_us, p.sla_us, p.windows_us)
+    assert "#define SM_TIME64 1" in src
+    log, n = pl.jit_compile(p.arrivals_us, p.sla_us, p.windows_us)
+    assert n > 0
+    p2 = W.make_config("C1", n_arrivals=20)
+    src2 = S.planner_for(p2).kernel_source(p2.arrivals_us, p2.sla_us, p2.windows_us)
+    assert "#define SM_TIME64 0" in src2

@@ -1,0 +1,283 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle (-m gpu).
+
+Bar (BASELINE.json north star): chosen index / config / window bit-exact with
+lowest-index tie-break, latencies exact in integer microseconds, cost within 1e-9
+relative in fp64 -- the design reaches 0 ulp, so costs are compared bit for bit and
+the 1e-9 bound is asserted as well.
+"""
+import numpy as np
+import pytest
+
+import workloads as W
+from oracle import OracleProblem
+from paper_conf_sc_luxl0y024_b200 import smiless as S
+
+pytestmark = pytest.mark.gpu
+
+COST_RTOL = 1e-9
+
+
+def plan_both(p, **kw):
+    pl = S.planner_for(p)
+    g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, **kw)
+    nf = kw.get("n_fixed", 0)
+    o = OracleProblem(p, n_fixed=nf, fixed_digits=kw.get("fixed_digits", ()))
+    ref = o.plan(begin=kw.get("begin", 0), end=kw.get("end", 0))
+    return pl, g, o, ref
+
+
+def assert_same_plan(g, ref, o):
+    if ref is None:
+        assert g.status == S.INFEASIBLE and g.index is None and g.max_latency_us == -1
+        assert (g.config == -1).all() and (g.window == -1).all()
+        return
+    assert g.status == S.OK
+    assert g.index == ref[0]
+    assert g.cost == ref[1] and abs(g.cost - ref[1]) <= COST_RTOL * abs(ref[1])
+    assert g.max_latency_us == ref[2]
+    c, w = o.decode(ref[0])
+    assert g.config.tolist() == c.tolist() and g.window.tolist() == w.tolist()
+
+
+def assert_same_eval(gc, gl, gf, oc, ol, of):
+    assert (gf == of).all()
+    assert (gl == ol).all()
+    assert np.array_equal(gc.view(np.uint64), oc.view(np.uint64))
+
+
+# ---------------------------------------------------------------------------------------
+# C1 (configs[0]): every candidate, and the plan, in every mode
+# ---------------------------------------------------------------------------------------
+
+def test_c1_evaluate_every_candidate():
+    p = W.make_config("C1")
+    pl = S.planner_for(p)
+    idx = np.arange(4096, dtype=np.uint64)
+    gc, gl, gf = pl.evaluate(idx, p.arrivals_us, p.sla_us, p.windows_us)
+    oc, ol, of = OracleProblem(p).evaluate(idx)
+    assert_same_eval(gc, gl, gf, oc, ol, of)
+    assert 0 < of.sum() < 4096
+
+
+@pytest.mark.parametrize("flags", [0, S.FLAG_NO_PRUNE, S.FLAG_FORCE_INT64, S.FLAG_NO_PRUNE | S.FLAG_FORCE_INT64])
+@pytest.mark.parametrize("sla", [300_000, 1_000_000, 1_500_000, 2_000_000, 3_000_000, 10_000_000])
+def test_c1_plan(flags, sla):
+    p = W.make_config("C1").replace(sla_us=sla)
+    pl, g, o, ref = plan_both(p, flags=flags)
+    assert_same_plan(g, ref, o)
+    assert g.n_decided == 4096
+    if flags & S.FLAG_NO_PRUNE:
+        assert g.n_full_evals == 4096
+    assert g.int64_path == bool(flags & S.FLAG_FORCE_INT64)
+
+
+def test_c1_ranges_and_shards_compose():
+    """[begin, end) sub-ranges (misaligned with W) and interleaved shards give the
+    same winner as the full range after a lexicographic (cost, index) min."""
+    p = W.make_config("C1")
+    pl = S.planner_for(p)
+    o = OracleProblem(p)
+    for b, e in [(0, 4096), (1, 4095), (7, 9), (1000, 3001), (4095, 4096), (5, 5)]:
+        g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, begin=b, end=e)
+        assert_same_plan(g, o.plan(begin=b, end=e), o)
+        assert g.n_decided == e - b
+    full = pl.plan(p.arrivals_us, p.sla_us, p.windows_us)
+    for n in (2, 3, 8):
+        parts = [pl.plan(p.arrivals_us, p.sla_us, p.windows_us, shard=s, n_shards=n) for s in range(n)]
+        assert sum(r.n_decided for r in parts) == 4096
+        best = min((r.cost, r.index) for r in parts if r.feasible)
+        assert best == (full.cost, full.index)
+
+
+def test_arrivals_on_device_tensor():
+    import torch
+    p = W.make_config("C1")
+    pl = S.planner_for(p)
+    host = pl.plan(p.arrivals_us, p.sla_us, p.windows_us)
+    dev = torch.as_tensor(p.arrivals_us).cuda()
+    d = pl.plan(dev, p.sla_us, p.windows_us)
+    assert (d.index, d.cost, d.max_latency_us) == (host.index, host.cost, host.max_latency_us)
+    bad = dev.clone()
+    bad[5] = bad[4] - 1
+    with pytest.raises(S.SmilessError) as e:
+        pl.plan(bad, p.sla_us, p.windows_us)
+    assert e.value.code == S.EINVAL
+
+
+# ---------------------------------------------------------------------------------------
+# Full-size configs: sampled exact evaluation at J = 10^4
+# ---------------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("name,nf", [("C2", 0), ("C3", 0), ("C5", 2)])
+def test_full_size_sampled_evaluate(name, nf):
+    p = W.make_config(name)
+    rng = np.random.default_rng(5)
+    fixed = [int(rng.integers(0, p.n_configs[k] * len(p.windows_us))) for k in range(nf)]
+    pl = S.planner_for(p)
+    space = pl.space_size(len(p.windows_us), nf)
+    idx = rng.integers(0, space, size=96, dtype=np.uint64)
+    kw = dict(n_fixed=nf, fixed_digits=fixed)
+    g = pl.evaluate(idx, p.arrivals_us, p.sla_us, p.windows_us, **kw)
+    r = OracleProblem(p, n_fixed=nf, fixed_digits=fixed).evaluate(idx)
+    assert_same_eval(*g, *r)
+
+
+# ---------------------------------------------------------------------------------------
+# Plan parity on oracle-sized sub-spaces of the real configs (pinned leading digits)
+# ---------------------------------------------------------------------------------------
+
+FAST = {"C2": 15, "C3": 11, "C4": 7, "C5": 7}   # GPU-100% config index per grid
+
+
+@pytest.mark.parametrize("name,J", [("C2", 200), ("C3", 150), ("C4", 100), ("C5", 120)])
+def test_plan_parity_on_subspaces(name, J):
+    p = W.make_config(name, n_arrivals=J)
+    Wn = len(p.windows_us)
+    n = p.n_funcs
+    rng = np.random.default_rng(11)
+    checked_feasible = 0
+    for trial in range(4):
+        nf = n - 2
+        fixed = []
+        for k in range(nf):
+            c = FAST[name] if rng.random() < 0.7 else int(rng.integers(0, p.n_configs[k]))
+            w = 0 if rng.random() < 0.6 else int(rng.integers(0, Wn))
+            fixed.append(c * Wn + w)
+        for sla in (p.sla_us, 4_000_000):
+            q = p.replace(sla_us=sla)
+            for flags in (0, S.FLAG_NO_PRUNE):
+                pl, g, o, ref = plan_both(q, n_fixed=nf, fixed_digits=fixed, flags=flags)
+                assert_same_plan(g, ref, o)
+                checked_feasible += ref is not None
+    assert checked_feasible > 0
+
+
+# ---------------------------------------------------------------------------------------
+# Random DAGs: exhaustive plan parity, ragged configs, edge cases
+# ---------------------------------------------------------------------------------------
+
+def test_random_dags_exhaustive_plan_parity():
+    rng = np.random.default_rng(2024)
+    n_checked = 0
+    for t in range(120):
+        n = int(rng.integers(1, 7))
+        p = W.random_problem(rng, n, 4, int(rng.integers(1, 6)), int(rng.integers(1, 80)))
+        if p.space_size() > 20000:
+            continue
+        flags = int(rng.choice([0, S.FLAG_NO_PRUNE, S.FLAG_FORCE_INT64]))
+        pl, g, o, ref = plan_both(p, flags=flags)
+        assert_same_plan(g, ref, o)
+        idx = rng.integers(0, p.space_size(), size=64, dtype=np.uint64)
+        assert_same_eval(*pl.evaluate(idx, p.arrivals_us, p.sla_us, p.windows_us), *o.evaluate(idx))
+        n_checked += 1
+    assert n_checked > 60
+
+
+@pytest.mark.parametrize("J", [1, 2, 3, 4, 5, 63, 64, 65, 127, 129, 257])
+def test_horizon_edges_and_ragged_tail(J):
+    """J = 1 (no steps), J - 1 below / at / above the chunk length and its multiples."""
+    rng = np.random.default_rng(J)
+    p = W.random_problem(rng, 4, 3, 3, J, sla_us=40_000)
+    pl, g, o, ref = plan_both(p)
+    assert_same_plan(g, ref, o)
+    pl, g, o, ref = plan_both(p, flags=S.FLAG_NO_PRUNE)
+    assert_same_plan(g, ref, o)
+
+
+def test_ties_go_to_lowest_index():
+    """Identical profiles for every config and zero prices: every candidate costs 0;
+    the winner must be the lowest feasible index."""
+    rng = np.random.default_rng(3)
+    p = W.random_problem(rng, 3, 3, 3, 20, sla_us=10**8)
+    p = p.replace(price_per_us=np.zeros_like(p.price_per_us))
+    pl, g, o, ref = plan_both(p)
+    assert ref[0] == 0 and g.index == 0 and g.cost == 0.0
+    p2 = p.replace(price_per_us=np.ones_like(p.price_per_us) / 1024)
+    pl, g, o, ref = plan_both(p2)
+    assert_same_plan(g, ref, o)
+
+
+def test_single_function_and_all_sources():
+    rng = np.random.default_rng(4)
+    for preds in ([[]], [[], []], [[], [], [], []]):
+        base = W.random_problem(rng, len(preds), 4, 4, 40)
+        ptr, idx = W.csr_from_preds(preds)
+        p = base.replace(pred_ptr=ptr, pred_idx=idx)
+        pl, g, o, ref = plan_both(p)
+        assert_same_plan(g, ref, o)
+
+
+def test_windows_without_keepalive_and_single_window():
+    rng = np.random.default_rng(6)
+    p = W.random_problem(rng, 3, 3, 4, 50)
+    p = p.replace(windows_us=np.array([700, 2500, 9000], np.int32))
+    pl, g, o, ref = plan_both(p)
+    assert_same_plan(g, ref, o)
+    p = p.replace(windows_us=np.array([0], np.int32))
+    pl, g, o, ref = plan_both(p)
+    assert_same_plan(g, ref, o)
+
+
+def test_fully_pinned_and_empty_ranges():
+    p = W.make_config("C1", n_arrivals=50)
+    pl = S.planner_for(p)
+    o = OracleProblem(p, n_fixed=3, fixed_digits=[15, 3, 0])
+    g = pl.plan(p.arrivals_us, 10**8 - 1, p.windows_us, n_fixed=3, fixed_digits=[15, 3, 0])
+    assert g.index == 0
+    c, l, f = o.evaluate([0])
+    assert g.cost == c[0] and g.max_latency_us == l[0]
+    g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, begin=100, end=100)
+    assert g.status == S.INFEASIBLE and g.n_decided == 0
+
+
+def test_large_gaps_exercise_clamp_and_int64_path_agree():
+    """Gaps far above d_cap (clamped on the int32 path) and the int64 path give the
+    oracle's answer; the natural int64 path (int32 range rule fails) as well."""
+    rng = np.random.default_rng(8)
+    for t in range(10):
+        p = W.random_problem(rng, 4, 3, 3, 60)
+        gaps = np.diff(p.arrivals_us, prepend=0)
+        gaps[rng.random(len(gaps)) < 0.3] = int(rng.integers(10**9, 10**12))
+        p = p.replace(arrivals_us=np.cumsum(gaps).astype(np.int64))
+        for flags in (0, S.FLAG_FORCE_INT64):
+            pl, g, o, ref = plan_both(p, flags=flags)
+            assert_same_plan(g, ref, o)
+    p = W.random_problem(rng, 3, 2, 3, 30, time_scale=10**7 // 8)
+    p = p.replace(windows_us=np.array([0, 1 << 28, (1 << 29) - 1], np.int32),
+                  init_us=np.minimum(p.init_us.astype(np.int64) * 8, (1 << 29) - 1).astype(np.int32),
+                  sla_us=(1 << 29) - 1)
+    pl, g, o, ref = plan_both(p)
+    assert g.int64_path
+    assert_same_plan(g, ref, o)
+
+
+# ---------------------------------------------------------------------------------------
+# The bench launch configuration at full size (C2, J = 10^4, 2^28-candidate slice)
+# ---------------------------------------------------------------------------------------
+
+def test_bench_configuration_full_size_properties():
+    """bench.py's step: C2 at J = 10^4, functions 0/1 pinned, 2^28 candidates, no pruning.
+    The oracle cannot walk 2^28 x 10^4 x 6 steps, so we check (a) the winner on the
+    oracle (cost bits, latency, feasibility), (b) no sampled feasible candidate beats it
+    (lexicographic), (c) the pruned run returns the same winner, (d) the exact plan of
+    the winner's own 2^14-candidate neighbourhood on the oracle contains it as OPT."""
+    import bench
+    p, kw = bench.workload("C2")
+    pl = S.planner_for(p)
+    full = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=S.FLAG_NO_PRUNE, **kw)
+    assert full.n_full_evals == full.n_decided == pl.space_size(len(p.windows_us), kw["n_fixed"])
+    o = OracleProblem(p, **kw)
+    pruned = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, **kw)
+    assert (pruned.index, pruned.cost) == (full.index, full.cost)
+    if full.feasible:
+        c, l, f = o.evaluate([full.index])
+        assert f[0] and c[0] == full.cost and l[0] == full.max_latency_us
+        lo = full.index - full.index % (1 << 14)
+        ref = o.plan(begin=lo, end=lo + (1 << 14))
+        assert ref[0] == full.index and ref[1] == full.cost
+    rng = np.random.default_rng(9)
+    idx = rng.integers(0, full.n_decided, size=256, dtype=np.uint64)
+    c, l, f = o.evaluate(idx)
+    for i in range(len(idx)):
+        if f[i]:
+            assert full.feasible and (full.cost, full.index) <= (c[i], int(idx[i]))
