@@ -374,7 +374,8 @@ RangePlan range_plan(const smiless_ctx *ctx, const smiless_plan_args *a) {
     if (a->flags & SMILESS_FLAG_FORCE_INT64) return rp;
     const i64 LIM = 0x7fffffffll;
     for (int K : {64, 32, 16, 8, 4}) {
-        const i64 bound = (i64)K * d_cap + sla + (i64)ctx->N * (ctx->Tmax + ctx->Imax) + wmax + ctx->Tmax;
+        const i64 bound = (i64)K * d_cap + sla + (i64)ctx->N * (ctx->Tmax + ctx->Imax) + wmax + ctx->Tmax +
+                          (i64)K * ctx->Imax;
         if (bound < LIM && (i64)K * wmax < LIM) return RangePlan{false, K, d_cap};
     }
     return rp;
@@ -413,9 +414,9 @@ typedef long long tm_t;
 #else
 typedef int tm_t;
 #endif
-static __device__ __forceinline__ void fstep(tm_t &F, tm_t &SU, tm_t x, tm_t I, tm_t Te, tm_t w);
-static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
-static __device__ __forceinline__ tm_t vaddmax(tm_t a, tm_t b, tm_t c);
+static __device__ __forceinline__ void fstep(tm_t &NF, tm_t &SU, tm_t g, tm_t NI, tm_t Te, tm_t w);
+static __device__ __forceinline__ tm_t vmin(tm_t a, tm_t b);
+static __device__ __forceinline__ tm_t vaddmin(tm_t a, tm_t b, tm_t c);
 )";
     // ---- decode: unit u -> digits (function N-1: config only) -------------------------
     s << "static __device__ __forceinline__ void dag_decode(u64 u, int (&dig)[SM_N], const int *fixed) {\n";
@@ -429,35 +430,39 @@ static __device__ __forceinline__ tm_t vaddmax(tm_t a, tm_t b, tm_t c);
     for (int k = 0; k < nf; ++k) s << "  dig[" << k << "] = fixed[" << k << "];\n";
     s << "  (void)u; (void)fixed;\n}\n";
 
-    // ---- input expressions --------------------------------------------------------------
-    auto x_expr = [&](int k, const char *src) {
+    // ---- input expressions, negated time (NF = -F) ---------------------------------------
+    // min over predecessors of NF  (= -max over predecessors of F: the AND-join)
+    auto nf_min = [&](int k) {
         const int e0 = ctx->pred_ptr[k], e1 = ctx->pred_ptr[k + 1];
-        if (e0 == e1) return std::string(src);
-        std::string e = "F[" + std::to_string(ctx->pred_idx[e0]) + "]";
-        for (int e_ = e0 + 1; e_ < e1; ++e_) e = "vmax(" + e + ", F[" + std::to_string(ctx->pred_idx[e_]) + "])";
+        std::string e = "NF[" + std::to_string(ctx->pred_idx[e0]) + "]";
+        for (int e_ = e0 + 1; e_ < e1; ++e_) e = "vmin(" + e + ", NF[" + std::to_string(ctx->pred_idx[e_]) + "])";
         return e;
     };
+    auto is_src = [&](int k) { return ctx->pred_ptr[k] == ctx->pred_ptr[k + 1]; };
     // ---- j = 0 ----------------------------------------------------------------------------
-    s << "template <int A> static __device__ __forceinline__ void dag_first(tm_t (&F)[A], const tm_t (&I)[A], "
-         "tm_t *st0, int tid, tm_t &xl, tm_t &upL) {\n";
+    s << "template <int A> static __device__ __forceinline__ void dag_first(tm_t (&NF)[A], const tm_t (&NI)[A], "
+         "tm_t *st0, int tid, tm_t &xl, tm_t &nlu) {\n";
     for (int k = 0; k < N - 1; ++k) {
-        s << "  { const tm_t x = " << x_expr(k, "(tm_t)0") << "; st0[" << k << " * SM_THREADS + tid] = x; F[" << k
-          << "] = x + I[" << k << "]; }\n";
+        s << "  { const tm_t x = " << (is_src(k) ? std::string("(tm_t)0") : "-" + nf_min(k)) << "; st0[" << k
+          << " * SM_THREADS + tid] = x; NF[" << k << "] = NI[" << k << "] - x; }\n";
     }
-    s << "  xl = " << x_expr(N - 1, "(tm_t)0") << ";\n";
+    s << "  xl = " << (is_src(N - 1) ? std::string("(tm_t)0") : "-" + nf_min(N - 1)) << ";\n";
     for (int k = 0; k < N - 1; ++k)
-        if ((ctx->sinkmask >> k) & 1ull) s << "  upL = vmax(upL, F[" << k << "]);\n";
-    s << "  (void)F; (void)I; (void)st0; (void)tid; (void)upL;\n}\n";
-    // ---- j >= 1 -----------------------------------------------------------------------------
-    s << "template <int A> static __device__ __forceinline__ void dag_step(tm_t (&F)[A], tm_t (&SU)[A], const tm_t "
-         "(&I)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], tm_t o, tm_t negO, tm_t &xl, tm_t &upL) {\n";
+        if ((ctx->sinkmask >> k) & 1ull) s << "  nlu = vmin(nlu, NF[" << k << "]);\n";
+    s << "  (void)NF; (void)NI; (void)st0; (void)tid; (void)nlu;\n}\n";
+    // ---- j >= 1: g = x - f = x + NF ---------------------------------------------------------
+    s << "template <int A> static __device__ __forceinline__ void dag_step(tm_t (&NF)[A], tm_t (&SU)[A], const tm_t "
+         "(&NI)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], tm_t o, tm_t &xl, tm_t &nlu) {\n";
+    for (int k = 0; k < N - 1; ++k) {
+        const std::string g = is_src(k) ? "o + NF[" + std::to_string(k) + "]"
+                                        : "NF[" + std::to_string(k) + "] - " + nf_min(k);
+        s << "  fstep(NF[" << k << "], SU[" << k << "], " << g << ", NI[" << k << "], Te[" << k << "], Wn[" << k
+          << "]);\n";
+    }
+    s << "  xl = " << (is_src(N - 1) ? std::string("o") : "-" + nf_min(N - 1)) << ";\n";
     for (int k = 0; k < N - 1; ++k)
-        s << "  fstep(F[" << k << "], SU[" << k << "], " << x_expr(k, "o") << ", I[" << k << "], Te[" << k
-          << "], Wn[" << k << "]);\n";
-    s << "  xl = " << x_expr(N - 1, "o") << ";\n";
-    for (int k = 0; k < N - 1; ++k)
-        if ((ctx->sinkmask >> k) & 1ull) s << "  upL = vaddmax(F[" << k << "], negO, upL);\n";
-    s << "  (void)F; (void)SU; (void)I; (void)Te; (void)Wn; (void)o; (void)negO; (void)upL;\n}\n";
+        if ((ctx->sinkmask >> k) & 1ull) s << "  nlu = vaddmin(NF[" << k << "], o, nlu);\n";
+    s << "  (void)NF; (void)SU; (void)NI; (void)Te; (void)Wn; (void)o; (void)nlu;\n}\n";
     return s.str();
 }
 
@@ -506,7 +511,8 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
     // offsets in shared memory when they fit next to the per-thread accumulators
     const size_t max_smem = 227 * 1024;
     bool off_smem = smem_bytes(ctx, a, rp, n_off, true) <= max_smem;
-    const int minb = 1;
+    const char *mb_env = getenv("SMILESS_MINB");     // tuning knob: min CTAs/SM for __launch_bounds__
+    const int minb = mb_env ? std::max(1, atoi(mb_env)) : 1;
     std::string src = full_source(ctx, a, rp, off_smem, minb);
     auto it = ctx->jit_cache.find(src);
     if (it == ctx->jit_cache.end()) {
