@@ -128,6 +128,9 @@ typedef struct {
     uint32_t flags;               /* SMILESS_FLAG_*                                                  */
     int32_t shard, n_shards;      /* multi-GPU: this rank plans chunks c with c % n_shards == shard;
                                      n_shards = 0 or 1: everything                                   */
+    double *cost_out;             /* optional (testing): host array [end - begin] receiving every
+                                     candidate's cost as the evaluator computed it, NaN when it is
+                                     infeasible or was pruned; NULL = off; end - begin <= 2^26     */
 } smiless_plan_args;
 
 typedef struct {
@@ -178,10 +181,11 @@ SMILESS_API int smiless_kernel_source(smiless_ctx *ctx, const smiless_plan_args 
                                       size_t *len);
 
 /* NVRTC-compile that source for sm_100a without loading it (works without a GPU);
- * the compile/ptxas log (registers, spills) goes to log.  Returns OK, EJIT or an
- * argument error. */
+ * the compile/ptxas log (registers, spills) goes to log, the cubin (SASS for
+ * cuobjdump) to cubin when cubin_cap is large enough; *cubin_size gets its size.
+ * Returns OK, EJIT or an argument error. */
 SMILESS_API int smiless_jit_compile(smiless_ctx *ctx, const smiless_plan_args *a, char *log, size_t logcap,
-                                    size_t *cubin_size);
+                                    void *cubin, size_t cubin_cap, size_t *cubin_size);
 
 #ifdef __cplusplus
 }

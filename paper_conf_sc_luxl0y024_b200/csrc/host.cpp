@@ -146,6 +146,9 @@ struct PlanParamsHost {
     int prune;
     int shard, n_shards;
     int chunk_units;
+    double *dump;
+    const int *tabNI;
+    int zero;
     int fixed[SMILESS_MAX_FUNCS];  // evaluator uses SM_NFIXED_ALLOC <= SMILESS_MAX_FUNCS; extra tail is ignored
 };
 
@@ -206,7 +209,7 @@ struct smiless_ctx {
     // device state
     bool dev_ready = false;
     int n_sms = 0;
-    DevBuf<int> dI, dT, dPtr, dIdx;
+    DevBuf<int> dI, dNI, dT, dPtr, dIdx;
     DevBuf<double> dU;
     DevBuf<i64> dArr;
     DevBuf<unsigned char> dOff;
@@ -216,6 +219,7 @@ struct smiless_ctx {
     DevBuf<double> dCost;
     DevBuf<i64> dLat;
     DevBuf<unsigned char> dFeas;
+    DevBuf<double> dDump;
     DevBuf<ResBlock> dRes;
     ResBlock *hRes = nullptr;    // pinned
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -283,17 +287,20 @@ int upload_tables(smiless_ctx *ctx) {
     if (!ctx->tables_dirty) return SMILESS_OK;
     const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
     const size_t padU = (size_t)((ctx->sumM + 1) & ~1);
-    std::vector<int> I(padI, 0), T(padI, 0);
+    std::vector<int> I(padI, 0), NI(padI, 0), T(padI, 0);
     std::vector<double> U(padU, 0.0);
     std::copy(ctx->I.begin(), ctx->I.end(), I.begin());
+    for (int r = 0; r < ctx->sumM; ++r) NI[r] = -ctx->I[r];
     std::copy(ctx->T.begin(), ctx->T.end(), T.begin());
     std::copy(ctx->U.begin(), ctx->U.end(), U.begin());
     CK(ctx->dI.ensure(padI), "cudaMalloc");
+    CK(ctx->dNI.ensure(padI), "cudaMalloc");
     CK(ctx->dT.ensure(padI), "cudaMalloc");
     CK(ctx->dU.ensure(padU), "cudaMalloc");
     CK(ctx->dPtr.ensure(ctx->pred_ptr.size()), "cudaMalloc");
     CK(ctx->dIdx.ensure(std::max<size_t>(ctx->pred_idx.size(), 1)), "cudaMalloc");
     CK(cudaMemcpy(ctx->dI.p, I.data(), padI * sizeof(int), cudaMemcpyHostToDevice), "H2D tables");
+    CK(cudaMemcpy(ctx->dNI.p, NI.data(), padI * sizeof(int), cudaMemcpyHostToDevice), "H2D tables");
     CK(cudaMemcpy(ctx->dT.p, T.data(), padI * sizeof(int), cudaMemcpyHostToDevice), "H2D tables");
     CK(cudaMemcpy(ctx->dU.p, U.data(), padU * sizeof(double), cudaMemcpyHostToDevice), "H2D tables");
     CK(cudaMemcpy(ctx->dPtr.p, ctx->pred_ptr.data(), ctx->pred_ptr.size() * sizeof(int), cudaMemcpyHostToDevice),
@@ -415,8 +422,10 @@ typedef long long tm_t;
 typedef int tm_t;
 #endif
 static __device__ __forceinline__ void fstep(tm_t &NF, tm_t &SU, tm_t g, tm_t NI, tm_t Te, tm_t w);
-static __device__ __forceinline__ tm_t vmin(tm_t a, tm_t b);
+static __device__ __forceinline__ tm_t vminz(tm_t a, tm_t b, tm_t z);
 static __device__ __forceinline__ tm_t vaddmin(tm_t a, tm_t b, tm_t c);
+static __device__ __forceinline__ tm_t opaque_add(tm_t a, tm_t b);
+static __device__ __forceinline__ tm_t opaque_sub(tm_t a, tm_t b);
 )";
     // ---- decode: unit u -> digits (function N-1: config only) -------------------------
     s << "static __device__ __forceinline__ void dag_decode(u64 u, int (&dig)[SM_N], const int *fixed) {\n";
@@ -431,38 +440,41 @@ static __device__ __forceinline__ tm_t vaddmin(tm_t a, tm_t b, tm_t c);
     s << "  (void)u; (void)fixed;\n}\n";
 
     // ---- input expressions, negated time (NF = -F) ---------------------------------------
-    // min over predecessors of NF  (= -max over predecessors of F: the AND-join)
+    // min over predecessors of NF (= -(max over predecessors of F): the AND-join).
+    // vminz blocks VIMNMX3 formation (ptxas erratum); nothing below negates a min/max input.
     auto nf_min = [&](int k) {
         const int e0 = ctx->pred_ptr[k], e1 = ctx->pred_ptr[k + 1];
         std::string e = "NF[" + std::to_string(ctx->pred_idx[e0]) + "]";
-        for (int e_ = e0 + 1; e_ < e1; ++e_) e = "vmin(" + e + ", NF[" + std::to_string(ctx->pred_idx[e_]) + "])";
+        for (int e_ = e0 + 1; e_ < e1; ++e_) e = "vminz(" + e + ", NF[" + std::to_string(ctx->pred_idx[e_]) + "], z)";
         return e;
     };
     auto is_src = [&](int k) { return ctx->pred_ptr[k] == ctx->pred_ptr[k + 1]; };
-    // ---- j = 0 ----------------------------------------------------------------------------
+    // ---- j = 0: start = x; nx = -x is stored (st0) ---------------------------------------
     s << "template <int A> static __device__ __forceinline__ void dag_first(tm_t (&NF)[A], const tm_t (&NI)[A], "
-         "tm_t *st0, int tid, tm_t &xl, tm_t &nlu) {\n";
+         "tm_t *st0, int tid, tm_t &nxl, tm_t &nlu, const tm_t z) {\n";
     for (int k = 0; k < N - 1; ++k) {
-        s << "  { const tm_t x = " << (is_src(k) ? std::string("(tm_t)0") : "-" + nf_min(k)) << "; st0[" << k
-          << " * SM_THREADS + tid] = x; NF[" << k << "] = NI[" << k << "] - x; }\n";
+        s << "  { const tm_t nx = " << (is_src(k) ? std::string("(tm_t)0") : nf_min(k)) << "; st0[" << k
+          << " * SM_THREADS + tid] = nx; NF[" << k << "] = NI[" << k << "] + nx; }\n";
     }
-    s << "  xl = " << (is_src(N - 1) ? std::string("(tm_t)0") : "-" + nf_min(N - 1)) << ";\n";
+    s << "  nxl = " << (is_src(N - 1) ? std::string("(tm_t)0") : nf_min(N - 1)) << ";\n";
     for (int k = 0; k < N - 1; ++k)
-        if ((ctx->sinkmask >> k) & 1ull) s << "  nlu = vmin(nlu, NF[" << k << "]);\n";
-    s << "  (void)NF; (void)NI; (void)st0; (void)tid; (void)nlu;\n}\n";
-    // ---- j >= 1: g = x - f = x + NF ---------------------------------------------------------
-    s << "template <int A> static __device__ __forceinline__ void dag_step(tm_t (&NF)[A], tm_t (&SU)[A], const tm_t "
-         "(&NI)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], tm_t o, tm_t &xl, tm_t &nlu) {\n";
+        if ((ctx->sinkmask >> k) & 1ull) s << "  nlu = vminz(nlu, NF[" << k << "], z);\n";
+    s << "  (void)NF; (void)NI; (void)st0; (void)tid; (void)nlu; (void)z;\n}\n";
+    // ---- j >= 1: g = x - f = x + NF; returns x_last + CN ------------------------------------
+    s << "template <int A> static __device__ __forceinline__ tm_t dag_step(tm_t (&NF)[A], tm_t (&SU)[A], const tm_t "
+         "(&NI)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], const tm_t o, const tm_t CN, tm_t &nlu, const tm_t z) "
+         "{\n";
     for (int k = 0; k < N - 1; ++k) {
         const std::string g = is_src(k) ? "o + NF[" + std::to_string(k) + "]"
                                         : "NF[" + std::to_string(k) + "] - " + nf_min(k);
         s << "  fstep(NF[" << k << "], SU[" << k << "], " << g << ", NI[" << k << "], Te[" << k << "], Wn[" << k
           << "]);\n";
     }
-    s << "  xl = " << (is_src(N - 1) ? std::string("o") : "-" + nf_min(N - 1)) << ";\n";
     for (int k = 0; k < N - 1; ++k)
         if ((ctx->sinkmask >> k) & 1ull) s << "  nlu = vaddmin(NF[" << k << "], o, nlu);\n";
-    s << "  (void)NF; (void)SU; (void)NI; (void)Te; (void)Wn; (void)o; (void)nlu;\n}\n";
+    s << "  (void)NF; (void)SU; (void)NI; (void)Te; (void)Wn; (void)o; (void)nlu; (void)z;\n";
+    s << "  return " << (is_src(N - 1) ? std::string("opaque_add(o, CN)") : "opaque_sub(CN, " + nf_min(N - 1) + ")")
+      << ";\n}\n";
     return s.str();
 }
 
@@ -614,10 +626,10 @@ void smiless_destroy(smiless_ctx *ctx) {
         cudaSetDevice(ctx->device);
         for (auto &kv : ctx->jit_cache)
             if (kv.second.mod) driver().moduleUnload(kv.second.mod);
-        ctx->dI.release(); ctx->dT.release(); ctx->dU.release(); ctx->dPtr.release(); ctx->dIdx.release();
+        ctx->dI.release(); ctx->dNI.release(); ctx->dT.release(); ctx->dU.release(); ctx->dPtr.release(); ctx->dIdx.release();
         ctx->dArr.release(); ctx->dOff.release(); ctx->dScal.release(); ctx->dErr.release();
         ctx->dCounter.release(); ctx->dStats.release(); ctx->dBlk.release(); ctx->dIdxEval.release();
-        ctx->dCost.release(); ctx->dLat.release(); ctx->dFeas.release(); ctx->dRes.release();
+        ctx->dCost.release(); ctx->dLat.release(); ctx->dFeas.release(); ctx->dRes.release(); ctx->dDump.release();
         if (ctx->hRes) cudaFreeHost(ctx->hRes);
         for (auto &ev : ctx->ev)
             if (ev) cudaEventDestroy(ev);
@@ -789,6 +801,7 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
     const u64 cb = a->begin;
     const u64 ce = (a->end == 0 || a->end > space) ? space : a->end;
     if (cb > ce) return fail(ctx, SMILESS_EINVAL, "begin > end");
+    if (a->cost_out && ce - cb > ((u64)1 << 26)) return fail(ctx, SMILESS_EINVAL, "cost_out range larger than 2^26");
     const int n_shards = a->n_shards <= 0 ? 1 : a->n_shards;
     const int shard = a->n_shards <= 0 ? 0 : a->shard;
     if ((rc = ensure_device(ctx))) return rc;
@@ -832,6 +845,8 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
         PlanParamsHost pp;
         memset(&pp, 0, sizeof pp);
         pp.tabI = ctx->dI.p;
+        pp.tabNI = ctx->dNI.p;
+        pp.zero = 0;
         pp.tabT = ctx->dT.p;
         pp.tabU = ctx->dU.p;
         pp.off = ctx->dOff.p;
@@ -852,6 +867,11 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
         pp.n_shards = n_shards;
         pp.chunk_units = kChunkUnits;
         for (int k = 0; k < a->n_fixed; ++k) pp.fixed[k] = a->fixed_digits[k];
+        if (a->cost_out) {
+            CK(ctx->dDump.ensure((size_t)(ce - cb)), "cudaMalloc dump");
+            CK(cudaMemsetAsync(ctx->dDump.p, 0xff, (size_t)(ce - cb) * sizeof(double), st), "memset dump");  // NaN
+            pp.dump = ctx->dDump.p;
+        }
         // split very large ranges into several launches (bounded kernel duration)
         const u64 claims_per_launch = (u64)1 << 28;  // units (x W candidates)
         CK(cudaEventRecord(ctx->ev[1], st), "event");
@@ -871,6 +891,9 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
         if (e) return cuda_fail(ctx, (cudaError_t)e, "reduce launch");
         ++launches;
         CK(cudaMemcpyAsync(&ctx->dRes.p->stats[0], ctx->dStats.p, 16, cudaMemcpyDeviceToDevice, st), "D2D stats");
+        if (a->cost_out)
+            CK(cudaMemcpyAsync(a->cost_out, ctx->dDump.p, (size_t)(ce - cb) * sizeof(double), cudaMemcpyDeviceToHost, st),
+               "D2H dump");
     } else if (single && ce > cb) {
         // the space is the single candidate of the pinned digits: index 0
         CK(cudaMemsetAsync(&ctx->dRes.p->best_c, 0, 16, st), "memset");
@@ -965,7 +988,8 @@ int smiless_kernel_source(smiless_ctx *ctx, const smiless_plan_args *a, char *bu
     return SMILESS_OK;
 }
 
-int smiless_jit_compile(smiless_ctx *ctx, const smiless_plan_args *a, char *log, size_t logcap, size_t *cubin_size) {
+int smiless_jit_compile(smiless_ctx *ctx, const smiless_plan_args *a, char *log, size_t logcap, void *cubin_out,
+                        size_t cubin_cap, size_t *cubin_size) {
     if (!ctx) return SMILESS_EINVAL;
     ctx->err.clear();
     int rc = validate_args(ctx, a, false);
@@ -983,6 +1007,7 @@ int smiless_jit_compile(smiless_ctx *ctx, const smiless_plan_args *a, char *log,
         log[n] = '\0';
     }
     if (cubin_size) *cubin_size = cubin.size();
+    if (cubin_out && cubin_cap >= cubin.size()) memcpy(cubin_out, cubin.data(), cubin.size());
     return rc;
 }
 

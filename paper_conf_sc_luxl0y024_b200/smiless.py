@@ -48,6 +48,7 @@ class PlanArgs(ctypes.Structure):
         ("flags", ctypes.c_uint32),
         ("shard", ctypes.c_int32),
         ("n_shards", ctypes.c_int32),
+        ("cost_out", ctypes.c_void_p),
     ]
 
 
@@ -114,7 +115,7 @@ def load_library(build_if_missing: bool = True):
     lib.smiless_kernel_source.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.c_char_p, ctypes.c_size_t,
                                           ctypes.POINTER(ctypes.c_size_t)]
     lib.smiless_jit_compile.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.c_char_p, ctypes.c_size_t,
-                                        ctypes.POINTER(ctypes.c_size_t)]
+                                        vp, ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t)]
     for name in EXPORTS:
         if name not in ("smiless_destroy", "smiless_last_error"):
             getattr(lib, name).restype = ctypes.c_int
@@ -178,7 +179,7 @@ class Planner:
 
     # ---- args ----------------------------------------------------------------------------
     def _args(self, arrivals, sla_us, windows_us, n_fixed=0, fixed_digits=(), begin=0, end=0, flags=0,
-              shard=0, n_shards=0):
+              shard=0, n_shards=0, cost_out=None):
         keep = []
         if _is_device_tensor(arrivals):
             import torch
@@ -197,7 +198,11 @@ class Planner:
         a = PlanArgs(arrivals_us=ptr, n_arrivals=n, sla_us=int(sla_us), windows_us=win.ctypes.data,
                      n_windows=int(win.shape[0]), n_fixed=int(n_fixed),
                      fixed_digits=fixed.ctypes.data if n_fixed else None, begin=int(begin), end=int(end),
-                     flags=int(flags), shard=int(shard), n_shards=int(n_shards))
+                     flags=int(flags), shard=int(shard), n_shards=int(n_shards),
+                     cost_out=cost_out.ctypes.data if cost_out is not None else None)
+        if cost_out is not None:
+            assert cost_out.dtype == np.float64 and cost_out.flags.c_contiguous
+            keep.append(cost_out)
         return a, keep
 
     # ---- API -----------------------------------------------------------------------------
@@ -249,12 +254,19 @@ class Planner:
         self._check(self._lib.smiless_kernel_source(self._ctx, ctypes.byref(a), buf, n.value, ctypes.byref(n)))
         return buf.value.decode()
 
-    def jit_compile(self, arrivals, sla_us, windows_us, **kw) -> Tuple[str, int]:
-        """NVRTC-compile the specialised evaluator (no GPU needed); returns (ptxas log, cubin bytes)."""
+    def jit_compile(self, arrivals, sla_us, windows_us, want_cubin: bool = False, **kw):
+        """NVRTC-compile the specialised evaluator (no GPU needed).
+
+        Returns (ptxas log, cubin size) or, with want_cubin, (ptxas log, cubin bytes)."""
         a, keep = self._args(arrivals, sla_us, windows_us, **kw)
         log = ctypes.create_string_buffer(1 << 16)
         n = ctypes.c_size_t()
-        self._check(self._lib.smiless_jit_compile(self._ctx, ctypes.byref(a), log, 1 << 16, ctypes.byref(n)))
+        cap = 8 << 20 if want_cubin else 0
+        buf = ctypes.create_string_buffer(cap) if want_cubin else None
+        self._check(self._lib.smiless_jit_compile(self._ctx, ctypes.byref(a), log, 1 << 16,
+                                                  buf if want_cubin else None, cap, ctypes.byref(n)))
+        if want_cubin:
+            return log.value.decode(), buf.raw[:n.value]
         return log.value.decode(), int(n.value)
 
 

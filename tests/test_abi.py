@@ -178,3 +178,36 @@ def test_int64_path_selected_when_int32_range_fails():
     p2 = W.make_config("C1", n_arrivals=20)
     src2 = S.planner_for(p2).kernel_source(p2.arrivals_us, p2.sla_us, p2.windows_us)
     assert "#define SM_TIME64 0" in src2
+
+
+def _sass(pl, p, **kw):
+    import subprocess
+    import tempfile
+    log, cubin = pl.jit_compile(p.arrivals_us, p.sla_us, p.windows_us, want_cubin=True, **kw)
+    with tempfile.NamedTemporaryFile(suffix=".cubin") as f:
+        f.write(cubin)
+        f.flush()
+        return subprocess.run(["cuobjdump", "-sass", f.name], capture_output=True, text=True, check=True).stdout
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C3", "C4", "C5"])
+def test_sass_has_no_vimnmx3_and_is_dpx(name):
+    """ptxas 12.9 drops operand negations it folds into VIMNMX3 (tools/repro_vimnmx3.cu,
+    DESIGN.md "Compiler erratum"): the evaluator must contain no VIMNMX3.  Also checks the
+    hot loop really is DPX integer code with the busy mask on the FMA pipe (IMAD.HI)."""
+    p = W.make_config(name, n_arrivals=100)
+    pl = S.planner_for(p)
+    nf = 3 if name == "C5" else 0
+    sass = _sass(pl, p, n_fixed=nf, fixed_digits=[0] * nf)
+    assert "VIMNMX3" not in sass
+    for op in ("VIADDMNMX", "VIMNMX.RELU", "IMAD.HI", "LDS.128"):
+        assert op in sass, op
+    assert "HMMA" not in sass and "UTC" not in sass          # no tensor cores on this path
+    assert "LDL" not in sass and "STL" not in sass            # no local memory
+
+
+def test_library_kernels_have_no_vimnmx3():
+    import subprocess
+    out = subprocess.run(["cuobjdump", "-sass", S.LIB_PATH], capture_output=True, text=True, check=True).stdout
+    assert "prep_offsets_kernel" in out and "eval_exact_kernel" in out
+    assert "VIMNMX3" not in out

@@ -283,3 +283,66 @@ def test_bench_configuration_full_size_properties():
     for i in range(len(idx)):
         if f[i]:
             assert full.feasible and (full.cost, full.index) <= (c[i], int(idx[i]))
+
+
+# ---------------------------------------------------------------------------------------
+# Per-candidate parity of the fast evaluator itself (cost_out), not only of its argmin
+# ---------------------------------------------------------------------------------------
+
+def assert_dump_matches(out, oc, of):
+    feas = ~np.isnan(out)
+    assert (feas == of).all(), np.nonzero(feas != of)[0][:10]
+    bad = np.nonzero(feas & (out.view(np.uint64) != oc.view(np.uint64)))[0]
+    assert len(bad) == 0, (bad[:10], out[bad[:10]], oc[bad[:10]])
+
+
+def test_random_dags_per_candidate_costs():
+    """Every candidate's cost as the int32/int64 evaluator computes it (sink sharing,
+    rebasing, clamped gaps, negated time, busy mask) equals the oracle's, bit for bit;
+    infeasible candidates are exactly the oracle's infeasible ones.  Joins of up to 3
+    predecessors (the VIMNMX3 erratum pattern) are frequent here."""
+    rng = np.random.default_rng(77)
+    n_checked = 0
+    for t in range(160):
+        n = int(rng.integers(1, 7))
+        p = W.random_problem(rng, n, 4, int(rng.integers(1, 6)), int(rng.integers(1, 140)))
+        space = p.space_size()
+        if space > 30000:
+            continue
+        flags = int(rng.choice([0, S.FLAG_NO_PRUNE, S.FLAG_FORCE_INT64]))
+        pl = S.planner_for(p)
+        out = np.empty(space)
+        pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=flags, cost_out=out)
+        oc, ol, of = OracleProblem(p).evaluate(np.arange(space, dtype=np.uint64))
+        assert_dump_matches(out, oc, of)
+        n_checked += 1
+    assert n_checked > 80
+
+
+@pytest.mark.parametrize("name", ["C1", "C4"])
+def test_config_per_candidate_costs(name):
+    p = W.make_config(name)
+    if name == "C4":
+        p = p.replace(sla_us=3_000_000)
+    pl = S.planner_for(p)
+    space = min(pl.space_size(len(p.windows_us)), 1 << 14)
+    for flags in (0, S.FLAG_NO_PRUNE):
+        out = np.empty(space)
+        pl.plan(p.arrivals_us, p.sla_us, p.windows_us, end=space, flags=flags, cost_out=out)
+        oc, ol, of = OracleProblem(p).evaluate(np.arange(space, dtype=np.uint64))
+        assert_dump_matches(out, oc, of)
+
+
+def test_bench_slice_per_candidate_costs_full_J():
+    """bench.py's C2 slice at J = 10^4: 2^12 consecutive candidates around the winner."""
+    import bench
+    p, kw = bench.workload("C2")
+    pl = S.planner_for(p)
+    full = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, **kw)
+    lo = (full.index if full.feasible else 0) // 4096 * 4096
+    out = np.empty(4096)
+    pl.plan(p.arrivals_us, p.sla_us, p.windows_us, begin=lo, end=lo + 4096, flags=S.FLAG_NO_PRUNE,
+            cost_out=out, **kw)
+    oc, ol, of = OracleProblem(p, **kw).evaluate(np.arange(lo, lo + 4096, dtype=np.uint64))
+    assert_dump_matches(out, oc, of)
+    assert of.any() == full.feasible
