@@ -55,19 +55,37 @@ def workload(name: str = "C2"):
     raise KeyError(name)
 
 
-def algorithmic_ops_per_unit(p, n_fixed: int) -> int:
-    """Integer ops one lane-unit (one upstream prefix x all W windows of the last
-    function) needs per the model: per invocation j >= 1, 6 ops
-    per upstream function-step (g, u, busy, delta, select, F), +1 per extra join input,
-    +1 per upstream sink latency check, 7 per last-function window variant (6 + the
-    latency max), +1 shared offset negation."""
+def configs_per_lane(p) -> int:
+    """Mirror of host.cpp configs_per_lane (G): last-function configs carried per lane."""
+    M = int(p.n_configs[-1])
+    Wn = len(p.windows_us)
+    want = int(os.environ.get("SMILESS_G", "0")) or max(1, 16 // Wn)
+    G = 1
+    for g in range(1, want + 1):
+        if M % g == 0 and g * Wn <= 32:
+            G = g
+    return G
+
+
+def algorithmic_ops_per_candidate(p) -> float:
+    """Integer ops per candidate over the whole horizon for the algorithm as implemented
+    (DESIGN.md "Roofline"): per invocation j >= 1 a lane-unit (one upstream prefix x G
+    configs x W windows of the last function) executes
+      7 per upstream function-step (g, u, delta, busy mask, masked update, +I, sum u),
+      +1 per extra join input, +1 per upstream sink latency check,
+      per last-function config 3 shared (x + CN, CN += -I, o + CN),
+      7 per window variant (g, u, delta, mask, update, sum u, latency) or 4 for keep-alive,
+    divided by the G*W candidates of the unit."""
     n = p.n_funcs
     Wn = len(p.windows_us)
-    joins = sum(max(0, len(p.preds(k)) - 1) for k in range(n))
+    G = configs_per_lane(p)
+    joins = sum(max(0, len(p.preds(k)) - 1) for k in range(n - 1))
     listed = set(int(v) for v in p.pred_idx)
     up_sinks = sum(1 for k in range(n - 1) if k not in listed)
-    per_step = 6 * (n - 1) + joins + up_sinks + 7 * Wn + 1
-    return per_step * (len(p.arrivals_us) - 1)
+    w0 = 1 if int(p.windows_us[0]) == 0 else 0
+    per_unit_step = 7 * (n - 1) + joins + max(0, len(p.preds(n - 1)) - 1) + up_sinks + \
+        G * (3 + 4 * w0 + 7 * (Wn - w0))
+    return per_unit_step * (len(p.arrivals_us) - 1) / (G * Wn)
 
 
 class ClockSampler:
@@ -323,8 +341,8 @@ def main():
     clocks = clk.summary()
     sm_mhz = clocks["sm_mhz"] or peaks.get("sm_max_mhz", 1965.0)
     peak_ops = props.multi_processor_count * ISSUE_LANES_PER_CLK_PER_SM * float(clocks["sm_max_mhz"] or 1965.0) * 1e6
-    units_per_launch = res.n_decided / len(p.windows_us)
-    ops = algorithmic_ops_per_unit(p, kw["n_fixed"]) * units_per_launch
+    ops_per_cand = algorithmic_ops_per_candidate(p)
+    ops = ops_per_cand * res.n_decided
     kernel_ms_per_step = kernel_ms / args.steps
     achieved = ops / (kernel_ms_per_step / 1e3)
     line = {
@@ -343,7 +361,7 @@ def main():
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_ops, "unit": "int-ops/s",
                      "frac": achieved / peak_ops, "traffic": ncu_traffic(),
                      "kernel": "smiless_plan_kernel", "kernel_ms_per_launch": kernel_ms_per_step,
-                     "ops_per_unit": algorithmic_ops_per_unit(p, kw["n_fixed"]),
+                     "int_ops_per_candidate": ops_per_cand, "configs_per_lane": configs_per_lane(p),
                      "peak_basis": "issue peak: SMs x 4 SMSP x 32 lanes x sm_max_mhz (DESIGN.md Roofline)"},
         "kernel_share_of_step": kernel_ms_per_step / (ms / args.steps),
     }

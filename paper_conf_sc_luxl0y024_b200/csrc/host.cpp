@@ -391,9 +391,24 @@ RangePlan range_plan(const smiless_ctx *ctx, const smiless_plan_args *a) {
 // ------------------------------------------------------------------------------------
 // NVRTC specialisation
 // ------------------------------------------------------------------------------------
+// Configs of the last function carried per lane (a unit = G x W candidates): as many as keep
+// G * W <= 16 variants (registers) and divide M_{N-1}.  SMILESS_G overrides (tuning).
+int configs_per_lane(const smiless_ctx *ctx, const smiless_plan_args *a) {
+    const int M = ctx->M[ctx->N - 1], W = a->n_windows;
+    int G = 1;
+    const char *env = getenv("SMILESS_G");
+    const int want = env ? std::max(1, atoi(env)) : std::max(1, 16 / W);
+    for (int g = 1; g <= want; ++g)
+        if (M % g == 0 && g * W <= 32) G = g;
+    return G;
+}
+
 std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, bool off_smem,
                             int minb) {
     const int N = ctx->N, W = a->n_windows, NU = N - 1, nf = a->n_fixed;
+    const int G = configs_per_lane(ctx, a);
+    const char *un_env = getenv("SMILESS_UNROLL");
+    const int unroll = (un_env && atoi(un_env) == 2) ? 2 : 4;
     std::ostringstream s;
     s << "// generated by host.cpp:dag_spec_source -- DAG-specialised prefix of evaluator.cuh\n";
     s << "#define SM_N " << N << "\n#define SM_NU " << NU << "\n#define SM_NU_ALLOC " << std::max(NU, 1) << "\n";
@@ -403,6 +418,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_OFF_SMEM " << (off_smem ? 1 : 0) << "\n#define SM_THREADS " << kThreads
       << "\n#define SM_MINB " << minb << "\n";
     s << "#define SM_W0_ZERO " << (a->windows_us[0] == 0 ? 1 : 0) << "\n";
+    s << "#define SM_G " << G << "\n#define SM_UNROLL " << unroll << "\n";
     // compile-time window grid (immediates) and a constant-bank copy for runtime indices
     s << "#define SM_WIN(v) (";
     for (int v = 0; v < W; ++v) s << "(v)==" << v << "?" << a->windows_us[v] << ":";
@@ -426,11 +442,13 @@ static __device__ __forceinline__ tm_t vminz(tm_t a, tm_t b, tm_t z);
 static __device__ __forceinline__ tm_t vaddmin(tm_t a, tm_t b, tm_t c);
 static __device__ __forceinline__ tm_t opaque_add(tm_t a, tm_t b);
 static __device__ __forceinline__ tm_t opaque_sub(tm_t a, tm_t b);
+static __device__ __forceinline__ tm_t vaddmax(tm_t a, tm_t b, tm_t c);
 )";
     // ---- decode: unit u -> digits (function N-1: config only) -------------------------
     s << "static __device__ __forceinline__ void dag_decode(u64 u, int (&dig)[SM_N], const int *fixed) {\n";
     if (nf <= N - 1) {
-        s << "  dig[" << N - 1 << "] = (int)(u % " << ctx->M[N - 1] << "ull); u /= " << ctx->M[N - 1] << "ull;\n";
+        const int groups = ctx->M[N - 1] / G;   // config groups of the last function
+        s << "  dig[" << N - 1 << "] = (int)(u % " << groups << "ull); u /= " << groups << "ull;\n";
         for (int k = N - 2; k >= nf; --k) {
             const u64 radix = (u64)ctx->M[k] * (u64)W;
             s << "  dig[" << k << "] = (int)(u % " << radix << "ull); u /= " << radix << "ull;\n";
@@ -460,21 +478,23 @@ static __device__ __forceinline__ tm_t opaque_sub(tm_t a, tm_t b);
     for (int k = 0; k < N - 1; ++k)
         if ((ctx->sinkmask >> k) & 1ull) s << "  nlu = vminz(nlu, NF[" << k << "], z);\n";
     s << "  (void)NF; (void)NI; (void)st0; (void)tid; (void)nlu; (void)z;\n}\n";
-    // ---- j >= 1: g = x - f = x + NF; returns x_last + CN ------------------------------------
+    // ---- j >= 1: g = x - f = x + NF; returns x of the last function ----------------------
     s << "template <int A> static __device__ __forceinline__ tm_t dag_step(tm_t (&NF)[A], tm_t (&SU)[A], const tm_t "
-         "(&NI)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], const tm_t o, const tm_t CN, tm_t &nlu, const tm_t z) "
-         "{\n";
+         "(&NI)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], const tm_t o, const tm_t z) {\n";
     for (int k = 0; k < N - 1; ++k) {
         const std::string g = is_src(k) ? "o + NF[" + std::to_string(k) + "]"
                                         : "NF[" + std::to_string(k) + "] - " + nf_min(k);
         s << "  fstep(NF[" << k << "], SU[" << k << "], " << g << ", NI[" << k << "], Te[" << k << "], Wn[" << k
           << "]);\n";
     }
+    s << "  (void)NF; (void)SU; (void)NI; (void)Te; (void)Wn; (void)o; (void)z;\n";
+    s << "  return " << (is_src(N - 1) ? std::string("o") : "opaque_sub(z, " + nf_min(N - 1) + ")") << ";\n}\n";
+    // ---- upstream sinks' latency: nlu = min_j (NF_k + o_j) = -max_j L_j -------------------
+    s << "template <int A> static __device__ __forceinline__ void dag_sinks(const tm_t (&NF)[A], const tm_t o, tm_t "
+         "&nlu) {\n";
     for (int k = 0; k < N - 1; ++k)
         if ((ctx->sinkmask >> k) & 1ull) s << "  nlu = vaddmin(NF[" << k << "], o, nlu);\n";
-    s << "  (void)NF; (void)SU; (void)NI; (void)Te; (void)Wn; (void)o; (void)nlu; (void)z;\n";
-    s << "  return " << (is_src(N - 1) ? std::string("opaque_add(o, CN)") : "opaque_sub(CN, " + nf_min(N - 1) + ")")
-      << ";\n}\n";
+    s << "  (void)NF; (void)o; (void)nlu;\n}\n";
     return s.str();
 }
 
@@ -513,7 +533,7 @@ size_t smem_bytes(const smiless_ctx *ctx, const smiless_plan_args *a, const Rang
     const size_t padU = (size_t)((ctx->sumM + 1) & ~1);
     const size_t tsz = rp.time64 ? 8 : 4;
     size_t b = 2 * padI * 4 + padU * 8;
-    b += 8ull * (size_t)(ctx->N - 1 + a->n_windows) * kThreads;
+    b += 8ull * (size_t)(ctx->N - 1 + a->n_windows * configs_per_lane(ctx, a)) * kThreads;
     b += (tsz * (size_t)ctx->N * kThreads + 15) & ~(size_t)15;
     if (off_smem) b += tsz * (size_t)n_off;
     return b;
@@ -832,8 +852,8 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
     if (!single && ce > cb) {
         JitKernel *jk = nullptr;
         if ((rc = get_kernel(ctx, a, rp, n_off, &jk))) return rc;
-        const int W = a->n_windows;
-        const u64 ub = cb / (u64)W, ue = (ce + (u64)W - 1) / (u64)W;
+        const u64 V = (u64)a->n_windows * (u64)configs_per_lane(ctx, a);   // candidates per unit
+        const u64 ub = cb / V, ue = (ce + V - 1) / V;
         const u64 U = ue - ub;
         const u64 n_chunks = (U + kChunkUnits - 1) / kChunkUnits;
         const u64 my_chunks = n_chunks > (u64)shard ? (n_chunks - 1 - (u64)shard) / (u64)n_shards + 1 : 0;
