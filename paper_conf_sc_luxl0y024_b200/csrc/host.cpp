@@ -419,6 +419,9 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
       << "\n#define SM_MINB " << minb << "\n";
     s << "#define SM_W0_ZERO " << (a->windows_us[0] == 0 ? 1 : 0) << "\n";
     s << "#define SM_G " << G << "\n#define SM_UNROLL " << unroll << "\n";
+    const char *ck_env = getenv("SMILESS_CHECK");     // SLA early-exit check period (steps)
+    const int check = std::max(unroll, ck_env ? atoi(ck_env) : 16);
+    s << "#define SM_CHECK " << check << "\n";
     // compile-time window grid (immediates) and a constant-bank copy for runtime indices
     s << "#define SM_WIN(v) (";
     for (int v = 0; v < W; ++v) s << "(v)==" << v << "?" << a->windows_us[v] << ":";
