@@ -185,12 +185,13 @@ def run_reference(args):
     from oracle import OracleProblem
     threads = os.cpu_count() or 1
     o = OracleProblem(p, n_fixed=kw["n_fixed"], fixed_digits=kw["fixed_digits"])
-    # size one step to ~8 s of host work
+    # size one step so the whole --steps K --warmup W run takes ~2 minutes of host work
     probe = max(threads, 8)
     t0 = time.perf_counter()
     o.plan(0, probe, n_threads=threads)
     per = (time.perf_counter() - t0) / probe
-    n_step = max(threads, int(8.0 / max(per, 1e-9)))
+    step_s = max(1.0, min(8.0, 120.0 / max(1, args.steps)))
+    n_step = max(threads, int(step_s / max(per, 1e-9)))
     for _ in range(args.warmup):
         o.plan(0, min(n_step, threads * 2), n_threads=threads)
     t0 = time.perf_counter()
@@ -236,6 +237,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-pruned", action="store_true")
+    ap.add_argument("--no-full-space", action="store_true",
+                    help="skip the exhaustive pruned plan of the whole workload space (time-to-optimal)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -331,6 +334,35 @@ def main():
         pruned = {"time_to_optimal_ms": a.elapsed_time(b), "index": rp.index, "cost": rp.cost,
                   "max_latency_us": rp.max_latency_us, "full_evals_fraction": rp.n_full_evals / max(1, rp.n_decided)}
 
+    # time-to-optimal of the WHOLE configuration space (C2: 2^42 candidates): exact plan with
+    # pruning, sharded over the ranks (interleaved chunks) + NCCL reduction of the winner
+    full = None
+    if not args.no_full_space:
+        full_space = pl.space_size(len(p.windows_us))
+        barrier()
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        t0 = time.perf_counter()
+        a.record(stream)
+        rf = pl.plan(arr_dev, p.sla_us, p.windows_us, shard=rank, n_shards=world)
+        if world > 1:
+            g_cost, g_idx, g_lat, g_dec = reduce_best(rf.cost if rf.feasible else None, rf.index,
+                                                      rf.max_latency_us, rf.n_decided, dev)
+        else:
+            g_cost, g_idx, g_lat, g_dec = (rf.cost if rf.feasible else None), rf.index, rf.max_latency_us, rf.n_decided
+        b.record(stream)
+        torch.cuda.synchronize(dev)
+        wall = time.perf_counter() - t0
+        tt = torch.tensor([a.elapsed_time(b)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        full = {"candidates": full_space, "time_to_optimal_s": float(tt.item()) / 1e3, "wall_s": wall,
+                "decided_per_s": full_space / (float(tt.item()) / 1e3), "decided": g_dec,
+                "full_evals_local": rf.n_full_evals, "index": g_idx, "cost": g_cost, "max_latency_us": g_lat}
+        if rank == 0 and g_idx is not None:
+            c, w = pl.decode(g_idx, len(p.windows_us))
+            full["config"], full["window"] = c.tolist(), w.tolist()
+
     if rank != 0:
         if world > 1:
             dist.destroy_process_group()
@@ -354,6 +386,7 @@ def main():
         "winner": {"index": res.index, "cost": res.cost, "max_latency_us": res.max_latency_us,
                    "config": res.config.tolist(), "window": res.window.tolist()} if world == 1 else None,
         "pruned": pruned,
+        "time_to_optimal_full_space": full,
         "gpu_launches": launches,
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(p.arrivals_us.nbytes),
                 "d2h_bytes_per_step": 312},
@@ -369,6 +402,12 @@ def main():
         rate, n, dt, threads = cpu_oracle_rate(p, kw)
         line["cpu_baseline"] = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle",
                                 "sample": f"first {n} candidates of the slice ({dt:.1f} s, J={len(p.arrivals_us)})"}
+        if full is not None and full["index"] is not None:
+            from oracle import OracleProblem
+            oc, ol, of = OracleProblem(p).evaluate([full["index"]])
+            full["oracle_check"] = {"feasible": bool(of[0]), "cost_bits_equal": bool(oc[0] == full["cost"]),
+                                    "latency_equal": int(ol[0]) == full["max_latency_us"]}
+            full["oracle_extrapolated_s"] = full["candidates"] / rate
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

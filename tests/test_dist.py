@@ -1,0 +1,135 @@
+"""Multi-process (gloo, CPU) tests of the cross-rank exchange of paper_conf_sc_luxl0y024_b200.dist.
+
+The only collective of the path is the lexicographic (cost, index) MIN of
+the per-rank winners.  On CPU we check it with world sizes 2 and 3: ties go to the lowest
+index on any rank, infeasible ranks never win, all-infeasible stays infeasible, and the
+decided counts sum.  The end-to-end check shards a small problem's candidate space the
+way the kernel does (interleaved chunks of units) and compares the reduced winner with
+the oracle's plan of the whole space.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_sc_luxl0y024_b200.dist import reduce_best, cost_bits, bits_cost, INF_BITS
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def _worker(rank, world, port, cases, out_q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    res = []
+    for case in cases:
+        cost, idx, lat, dec = case[rank]
+        res.append(reduce_best(cost, idx, lat, dec, "cpu"))
+    out_q.put((rank, res))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def run_world(world, cases):
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, cases, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = dict(q.get(timeout=120) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    return out
+
+
+def test_cost_bits_order_like_doubles():
+    vals = [0.0, 1e-300, 0.5, 1.0, 3.25, 1e10, 8.3e1]
+    bits = [cost_bits(v) for v in vals]
+    assert sorted(range(len(vals)), key=lambda i: vals[i]) == sorted(range(len(vals)), key=lambda i: bits[i])
+    assert all(bits_cost(b) == v for b, v in zip(bits, vals))
+    assert cost_bits(None) == INF_BITS and bits_cost(INF_BITS) is None
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_reduce_best_gloo(world):
+    cases = [
+        # (cost, index, latency, decided) per rank
+        [(5.0, 10, 100, 7), (3.0, 20, 200, 5), (4.0, 1, 300, 1)][:world],
+        [(3.0, 25, 100, 1), (3.0, 20, 200, 1), (3.0, 21, 300, 1)][:world],       # tie -> lowest index
+        [(None, None, -1, 4), (2.0, 99, 50, 4), (None, None, -1, 4)][:world],     # infeasible ranks
+        [(None, None, -1, 3), (None, None, -1, 3), (None, None, -1, 3)][:world],  # all infeasible
+    ]
+    out = run_world(world, cases)
+    exp = [
+        (3.0, 20, 200, sum([7, 5, 1][:world])),
+        (3.0, 20, 200, world),
+        (2.0, 99, 50, 4 * world),
+        (None, None, -1, 3 * world),
+    ]
+    for r in range(world):
+        assert out[r] == exp, (r, out[r])
+
+
+def _shard_candidates(space, V, world, rank, chunk_units=256):
+    """Candidates the kernel assigns to `rank`: units of V candidates, chunks of
+    chunk_units units, chunk c belongs to rank c % world (csrc/evaluator.cuh)."""
+    n_units = (space + V - 1) // V
+    idx = []
+    for u in range(n_units):
+        if (u // chunk_units) % world == rank:
+            idx.extend(range(u * V, min(space, u * V + V)))
+    return np.asarray(idx, dtype=np.uint64)
+
+
+def _plan_worker(rank, world, port, out_q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import workloads as W
+    from oracle import OracleProblem
+    p = W.make_config("C1", n_arrivals=40)
+    o = OracleProblem(p)
+    cand = _shard_candidates(o.space_size(), 4 * len(p.windows_us), world, rank, chunk_units=8)
+    c, l, f = o.evaluate(cand)
+    best = None
+    for i in np.nonzero(f)[0]:
+        if best is None or (c[i], int(cand[i])) < best[:2]:
+            best = (c[i], int(cand[i]), int(l[i]))
+    r = reduce_best(best[0] if best else None, best[1] if best else None, best[2] if best else -1,
+                    len(cand), "cpu")
+    out_q.put((rank, r))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_sharded_plan_reduces_to_global_opt(world):
+    import workloads as W
+    from oracle import OracleProblem
+    p = W.make_config("C1", n_arrivals=40)
+    ref = OracleProblem(p).plan()
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_plan_worker, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    out = dict(q.get(timeout=180) for _ in range(world))
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    for r in range(world):
+        cost, idx, lat, dec = out[r]
+        assert (idx, cost, lat) == ref and dec == 4096
