@@ -149,6 +149,12 @@ struct PlanParamsHost {
     double *dump;
     const int *tabNI;
     int zero;
+    const unsigned *list_in;
+    const unsigned *list_n;
+    unsigned *list_out;
+    unsigned *list_cnt;
+    u64 list_base;
+    i64 horizon;
     int fixed[SMILESS_MAX_FUNCS];  // evaluator uses SM_NFIXED_ALLOC <= SMILESS_MAX_FUNCS; extra tail is ignored
 };
 
@@ -220,6 +226,7 @@ struct smiless_ctx {
     DevBuf<i64> dLat;
     DevBuf<unsigned char> dFeas;
     DevBuf<double> dDump;
+    DevBuf<unsigned> dList, dListCnt;
     DevBuf<ResBlock> dRes;
     ResBlock *hRes = nullptr;    // pinned
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -653,6 +660,7 @@ void smiless_destroy(smiless_ctx *ctx) {
         ctx->dArr.release(); ctx->dOff.release(); ctx->dScal.release(); ctx->dErr.release();
         ctx->dCounter.release(); ctx->dStats.release(); ctx->dBlk.release(); ctx->dIdxEval.release();
         ctx->dCost.release(); ctx->dLat.release(); ctx->dFeas.release(); ctx->dRes.release(); ctx->dDump.release();
+        ctx->dList.release(); ctx->dListCnt.release();
         if (ctx->hRes) cudaFreeHost(ctx->hRes);
         for (auto &ev : ctx->ev)
             if (ev) cudaEventDestroy(ev);
@@ -895,19 +903,55 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
             CK(cudaMemsetAsync(ctx->dDump.p, 0xff, (size_t)(ce - cb) * sizeof(double), st), "memset dump");  // NaN
             pp.dump = ctx->dDump.p;
         }
-        // split very large ranges into several launches (bounded kernel duration)
-        const u64 claims_per_launch = (u64)1 << 28;  // units (x W candidates)
+        // split very large ranges into several launches (bounded kernel duration).  Prune mode
+        // with J - 1 > horizon runs each batch twice: pass 1 (every unit, `horizon` steps,
+        // survivors compacted into a list), pass 2 (survivors only, all steps).
+        const char *hz_env = getenv("SMILESS_HORIZON");
+        i64 horizon = hz_env ? atoll(hz_env) : 128;
+        horizon = horizon / rp.K * rp.K;
+        const bool compact = pp.prune && horizon > 0 && horizon < n_steps;
+        const u64 claims_per_launch = compact ? ((u64)1 << 24) : ((u64)1 << 28);   // units
+        if (compact) {
+            CK(ctx->dList.ensure((size_t)claims_per_launch), "cudaMalloc list");
+            CK(ctx->dListCnt.ensure(1), "cudaMalloc");
+        }
         CK(cudaEventRecord(ctx->ev[1], st), "event");
         for (u64 q0 = 0; q0 < claims_total; q0 += claims_per_launch) {
             const u64 q1 = std::min(claims_total, q0 + claims_per_launch);
             CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
             pp.claims_begin = q0;
             pp.claims_end = q1;
+            pp.list_in = nullptr;
+            pp.list_n = nullptr;
+            pp.list_out = nullptr;
+            pp.list_cnt = nullptr;
+            pp.horizon = 0;
+            if (compact) {
+                CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
+                pp.list_out = ctx->dList.p;
+                pp.list_cnt = ctx->dListCnt.p;
+                pp.list_base = ub + (q0 / kChunkUnits * (u64)n_shards + (u64)shard) * kChunkUnits;
+                pp.horizon = horizon;
+            }
             void *args[] = {&pp};
             CUresult r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
                                                (CUstream)st, args, nullptr);
             if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
             ++launches;
+            if (compact) {                                    // pass 2 over the survivors
+                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                pp.claims_begin = 0;
+                pp.claims_end = ~0ull;
+                pp.list_in = ctx->dList.p;
+                pp.list_n = ctx->dListCnt.p;
+                pp.list_out = nullptr;
+                pp.list_cnt = nullptr;
+                pp.horizon = 0;
+                r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
+                                          (CUstream)st, args, nullptr);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
+                ++launches;
+            }
         }
         CK(cudaEventRecord(ctx->ev[2], st), "event");
         e = smiless_dev_reduce_best(ctx->dBlk.p, grid, ctx->dRes.p, st);

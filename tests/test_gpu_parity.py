@@ -346,3 +346,30 @@ def test_bench_slice_per_candidate_costs_full_J():
     oc, ol, of = OracleProblem(p, **kw).evaluate(np.arange(lo, lo + 4096, dtype=np.uint64))
     assert_dump_matches(out, oc, of)
     assert of.any() == full.feasible
+
+
+@pytest.mark.parametrize("horizon", ["64", "128", "0"])
+def test_stream_compaction_passes_are_exact(horizon, monkeypatch):
+    """Prune mode runs pass 1 (all units, `horizon` steps, survivors compacted) and pass 2
+    (survivors, all steps).  Every candidate's cost / feasibility and the winner must not
+    depend on the horizon (0 = single pass)."""
+    monkeypatch.setenv("SMILESS_HORIZON", horizon)
+    rng = np.random.default_rng(31)
+    n_checked = 0
+    for t in range(40):
+        n = int(rng.integers(2, 6))
+        p = W.random_problem(rng, n, 3, int(rng.integers(2, 5)), int(rng.integers(130, 400)),
+                             sla_us=int(rng.integers(20_000, 60_000)))
+        space = p.space_size()
+        if space > 20000:
+            continue
+        pl = S.planner_for(p)
+        out = np.empty(space)
+        g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, cost_out=out)
+        o = OracleProblem(p)
+        oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
+        assert_dump_matches(out, oc, of)
+        assert_same_plan(g, o.plan(), o)
+        assert g.n_decided == space
+        n_checked += 1
+    assert n_checked > 15
