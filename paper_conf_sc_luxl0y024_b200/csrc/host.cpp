@@ -151,11 +151,34 @@ struct PlanParamsHost {
     int zero;
     const unsigned *list_in;
     const unsigned *list_n;
+    u64 list_upp;
     unsigned *list_out;
     unsigned *list_cnt;
     u64 list_base;
     i64 horizon;
     int fixed[SMILESS_MAX_FUNCS];  // evaluator uses SM_NFIXED_ALLOC <= SMILESS_MAX_FUNCS; extra tail is ignored
+};
+
+// Mirror of BoundParams (evaluator.cuh, B&B pre-pass kernel).
+struct BoundParamsHost {
+    const int *tabNI;
+    const int *tabT;
+    const void *off;
+    u64 *counter;
+    u64 *stats;
+    unsigned *list_out;
+    unsigned *list_cnt;
+    u64 prefix_begin, prefix_end;
+    u64 cands_per_prefix;
+    u64 cand_begin, cand_end;
+    i64 n_steps;
+    i64 n_off;
+    int sumM;
+    int sla;
+    int prune_check;
+    int zero;
+    int nimin[SMILESS_MAX_FUNCS];
+    int fixed[SMILESS_MAX_FUNCS];
 };
 
 constexpr int kThreads = 256;
@@ -164,8 +187,9 @@ constexpr int kChunkUnits = 256;     // sharding / claim granularity in units (m
 struct JitKernel {
     CUmodule mod = nullptr;
     CUfunction fn = nullptr;
-    size_t smem = 0;
-    int blocks_per_sm = 0;
+    CUfunction fn_bound = nullptr;
+    size_t smem = 0, smem_bound = 0;
+    int blocks_per_sm = 0, blocks_bound = 0;
     int regs = 0;
     size_t params_size = 0;
 };
@@ -410,6 +434,35 @@ int configs_per_lane(const smiless_ctx *ctx, const smiless_plan_args *a) {
     return G;
 }
 
+// Branch-and-bound depth D (functions 0..D-1 assigned per prefix, D..N-1 relaxed), or 0 for
+// no pre-pass: prune mode, a large space, and a subtree of >= 4096 candidates per prefix.
+// SMILESS_BB_DEPTH overrides (0 disables).
+int bb_depth(const smiless_ctx *ctx, const smiless_plan_args *a) {
+    if (a->flags & SMILESS_FLAG_NO_PRUNE) return 0;
+    const int N = ctx->N, W = a->n_windows, nf = a->n_fixed;
+    const char *env = getenv("SMILESS_BB_DEPTH");
+    if (env) {
+        const int d = atoi(env);
+        return (d > nf && d <= N - 1) ? d : 0;
+    }
+    u64 space = 1;
+    for (int k = nf; k < N; ++k) space *= (u64)ctx->M[k] * (u64)W;
+    if (N < 3 || space < ((u64)1 << 26)) return 0;
+    int best = 0;
+    unsigned __int128 sub = (u64)ctx->M[N - 1] * (u64)W;
+    for (int d = N - 2; d > nf; --d) {
+        sub *= (u64)ctx->M[d] * (u64)W;                  // candidates per prefix of depth d
+        if (sub >= 4096) { best = d; break; }
+    }
+    return best;
+}
+
+u64 cands_per_prefix(const smiless_ctx *ctx, const smiless_plan_args *a, int d) {
+    u64 s = 1;
+    for (int k = d; k < ctx->N; ++k) s *= (u64)ctx->M[k] * (u64)a->n_windows;
+    return s;
+}
+
 std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, bool off_smem,
                             int minb) {
     const int N = ctx->N, W = a->n_windows, NU = N - 1, nf = a->n_fixed;
@@ -429,6 +482,8 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     const char *ck_env = getenv("SMILESS_CHECK");     // SLA early-exit check period (steps)
     const int check = std::max(unroll, ck_env ? atoi(ck_env) : 16);
     s << "#define SM_CHECK " << check << "\n";
+    const int D = bb_depth(ctx, a);
+    s << "#define SM_D " << (D > 0 ? D : N - 1) << "\n#define SMILESS_MAXF " << SMILESS_MAX_FUNCS << "\n";
     // compile-time window grid (immediates) and a constant-bank copy for runtime indices
     s << "#define SM_WIN(v) (";
     for (int v = 0; v < W; ++v) s << "(v)==" << v << "?" << a->windows_us[v] << ":";
@@ -453,6 +508,7 @@ static __device__ __forceinline__ tm_t vaddmin(tm_t a, tm_t b, tm_t c);
 static __device__ __forceinline__ tm_t opaque_add(tm_t a, tm_t b);
 static __device__ __forceinline__ tm_t opaque_sub(tm_t a, tm_t b);
 static __device__ __forceinline__ tm_t vaddmax(tm_t a, tm_t b, tm_t c);
+static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
 )";
     // ---- decode: unit u -> digits (function N-1: config only) -------------------------
     s << "static __device__ __forceinline__ void dag_decode(u64 u, int (&dig)[SM_N], const int *fixed) {\n";
@@ -505,6 +561,39 @@ static __device__ __forceinline__ tm_t vaddmax(tm_t a, tm_t b, tm_t c);
     for (int k = 0; k < N - 1; ++k)
         if ((ctx->sinkmask >> k) & 1ull) s << "  nlu = vaddmin(NF[" << k << "], o, nlu);\n";
     s << "  (void)NF; (void)o; (void)nlu;\n}\n";
+    // ---- B&B pre-pass (smiless_bound_kernel): prefix decode, relaxed first/step ---------------
+    {
+        const int Dg = D > 0 ? D : N - 1;
+        s << "static __device__ __forceinline__ void dag_bdecode(u64 u, int (&dig)[SM_N], const int *fixed) {\n";
+        for (int k = 0; k < N; ++k) s << "  dig[" << k << "] = 0;\n";
+        for (int k = Dg - 1; k >= nf; --k) {
+            const u64 radix = (u64)ctx->M[k] * (u64)W;
+            s << "  dig[" << k << "] = (int)(u % " << radix << "ull); u /= " << radix << "ull;\n";
+        }
+        for (int k = 0; k < nf; ++k) s << "  dig[" << k << "] = fixed[" << k << "];\n";
+        s << "  (void)u; (void)fixed;\n}\n";
+        s << "template <int A> static __device__ __forceinline__ void dag_bfirst(tm_t (&NF)[A], const tm_t (&NI)[A], "
+             "tm_t &nl, const tm_t z) {\n";
+        for (int k = 0; k < N; ++k)
+            s << "  NF[" << k << "] = NI[" << k << "] + " << (is_src(k) ? std::string("(tm_t)0") : nf_min(k)) << ";\n";
+        for (int k = 0; k < N; ++k)
+            if ((ctx->sinkmask >> k) & 1ull) s << "  nl = vminz(nl, NF[" << k << "], z);\n";
+        s << "  (void)z;\n}\n";
+        s << "template <int A> static __device__ __forceinline__ void dag_bstep(tm_t (&NF)[A], const tm_t (&NI)[A], "
+             "const tm_t (&Te)[A], const tm_t (&Wn)[A], const tm_t o, tm_t &nl, const tm_t z) {\n  tm_t su = 0;\n";
+        for (int k = 0; k < N; ++k) {
+            const std::string g = is_src(k) ? "o + NF[" + std::to_string(k) + "]"
+                                            : "NF[" + std::to_string(k) + "] - " + nf_min(k);
+            if (k < Dg)
+                s << "  fstep(NF[" << k << "], su, " << g << ", NI[" << k << "], Te[" << k << "], Wn[" << k << "]);\n";
+            else   // relaxed: keep-alive (start - f = max(g, 0)) with the smallest exec time
+                s << "  { const tm_t g = " << g << "; NF[" << k << "] = NF[" << k << "] + NI[" << k
+                  << "] - vmax(g, (tm_t)0); }\n";
+        }
+        for (int k = 0; k < N; ++k)
+            if ((ctx->sinkmask >> k) & 1ull) s << "  nl = vaddmin(NF[" << k << "], o, nl);\n";
+        s << "  (void)su; (void)Te; (void)Wn; (void)z;\n}\n";
+    }
     return s.str();
 }
 
@@ -574,6 +663,19 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
         r = driver().occupancy(&jk.blocks_per_sm, jk.fn, kThreads, jk.smem);
         if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuOccupancyMaxActiveBlocksPerMultiprocessor");
         if (jk.blocks_per_sm < 1) return fail(ctx, SMILESS_ECUDA, "evaluator does not fit on an SM (smem %zu)", jk.smem);
+        r = driver().moduleGetFunction(&jk.fn_bound, jk.mod, "smiless_bound_kernel");
+        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound)");
+        {
+            const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
+            jk.smem_bound = 2 * padI * 4 + (rp.time64 ? 8 : 4) * (size_t)n_off;
+            if (jk.smem_bound <= 227 * 1024) {
+                r = driver().funcSetAttribute(jk.fn_bound, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
+                                              (int)jk.smem_bound);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(bound smem)");
+                r = driver().occupancy(&jk.blocks_bound, jk.fn_bound, kThreads, jk.smem_bound);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(bound)");
+            }
+        }
         it = ctx->jit_cache.emplace(src, jk).first;
     }
     *out = &it->second;
@@ -903,54 +1005,120 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
             CK(cudaMemsetAsync(ctx->dDump.p, 0xff, (size_t)(ce - cb) * sizeof(double), st), "memset dump");  // NaN
             pp.dump = ctx->dDump.p;
         }
-        // split very large ranges into several launches (bounded kernel duration).  Prune mode
-        // with J - 1 > horizon runs each batch twice: pass 1 (every unit, `horizon` steps,
-        // survivors compacted into a list), pass 2 (survivors only, all steps).
-        const char *hz_env = getenv("SMILESS_HORIZON");
-        i64 horizon = hz_env ? atoll(hz_env) : 128;
-        horizon = horizon / rp.K * rp.K;
-        const bool compact = pp.prune && horizon > 0 && horizon < n_steps;
-        const u64 claims_per_launch = compact ? ((u64)1 << 24) : ((u64)1 << 28);   // units
-        if (compact) {
-            CK(ctx->dList.ensure((size_t)claims_per_launch), "cudaMalloc list");
+        const int D = bb_depth(ctx, a);
+        pp.list_upp = 1;
+        if (D > 0 && jk->blocks_bound > 0) {
+            // ---- exact branch-and-bound: prefixes of functions n_fixed..D-1, then list mode ----
+            const u64 S = cands_per_prefix(ctx, a, D);
+            const u64 upp = S / V;                            // evaluator units per prefix
+            const u64 p_lo = cb / S, p_hi = (ce + S - 1) / S;
+            const u64 batch = (u64)1 << 22;                   // prefixes per bound launch
+            CK(ctx->dList.ensure((size_t)batch), "cudaMalloc list");
             CK(ctx->dListCnt.ensure(1), "cudaMalloc");
-        }
-        CK(cudaEventRecord(ctx->ev[1], st), "event");
-        for (u64 q0 = 0; q0 < claims_total; q0 += claims_per_launch) {
-            const u64 q1 = std::min(claims_total, q0 + claims_per_launch);
-            CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-            pp.claims_begin = q0;
-            pp.claims_end = q1;
-            pp.list_in = nullptr;
-            pp.list_n = nullptr;
-            pp.list_out = nullptr;
-            pp.list_cnt = nullptr;
-            pp.horizon = 0;
-            if (compact) {
-                CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
-                pp.list_out = ctx->dList.p;
-                pp.list_cnt = ctx->dListCnt.p;
-                pp.list_base = ub + (q0 / kChunkUnits * (u64)n_shards + (u64)shard) * kChunkUnits;
-                pp.horizon = horizon;
+            BoundParamsHost bp;
+            memset(&bp, 0, sizeof bp);
+            bp.tabNI = ctx->dNI.p;
+            bp.tabT = ctx->dT.p;
+            bp.off = ctx->dOff.p;
+            bp.counter = ctx->dCounter.p;
+            bp.stats = ctx->dStats.p;
+            bp.list_out = ctx->dList.p;
+            bp.list_cnt = ctx->dListCnt.p;
+            bp.cands_per_prefix = S;
+            bp.cand_begin = cb;
+            bp.cand_end = ce;
+            bp.n_steps = n_steps;
+            bp.n_off = n_off;
+            bp.sumM = ctx->sumM;
+            bp.sla = (int)a->sla_us;
+            bp.zero = 0;
+            for (int k = 0; k < ctx->N; ++k) {
+                int m = ctx->I[ctx->row0[k]];
+                for (int c = 1; c < ctx->M[k]; ++c) m = std::min(m, ctx->I[ctx->row0[k] + c]);
+                bp.nimin[k] = -m;
             }
-            void *args[] = {&pp};
-            CUresult r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
-                                               (CUstream)st, args, nullptr);
-            if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
-            ++launches;
-            if (compact) {                                    // pass 2 over the survivors
+            for (int k = 0; k < a->n_fixed; ++k) bp.fixed[k] = a->fixed_digits[k];
+            const int grid_b = jk->blocks_bound * ctx->n_sms;
+            CK(cudaEventRecord(ctx->ev[1], st), "event");
+            u64 bi = 0;
+            for (u64 b0 = p_lo; b0 < p_hi; b0 += batch, ++bi) {
+                if (bi % (u64)n_shards != (u64)shard) continue;
+                const u64 b1 = std::min(p_hi, b0 + batch);
+                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
+                bp.prefix_begin = b0;
+                bp.prefix_end = b1;
+                void *bargs[] = {&bp};
+                CUresult r = driver().launchKernel(jk->fn_bound, (unsigned)grid_b, 1, 1, kThreads, 1, 1,
+                                                   (unsigned)jk->smem_bound, (CUstream)st, bargs, nullptr);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "bound launch");
+                ++launches;
                 CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
                 pp.claims_begin = 0;
                 pp.claims_end = ~0ull;
                 pp.list_in = ctx->dList.p;
                 pp.list_n = ctx->dListCnt.p;
+                pp.list_upp = upp;
+                pp.list_base = b0 * upp;
                 pp.list_out = nullptr;
                 pp.list_cnt = nullptr;
                 pp.horizon = 0;
+                void *args[] = {&pp};
                 r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
                                           (CUstream)st, args, nullptr);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
                 ++launches;
+            }
+        } else {
+            // split very large ranges into several launches (bounded kernel duration).  Prune mode
+            // with J - 1 > horizon runs each batch twice: pass 1 (every unit, `horizon` steps,
+            // survivors compacted into a list), pass 2 (survivors only, all steps).
+            const char *hz_env = getenv("SMILESS_HORIZON");
+            i64 horizon = hz_env ? atoll(hz_env) : 128;
+            horizon = horizon / rp.K * rp.K;
+            const bool compact = pp.prune && horizon > 0 && horizon < n_steps;
+            const u64 claims_per_launch = compact ? ((u64)1 << 24) : ((u64)1 << 28);   // units
+            if (compact) {
+                CK(ctx->dList.ensure((size_t)claims_per_launch), "cudaMalloc list");
+                CK(ctx->dListCnt.ensure(1), "cudaMalloc");
+            }
+            CK(cudaEventRecord(ctx->ev[1], st), "event");
+            for (u64 q0 = 0; q0 < claims_total; q0 += claims_per_launch) {
+                const u64 q1 = std::min(claims_total, q0 + claims_per_launch);
+                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                pp.claims_begin = q0;
+                pp.claims_end = q1;
+                pp.list_in = nullptr;
+                pp.list_n = nullptr;
+                pp.list_out = nullptr;
+                pp.list_cnt = nullptr;
+                pp.horizon = 0;
+                if (compact) {
+                    CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
+                    pp.list_out = ctx->dList.p;
+                    pp.list_cnt = ctx->dListCnt.p;
+                    pp.list_base = ub + (q0 / kChunkUnits * (u64)n_shards + (u64)shard) * kChunkUnits;
+                    pp.horizon = horizon;
+                }
+                void *args[] = {&pp};
+                CUresult r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
+                                                   (CUstream)st, args, nullptr);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
+                ++launches;
+                if (compact) {                                    // pass 2 over the survivors
+                    CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                    pp.claims_begin = 0;
+                    pp.claims_end = ~0ull;
+                    pp.list_in = ctx->dList.p;
+                    pp.list_n = ctx->dListCnt.p;
+                    pp.list_out = nullptr;
+                    pp.list_cnt = nullptr;
+                    pp.horizon = 0;
+                    r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
+                                              (CUstream)st, args, nullptr);
+                    if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
+                    ++launches;
+                }
             }
         }
         CK(cudaEventRecord(ctx->ev[2], st), "event");

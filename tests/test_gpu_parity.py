@@ -373,3 +373,40 @@ def test_stream_compaction_passes_are_exact(horizon, monkeypatch):
         assert g.n_decided == space
         n_checked += 1
     assert n_checked > 15
+
+
+def test_branch_and_bound_prefix_pruning_is_exact(monkeypatch):
+    """The B&B pre-pass (prefixes of D functions, the rest relaxed to keep-alive at their
+    fastest config) only discards infeasible subtrees: every depth gives the oracle's
+    per-candidate feasibility / cost, the same winner, and decides every candidate of the
+    range exactly once (also for misaligned ranges and interleaved shards)."""
+    rng = np.random.default_rng(47)
+    n_checked = 0
+    for t in range(40):
+        n = int(rng.integers(3, 7))
+        p = W.random_problem(rng, n, 3, int(rng.integers(2, 5)), int(rng.integers(20, 200)),
+                             sla_us=int(rng.integers(15_000, 60_000)))
+        space = p.space_size()
+        if space > 30000:
+            continue
+        o = OracleProblem(p)
+        oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
+        ref = o.plan()
+        for d in range(1, n):
+            monkeypatch.setenv("SMILESS_BB_DEPTH", str(d))
+            pl = S.planner_for(p)
+            out = np.empty(space)
+            g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, cost_out=out)
+            assert_dump_matches(out, oc, of)
+            assert_same_plan(g, ref, o)
+            assert g.n_decided == space
+            b, e = int(rng.integers(0, space // 2)), int(rng.integers(space // 2, space + 1))
+            g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, begin=b, end=e)
+            assert_same_plan(g, o.plan(begin=b, end=e), o)
+            assert g.n_decided == e - b
+            parts = [pl.plan(p.arrivals_us, p.sla_us, p.windows_us, shard=s_, n_shards=3) for s_ in range(3)]
+            assert sum(r.n_decided for r in parts) == space
+            feas = [(r.cost, r.index) for r in parts if r.feasible]
+            assert (min(feas) if feas else None) == (None if ref is None else (ref[1], ref[0]))
+        n_checked += 1
+    assert n_checked > 10
