@@ -77,6 +77,7 @@ enum {
 #define SMILESS_MAX_FUNCS 32
 #define SMILESS_MAX_WINDOWS 32
 #define SMILESS_MAX_CONFIGS 256
+#define SMILESS_MAX_SLAS 8
 
 /* Create a context bound to CUDA device `cuda_device` and stream `cuda_stream`
  * (a cudaStream_t; NULL = the legacy default stream; borrowed, not owned).
@@ -158,6 +159,15 @@ SMILESS_API int smiless_space_size(const smiless_ctx *ctx, int32_t n_windows, in
  * max_latency = -1, outputs set to -1), or an error. */
 SMILESS_API int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res,
                  int32_t *config_out, int32_t *window_out);
+
+/* SLA sweep (C4: "impact of SLA settings"): ONE evaluation of the space
+ * with one argmin key per SLA in slas[0..n_sla) (1 <= n_sla <= SMILESS_MAX_SLAS); pruning uses
+ * their maximum; a->sla_us is ignored and a->cost_out must be NULL.  res[n_sla] and, when not
+ * NULL, config_out / window_out [n_sla * n_funcs] receive each SLA's winner (index UINT64_MAX,
+ * outputs -1 for an SLA nothing meets).  Returns OK or an error. */
+SMILESS_API int smiless_plan_sla_sweep(smiless_ctx *ctx, const smiless_plan_args *a, const int64_t *slas,
+                                       int32_t n_sla, smiless_plan_result *res, int32_t *config_out,
+                                       int32_t *window_out);
 
 /* Exact int64 evaluation (no pruning, no clamping) of n explicit candidate
  * indices of the suffix space: cost, max_j L_j and feasibility per index.

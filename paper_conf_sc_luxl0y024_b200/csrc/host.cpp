@@ -156,6 +156,7 @@ struct PlanParamsHost {
     unsigned *list_cnt;
     u64 list_base;
     i64 horizon;
+    int slas[8];
     int fixed[SMILESS_MAX_FUNCS];  // evaluator uses SM_NFIXED_ALLOC <= SMILESS_MAX_FUNCS; extra tail is ignored
 };
 
@@ -252,7 +253,8 @@ struct smiless_ctx {
     DevBuf<double> dDump;
     DevBuf<unsigned> dList, dListCnt;
     DevBuf<ResBlock> dRes;
-    ResBlock *hRes = nullptr;    // pinned
+    ResBlock *hRes = nullptr;    // pinned [SMILESS_MAX_SLAS]
+    int nsla = 1;                // argmin keys of the plan being compiled (SLA sweep)
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
 
     std::map<std::string, JitKernel> jit_cache;
@@ -304,8 +306,8 @@ int ensure_device(smiless_ctx *ctx) {
     ctx->n_sms = prop.multiProcessorCount;
     if (!driver().ok) return fail(ctx, SMILESS_ECUDA, "CUDA driver API: %s", driver().why.c_str());
     for (auto &ev : ctx->ev) CK(cudaEventCreate(&ev), "cudaEventCreate");
-    CK(cudaMallocHost((void **)&ctx->hRes, sizeof(ResBlock)), "cudaMallocHost");
-    CK(ctx->dRes.ensure(1), "cudaMalloc");
+    CK(cudaMallocHost((void **)&ctx->hRes, sizeof(ResBlock) * SMILESS_MAX_SLAS), "cudaMallocHost");
+    CK(ctx->dRes.ensure(SMILESS_MAX_SLAS), "cudaMalloc");
     CK(ctx->dScal.ensure(2), "cudaMalloc");
     CK(ctx->dErr.ensure(1), "cudaMalloc");
     CK(ctx->dCounter.ensure(1), "cudaMalloc");
@@ -484,6 +486,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_CHECK " << check << "\n";
     const int D = bb_depth(ctx, a);
     s << "#define SM_D " << (D > 0 ? D : N - 1) << "\n#define SMILESS_MAXF " << SMILESS_MAX_FUNCS << "\n";
+    s << "#define SM_NSLA " << ctx->nsla << "\n";
     // compile-time window grid (immediates) and a constant-bank copy for runtime indices
     s << "#define SM_WIN(v) (";
     for (int v = 0; v < W; ++v) s << "(v)==" << v << "?" << a->windows_us[v] << ":";
@@ -922,13 +925,26 @@ int smiless_evaluate(smiless_ctx *ctx, const smiless_plan_args *a, const uint64_
     return SMILESS_OK;
 }
 
-int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res, int32_t *config_out,
-                 int32_t *window_out) {
-    if (!ctx) return SMILESS_EINVAL;
-    ctx->err.clear();
-    if (!res) return fail(ctx, SMILESS_EINVAL, "res is NULL");
+}  // extern "C"
+
+namespace {
+
+// The hot path.  n_sla = 1: an ordinary plan with a->sla_us.  n_sla > 1: one evaluation of the
+// space, one argmin key per SLA in slas[] (pruning against their maximum); a->sla_us is ignored.
+int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, int n_sla, smiless_plan_result *res,
+              int32_t *config_out, int32_t *window_out) {
+    if (!a_in) return fail(ctx, SMILESS_EINVAL, "args is NULL");
+    smiless_plan_args a_copy = *a_in;
+    i64 sla_max = slas[0];
+    for (int s_ = 1; s_ < n_sla; ++s_) sla_max = std::max<i64>(sla_max, slas[s_]);
+    a_copy.sla_us = sla_max;
+    const smiless_plan_args *a = &a_copy;
     int rc = validate_args(ctx, a, true);
     if (rc) return rc;
+    for (int s_ = 0; s_ < n_sla; ++s_)
+        if (slas[s_] < 0 || slas[s_] >= (1ll << 29)) return fail(ctx, SMILESS_EINVAL, "sla out of [0, 2^29)");
+    ctx->nsla = n_sla;
+    struct NslaReset { smiless_ctx *c; ~NslaReset() { c->nsla = 1; } } nsla_reset{ctx};
     u64 space;
     space_size_of(ctx, a->n_windows, a->n_fixed, &space);
     const u64 cb = a->begin;
@@ -953,7 +969,7 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
     const size_t tsz = rp.time64 ? 8 : 4;
     CK(ctx->dOff.ensure((size_t)n_off * tsz), "cudaMalloc offsets");
     CK(cudaMemsetAsync(ctx->dErr.p, 0, sizeof(int), st), "memset");
-    CK(cudaMemsetAsync(ctx->dRes.p, 0xff, sizeof(ResBlock), st), "memset");
+    CK(cudaMemsetAsync(ctx->dRes.p, 0xff, sizeof(ResBlock) * n_sla, st), "memset");
     int e = smiless_dev_prep_offsets(d_arr, a->n_arrivals, rp.d_cap, rp.K, rp.time64 ? 1 : 0, ctx->dOff.p, n_off,
                                      ctx->dScal.p, ctx->dErr.p, st);
     if (e) return cuda_fail(ctx, (cudaError_t)e, "prep_offsets launch");
@@ -972,8 +988,8 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
         const u64 my_chunks = n_chunks > (u64)shard ? (n_chunks - 1 - (u64)shard) / (u64)n_shards + 1 : 0;
         const u64 claims_total = my_chunks * (u64)kChunkUnits;
         const int grid = jk->blocks_per_sm * ctx->n_sms;
-        CK(ctx->dBlk.ensure((size_t)grid * 2), "cudaMalloc");
-        CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid * 16, st), "memset");
+        CK(ctx->dBlk.ensure((size_t)grid * 2 * n_sla), "cudaMalloc");
+        CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid * 16 * n_sla, st), "memset");
         CK(cudaMemsetAsync(ctx->dStats.p, 0, 16, st), "memset");
         PlanParamsHost pp;
         memset(&pp, 0, sizeof pp);
@@ -995,6 +1011,7 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
         pp.n_off = n_off;
         pp.sumM = ctx->sumM;
         pp.sla = (int)a->sla_us;
+        for (int s_ = 0; s_ < n_sla; ++s_) pp.slas[s_] = (int)slas[s_];
         pp.prune = (a->flags & SMILESS_FLAG_NO_PRUNE) ? 0 : 1;
         pp.shard = shard;
         pp.n_shards = n_shards;
@@ -1122,33 +1139,38 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
             }
         }
         CK(cudaEventRecord(ctx->ev[2], st), "event");
-        e = smiless_dev_reduce_best(ctx->dBlk.p, grid, ctx->dRes.p, st);
-        if (e) return cuda_fail(ctx, (cudaError_t)e, "reduce launch");
-        ++launches;
+        for (int s_ = 0; s_ < n_sla; ++s_) {
+            e = smiless_dev_reduce_best(ctx->dBlk.p + 2 * s_, grid, n_sla, ctx->dRes.p + s_, st);
+            if (e) return cuda_fail(ctx, (cudaError_t)e, "reduce launch");
+            ++launches;
+        }
         CK(cudaMemcpyAsync(&ctx->dRes.p->stats[0], ctx->dStats.p, 16, cudaMemcpyDeviceToDevice, st), "D2D stats");
         if (a->cost_out)
             CK(cudaMemcpyAsync(a->cost_out, ctx->dDump.p, (size_t)(ce - cb) * sizeof(double), cudaMemcpyDeviceToHost, st),
                "D2H dump");
     } else if (single && ce > cb) {
         // the space is the single candidate of the pinned digits: index 0
-        CK(cudaMemsetAsync(&ctx->dRes.p->best_c, 0, 16, st), "memset");
+        for (int s_ = 0; s_ < n_sla; ++s_) CK(cudaMemsetAsync(&ctx->dRes.p[s_].best_c, 0, 16, st), "memset");
         CK(cudaEventRecord(ctx->ev[1], st), "event");
         CK(cudaEventRecord(ctx->ev[2], st), "event");
     } else {
         CK(cudaEventRecord(ctx->ev[1], st), "event");
         CK(cudaEventRecord(ctx->ev[2], st), "event");
     }
-    // a10: exact int64 re-evaluation of the winner (also decodes its digits)
-    ExactParams ep;
-    fill_exact_params(ctx, a, d_arr, ep);
-    ep.n = 1;
-    ep.res = ctx->dRes.p;
-    ep.idx_from_res = 1;
-    e = smiless_dev_eval_exact(&ep, st);
-    if (e) return cuda_fail(ctx, (cudaError_t)e, "eval_exact launch");
-    ++launches;
+    // a10: exact int64 re-evaluation of each winner (also decodes its digits)
+    for (int s_ = 0; s_ < n_sla; ++s_) {
+        ExactParams ep;
+        fill_exact_params(ctx, a, d_arr, ep);
+        ep.sla = slas[s_];
+        ep.n = 1;
+        ep.res = ctx->dRes.p + s_;
+        ep.idx_from_res = 1;
+        e = smiless_dev_eval_exact(&ep, st);
+        if (e) return cuda_fail(ctx, (cudaError_t)e, "eval_exact launch");
+        ++launches;
+    }
     CK(cudaMemcpyAsync(&ctx->dRes.p->err, ctx->dErr.p, sizeof(int), cudaMemcpyDeviceToDevice, st), "D2D err");
-    CK(cudaMemcpyAsync(ctx->hRes, ctx->dRes.p, sizeof(ResBlock), cudaMemcpyDeviceToHost, st), "D2H result");
+    CK(cudaMemcpyAsync(ctx->hRes, ctx->dRes.p, sizeof(ResBlock) * n_sla, cudaMemcpyDeviceToHost, st), "D2H result");
     CK(cudaEventRecord(ctx->ev[3], st), "event");
     CK(cudaStreamSynchronize(st), "plan");
     float ms = 0.f, tot = 0.f;
@@ -1156,51 +1178,84 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
     cudaEventElapsedTime(&tot, ctx->ev[0], ctx->ev[3]);
     eval_ms = ms;
 
-    const ResBlock &h = *ctx->hRes;
-    if (h.err & 1) return fail(ctx, SMILESS_EINVAL, "arrivals must be non-decreasing");
-    if (h.err & 2) return fail(ctx, SMILESS_EINVAL, "arrival times out of range (|r| >= 2^62)");
+    const ResBlock &h0 = *ctx->hRes;
+    if (h0.err & 1) return fail(ctx, SMILESS_EINVAL, "arrivals must be non-decreasing");
+    if (h0.err & 2) return fail(ctx, SMILESS_EINVAL, "arrival times out of range (|r| >= 2^62)");
     if (!single && ce > cb) {
-        n_decided = h.stats[0];
-        n_full = h.stats[1];
+        n_decided = h0.stats[0];
+        n_full = h0.stats[1];
     } else if (single && ce > cb) {
         n_decided = n_full = 1;
     }
-    const bool found = h.best_i != ~0ull && h.feasible == 1;
-    if (!single && h.best_i != ~0ull && h.feasible != 1)
-        return fail(ctx, SMILESS_ECUDA, "internal: evaluator winner %llu not feasible on exact re-evaluation",
-                    (unsigned long long)h.best_i);
-    if (found && !single) {
-        double c;
-        memcpy(&c, &h.best_c, 8);
-        if (c != h.cost)
-            return fail(ctx, SMILESS_ECUDA, "internal: evaluator cost %.17g != exact %.17g for index %llu", c, h.cost,
+    int status = SMILESS_INFEASIBLE;
+    for (int s_ = 0; s_ < n_sla; ++s_) {
+        const ResBlock &h = ctx->hRes[s_];
+        const bool found = h.best_i != ~0ull && h.feasible == 1;
+        if (!single && h.best_i != ~0ull && h.feasible != 1)
+            return fail(ctx, SMILESS_ECUDA, "internal: evaluator winner %llu not feasible on exact re-evaluation",
                         (unsigned long long)h.best_i);
-    }
-    memset(res, 0, sizeof *res);
-    res->n_decided = n_decided;
-    res->n_full_evals = n_full;
-    res->eval_kernel_ms = eval_ms;
-    res->total_device_ms = tot;
-    res->int64_path = rp.time64 ? 1 : 0;
-    res->launches = launches;
-    if (!found) {
-        res->index = ~0ull;
-        res->cost = HUGE_VAL;
-        res->max_latency_us = -1;
-        for (int k = 0; k < ctx->N; ++k) {
-            if (config_out) config_out[k] = -1;
-            if (window_out) window_out[k] = -1;
+        if (found && !single) {
+            double c;
+            memcpy(&c, &h.best_c, 8);
+            if (c != h.cost)
+                return fail(ctx, SMILESS_ECUDA, "internal: evaluator cost %.17g != exact %.17g for index %llu", c,
+                            h.cost, (unsigned long long)h.best_i);
         }
-        return SMILESS_INFEASIBLE;
+        smiless_plan_result &r = res[s_];
+        memset(&r, 0, sizeof r);
+        r.n_decided = n_decided;
+        r.n_full_evals = n_full;
+        r.eval_kernel_ms = eval_ms;
+        r.total_device_ms = tot;
+        r.int64_path = rp.time64 ? 1 : 0;
+        r.launches = launches;
+        int32_t *co = config_out ? config_out + (size_t)s_ * ctx->N : nullptr;
+        int32_t *wo = window_out ? window_out + (size_t)s_ * ctx->N : nullptr;
+        if (!found) {
+            r.index = ~0ull;
+            r.cost = HUGE_VAL;
+            r.max_latency_us = -1;
+            for (int k = 0; k < ctx->N; ++k) {
+                if (co) co[k] = -1;
+                if (wo) wo[k] = -1;
+            }
+            continue;
+        }
+        if (s_ == 0) status = SMILESS_OK;
+        r.index = h.best_i;
+        r.cost = h.cost;
+        r.max_latency_us = h.maxlat;
+        for (int k = 0; k < ctx->N; ++k) {
+            if (co) co[k] = h.cfg[k];
+            if (wo) wo[k] = h.win[k];
+        }
     }
-    res->index = h.best_i;
-    res->cost = h.cost;
-    res->max_latency_us = h.maxlat;
-    for (int k = 0; k < ctx->N; ++k) {
-        if (config_out) config_out[k] = h.cfg[k];
-        if (window_out) window_out[k] = h.win[k];
-    }
-    return SMILESS_OK;
+    return status;
+}
+
+}  // namespace
+
+extern "C" {
+
+int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res, int32_t *config_out,
+                 int32_t *window_out) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->err.clear();
+    if (!res) return fail(ctx, SMILESS_EINVAL, "res is NULL");
+    if (!a) return fail(ctx, SMILESS_EINVAL, "args is NULL");
+    const i64 sla = a->sla_us;
+    return plan_impl(ctx, a, &sla, 1, res, config_out, window_out);
+}
+
+int smiless_plan_sla_sweep(smiless_ctx *ctx, const smiless_plan_args *a, const int64_t *slas, int32_t n_sla,
+                           smiless_plan_result *res, int32_t *config_out, int32_t *window_out) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->err.clear();
+    if (!res || !slas) return fail(ctx, SMILESS_EINVAL, "res / slas is NULL");
+    if (n_sla < 1 || n_sla > SMILESS_MAX_SLAS) return fail(ctx, SMILESS_EINVAL, "n_sla must be in [1, %d]", SMILESS_MAX_SLAS);
+    if (a && a->cost_out) return fail(ctx, SMILESS_EINVAL, "cost_out is not supported by the SLA sweep");
+    const int rc = plan_impl(ctx, a, (const i64 *)slas, n_sla, res, config_out, window_out);
+    return rc < 0 ? rc : SMILESS_OK;
 }
 
 // ---- introspection (build checks, SASS inspection, tests) ---------------------------------

@@ -53,11 +53,13 @@ __device__ __forceinline__ bool key_less(u64 ca, u64 ia, u64 cb, u64 ib) {
     return ca < cb || (ca == cb && ia < ib);
 }
 
-__global__ void reduce_best_kernel(const u64 *__restrict__ slots, int n, ResBlock *__restrict__ res) {
+__global__ void reduce_best_kernel(const u64 *__restrict__ slots, int n, int stride, ResBlock *__restrict__ res) {
     __shared__ u64 sc[256], si[256];
     u64 c = ~0ull, i = ~0ull;
-    for (int b = threadIdx.x; b < n; b += blockDim.x)
-        if (key_less(slots[2 * b], slots[2 * b + 1], c, i)) { c = slots[2 * b]; i = slots[2 * b + 1]; }
+    for (int b = threadIdx.x; b < n; b += blockDim.x) {
+        const u64 *sl = slots + 2 * (size_t)b * stride;
+        if (key_less(sl[0], sl[1], c, i)) { c = sl[0]; i = sl[1]; }
+    }
     sc[threadIdx.x] = c;
     si[threadIdx.x] = i;
     __syncthreads();
@@ -177,8 +179,8 @@ int smiless_dev_prep_offsets(const long long *arr, long long J, long long d_cap,
     return (int)cudaGetLastError();
 }
 
-int smiless_dev_reduce_best(const unsigned long long *slots, int n, ResBlock *res, cudaStream_t st) {
-    smiless_dev::reduce_best_kernel<<<1, 256, 0, st>>>(slots, n, res);
+int smiless_dev_reduce_best(const unsigned long long *slots, int n, int stride, ResBlock *res, cudaStream_t st) {
+    smiless_dev::reduce_best_kernel<<<1, 256, 0, st>>>(slots, n, stride, res);
     return (int)cudaGetLastError();
 }
 

@@ -25,7 +25,8 @@ _NAMES = {0: "OK", 1: "INFEASIBLE", -1: "EINVAL", -2: "ENOTTOPO", -3: "ERANGE", 
 # every symbol include/smiless.h declares (checked by tests/test_abi.py)
 EXPORTS = ("smiless_create", "smiless_set_stream", "smiless_destroy", "smiless_last_error",
            "smiless_load_dag", "smiless_load_profiles", "smiless_space_size", "smiless_plan",
-           "smiless_evaluate", "smiless_decode", "smiless_kernel_source", "smiless_jit_compile")
+           "smiless_plan_sla_sweep", "smiless_evaluate", "smiless_decode", "smiless_kernel_source",
+           "smiless_jit_compile")
 
 
 class SmilessError(RuntimeError):
@@ -110,6 +111,8 @@ def load_library(build_if_missing: bool = True):
     lib.smiless_load_profiles.argtypes = [vp, vp, vp, vp, vp]
     lib.smiless_space_size.argtypes = [vp, i32, i32, ctypes.POINTER(u64)]
     lib.smiless_plan.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.POINTER(PlanResultC), vp, vp]
+    lib.smiless_plan_sla_sweep.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i32, ctypes.POINTER(PlanResultC),
+                                           vp, vp]
     lib.smiless_evaluate.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i64, vp, vp, vp]
     lib.smiless_decode.argtypes = [vp, i32, u64, ctypes.POINTER(PlanArgs), vp, vp]
     lib.smiless_kernel_source.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.c_char_p, ctypes.c_size_t,
@@ -224,6 +227,28 @@ class Planner:
                           window=win[:self.n_funcs], n_decided=int(r.n_decided), n_full_evals=int(r.n_full_evals),
                           eval_kernel_ms=float(r.eval_kernel_ms), total_device_ms=float(r.total_device_ms),
                           int64_path=bool(r.int64_path), launches=int(r.launches))
+
+    def plan_sla_sweep(self, arrivals, slas_us, windows_us, **kw):
+        """One pass over the space, one winner per SLA (smiless_plan_sla_sweep)."""
+        sl = np.ascontiguousarray(np.asarray(slas_us, dtype=np.int64))
+        n = int(sl.shape[0])
+        a, keep = self._args(arrivals, int(sl.max()), windows_us, **kw)
+        rs = (PlanResultC * n)()
+        cfg = np.zeros((n, max(self.n_funcs, 1)), np.int32)
+        win = np.zeros((n, max(self.n_funcs, 1)), np.int32)
+        self._check(self._lib.smiless_plan_sla_sweep(self._ctx, ctypes.byref(a), sl.ctypes.data, n, rs,
+                                                     cfg.ctypes.data, win.ctypes.data))
+        del keep
+        out = []
+        for i, r in enumerate(rs):
+            feas = r.index != (1 << 64) - 1
+            out.append(PlanResult(status=OK if feas else INFEASIBLE, index=int(r.index) if feas else None,
+                                  cost=float(r.cost), max_latency_us=int(r.max_latency_us),
+                                  config=cfg[i, :self.n_funcs], window=win[i, :self.n_funcs],
+                                  n_decided=int(r.n_decided), n_full_evals=int(r.n_full_evals),
+                                  eval_kernel_ms=float(r.eval_kernel_ms), total_device_ms=float(r.total_device_ms),
+                                  int64_path=bool(r.int64_path), launches=int(r.launches)))
+        return out
 
     def evaluate(self, idx, arrivals, sla_us, windows_us, **kw) -> Tuple[np.ndarray, np.ndarray, np.ndarray]:
         a, keep = self._args(arrivals, sla_us, windows_us, **kw)

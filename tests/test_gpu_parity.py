@@ -410,3 +410,43 @@ def test_branch_and_bound_prefix_pruning_is_exact(monkeypatch):
             assert (min(feas) if feas else None) == (None if ref is None else (ref[1], ref[0]))
         n_checked += 1
     assert n_checked > 10
+
+
+# ---------------------------------------------------------------------------------------
+# C4: SLA sweep in one pass (one argmin key per SLA)
+# ---------------------------------------------------------------------------------------
+
+def test_sla_sweep_matches_per_sla_oracle_plans():
+    slas = W.C4_SLAS_US
+    p = W.make_config("C4")
+    Wn = len(p.windows_us)
+    pl = S.planner_for(p)
+    rng = np.random.default_rng(4)
+    for trial in range(3):
+        nf = 3
+        fixed = [(7 if trial == 0 else int(rng.integers(0, 8))) * Wn + int(rng.integers(0, Wn)) for _ in range(nf)]
+        rs = pl.plan_sla_sweep(p.arrivals_us, slas, p.windows_us, n_fixed=nf, fixed_digits=fixed)
+        prev = None
+        for sla, g in zip(slas, rs):
+            o = OracleProblem(p.replace(sla_us=sla), n_fixed=nf, fixed_digits=fixed)
+            assert_same_plan(g, o.plan(), o)
+            single = pl.plan(p.arrivals_us, sla, p.windows_us, n_fixed=nf, fixed_digits=fixed)
+            assert (single.index, single.cost) == (g.index, g.cost)
+            if prev is not None and prev.feasible:       # OPT non-increasing in the SLA
+                assert g.feasible and g.cost <= prev.cost
+            prev = g
+
+
+def test_sla_sweep_random_dags():
+    rng = np.random.default_rng(5)
+    for t in range(25):
+        n = int(rng.integers(1, 6))
+        p = W.random_problem(rng, n, 3, int(rng.integers(1, 5)), int(rng.integers(1, 90)))
+        if p.space_size() > 20000:
+            continue
+        slas = sorted(set(int(v) for v in rng.integers(1_000, 40_000, size=int(rng.integers(2, 8)))))
+        pl = S.planner_for(p)
+        rs = pl.plan_sla_sweep(p.arrivals_us, slas, p.windows_us)
+        for sla, g in zip(slas, rs):
+            o = OracleProblem(p.replace(sla_us=sla))
+            assert_same_plan(g, o.plan(), o)
