@@ -239,6 +239,7 @@ def main():
     ap.add_argument("--no-pruned", action="store_true")
     ap.add_argument("--no-full-space", action="store_true",
                     help="skip the exhaustive pruned plan of the whole workload space (time-to-optimal)")
+    ap.add_argument("--no-c4", action="store_true", help="skip the C4 SLA-sweep re-planning rate")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -363,6 +364,32 @@ def main():
             c, w = pl.decode(g_idx, len(p.windows_us))
             full["config"], full["window"] = c.tolist(), w.tolist()
 
+    # C4 (configs[3]): 1,000 re-plans of 100 predicted arrivals, 6 SLAs per pass, exhaustive each
+    c4 = None
+    if not args.no_c4 and world == 1:
+        p4 = W.make_config("C4")
+        pl4 = S.planner_for(p4, device=local, stream=stream.cuda_stream)
+        wins = [torch.as_tensor(w).to(dev) for w in W.c4_replans(1000)]
+        pl4.plan_sla_sweep(wins[0], W.C4_SLAS_US, p4.windows_us)
+        barrier()
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        feas = [0] * len(W.C4_SLAS_US)
+        mono = True
+        for w in wins:
+            rs = pl4.plan_sla_sweep(w, W.C4_SLAS_US, p4.windows_us)
+            cs = [r.cost if r.feasible else float("inf") for r in rs]
+            mono &= all(cs[i + 1] <= cs[i] for i in range(len(cs) - 1))
+            for i, r in enumerate(rs):
+                feas[i] += r.feasible
+        b.record(stream)
+        torch.cuda.synchronize(dev)
+        sec = a.elapsed_time(b) / 1e3
+        c4 = {"replans": len(wins), "slas": W.C4_SLAS_US, "candidates_per_replan": pl4.space_size(len(p4.windows_us)),
+              "replans_per_s": len(wins) / sec, "seconds": sec, "feasible_per_sla": feas,
+              "opt_non_increasing_in_sla": bool(mono)}
+
     if rank != 0:
         if world > 1:
             dist.destroy_process_group()
@@ -387,6 +414,7 @@ def main():
                    "config": res.config.tolist(), "window": res.window.tolist()} if world == 1 else None,
         "pruned": pruned,
         "time_to_optimal_full_space": full,
+        "c4_sla_sweep_replanning": c4,
         "gpu_launches": launches,
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(p.arrivals_us.nbytes),
                 "d2h_bytes_per_step": 312},

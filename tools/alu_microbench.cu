@@ -42,9 +42,17 @@ __global__ void __launch_bounds__(256) bench(int *out, int seed) {
                 asm volatile("mad.lo.s32 %0, %1, %2, %3;" : "=r"(x) : "r"(x), "r"(b), "r"(c));
                 asm volatile("{.reg .s32 t; add.s32 t, %1, %2; max.s32 %0, t, %3;}" : "=r"(x) : "r"(x), "r"(b), "r"(c));
             }
-            if (OP == 6) {  // plain 2-input add / sub
-                asm volatile("add.s32 %0, %1, %2;" : "=r"(x) : "r"(x), "r"(b));
-                asm volatile("sub.s32 %0, %1, %2;" : "=r"(x) : "r"(x), "r"(c));
+            if (OP == 6) {  // IMAD.HI (high word of a signed 32x32 product)
+                asm volatile("mul.hi.s32 %0, %1, %2;" : "=r"(x) : "r"(x), "r"(b));
+                asm volatile("mad.hi.s32 %0, %1, %2, %3;" : "=r"(x) : "r"(x), "r"(c), "r"(b));
+            }
+            if (OP == 7) {  // IMAD.HI + VIADDMNMX
+                asm volatile("mul.hi.s32 %0, %1, %2;" : "=r"(x) : "r"(x), "r"(b));
+                asm volatile("{.reg .s32 t; add.s32 t, %1, %2; max.s32 %0, t, %3;}" : "=r"(x) : "r"(x), "r"(b), "r"(c));
+            }
+            if (OP == 8) {  // IMAD.IADD-style adds forced onto the FMA pipe: x * 1 + b
+                asm volatile("mad.lo.s32 %0, %1, 1, %2;" : "=r"(x) : "r"(x), "r"(b));
+                asm volatile("mad.lo.s32 %0, %1, 1, %2;" : "=r"(x) : "r"(x), "r"(c));
             }
             a[i] = x;
         }
@@ -95,6 +103,9 @@ int main() {
     run<3>("IMAD", 2, blocks, hz, sms);
     run<4>("ISETP+SEL", 2, blocks, hz, sms);
     run<5>("IMAD+VIADDMNMX", 2, blocks, hz, sms);
+    run<6>("IMAD.HI", 2, blocks, hz, sms);
+    run<7>("IMAD.HI+VIADDMNMX", 2, blocks, hz, sms);
+    run<8>("IMAD.IADD(x*1+b)", 2, blocks, hz, sms);
 
     return 0;
 }
