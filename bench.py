@@ -59,7 +59,7 @@ def configs_per_lane(p) -> int:
     """Mirror of host.cpp configs_per_lane (G): last-function configs carried per lane."""
     M = int(p.n_configs[-1])
     Wn = len(p.windows_us)
-    want = int(os.environ.get("SMILESS_G", "0")) or max(1, 16 // Wn)
+    want = int(os.environ.get("SMILESS_G", "0")) or max(1, 16 // Wn)   # grid windows (no row windows)
     G = 1
     for g in range(1, want + 1):
         if M % g == 0 and g * Wn <= 32:

@@ -132,6 +132,11 @@ typedef struct {
     double *cost_out;             /* optional (testing): host array [end - begin] receiving every
                                      candidate's cost as the evaluator computed it, NaN when it is
                                      infeasible or was pruned; NULL = off; end - begin <= 2^26     */
+    const int32_t *row_windows_us;/* optional [sum(n_configs)] host array: the pre-warm window of
+                                     each (function, config) row instead of a searched grid (the
+                                     paper's adaptive pre-warming; see
+                                     smiless_derive_windows); requires n_windows == 1 (windows_us
+                                     is then ignored); 0 <= w < 2^29                               */
 } smiless_plan_args;
 
 typedef struct {
@@ -159,6 +164,13 @@ SMILESS_API int smiless_space_size(const smiless_ctx *ctx, int32_t n_windows, in
  * max_latency = -1, outputs set to -1), or an error. */
 SMILESS_API int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res,
                  int32_t *config_out, int32_t *window_out);
+
+/* The paper's adaptive pre-warming window per (function, config) row for a predicted
+ * inter-arrival time it_us: Case I (T + I < IT): IT - T - I, the unloaded gap
+ * that re-loads the instance exactly when the next input arrives; Case II (T + I >= IT):
+ * 0, keep alive.  Host-only.  row_windows_out has sum(n_configs) entries.
+ * Returns OK, ESTATE or EINVAL. */
+SMILESS_API int smiless_derive_windows(const smiless_ctx *ctx, int64_t it_us, int32_t *row_windows_out);
 
 /* SLA sweep (C4: "impact of SLA settings"): ONE evaluation of the space
  * with one argmin key per SLA in slas[0..n_sla) (1 <= n_sla <= SMILESS_MAX_SLAS); pruning uses

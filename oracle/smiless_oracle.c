@@ -48,6 +48,8 @@ typedef struct {
     int32_t n_windows;
     int32_t n_fixed;             /* digits of functions 0..n_fixed-1 are pinned   */
     const int32_t *fixed_digits; /* [n_fixed] digit = config * W + window         */
+    const int32_t *row_windows;  /* optional [sum M]: the window of (k, c) itself  */
+                                 /* (NEXT-1 derived windows; then W must be 1)    */
 } oracle_problem;
 
 /* Row offset of function k in the function-major profile arrays. */
@@ -124,7 +126,7 @@ static void simulate_into(const oracle_problem *P, const int32_t *config, const 
         int64_t row = row0(P, k) + config[k];
         I[k] = P->exec_us[row];
         T[k] = P->init_us[row];
-        w[k] = P->windows_us[window[k]];
+        w[k] = P->row_windows ? P->row_windows[row] : P->windows_us[window[k]];
         billed[k] = 0;
     }
     for (int64_t j = 0; j < J; ++j) {

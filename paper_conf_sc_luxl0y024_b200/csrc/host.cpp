@@ -157,6 +157,7 @@ struct PlanParamsHost {
     u64 list_base;
     i64 horizon;
     int slas[8];
+    const int *tabW;               // [sumM] per-row windows (SM_ROWWIN) or a dummy table
     int fixed[SMILESS_MAX_FUNCS];  // evaluator uses SM_NFIXED_ALLOC <= SMILESS_MAX_FUNCS; extra tail is ignored
 };
 
@@ -179,6 +180,7 @@ struct BoundParamsHost {
     int prune_check;
     int zero;
     int nimin[SMILESS_MAX_FUNCS];
+    const int *tabW;
     int fixed[SMILESS_MAX_FUNCS];
 };
 
@@ -252,6 +254,7 @@ struct smiless_ctx {
     DevBuf<unsigned char> dFeas;
     DevBuf<double> dDump;
     DevBuf<unsigned> dList, dListCnt;
+    DevBuf<int> dW;                          // per-row windows of the current plan (padded)
     DevBuf<ResBlock> dRes;
     ResBlock *hRes = nullptr;    // pinned [SMILESS_MAX_SLAS]
     int nsla = 1;                // argmin keys of the plan being compiled (SLA sweep)
@@ -371,6 +374,12 @@ int validate_args(smiless_ctx *ctx, const smiless_plan_args *a, bool need_arriva
             return fail(ctx, SMILESS_EINVAL, "windows must be strictly increasing");
     }
     if (a->sla_us < 0 || a->sla_us >= (1ll << 29)) return fail(ctx, SMILESS_EINVAL, "sla_us out of [0, 2^29)");
+    if (a->row_windows_us) {
+        if (a->n_windows != 1) return fail(ctx, SMILESS_EINVAL, "row_windows_us requires n_windows == 1");
+        for (int r = 0; r < ctx->sumM; ++r)
+            if (a->row_windows_us[r] < 0 || a->row_windows_us[r] >= (1 << 29))
+                return fail(ctx, SMILESS_EINVAL, "row window %d out of [0, 2^29)", r);
+    }
     if (a->n_arrivals < 1) return fail(ctx, SMILESS_EINVAL, "n_arrivals must be >= 1");
     if (a->n_arrivals > (1ll << 31)) return fail(ctx, SMILESS_EINVAL, "n_arrivals too large");
     if (!a->arrivals_us) return fail(ctx, SMILESS_EINVAL, "arrivals_us is NULL");
@@ -407,7 +416,11 @@ struct RangePlan {
 };
 
 RangePlan range_plan(const smiless_ctx *ctx, const smiless_plan_args *a) {
-    const i64 wmax = a->windows_us[a->n_windows - 1];
+    i64 wmax = a->windows_us[a->n_windows - 1];
+    if (a->row_windows_us) {
+        wmax = 0;
+        for (int r = 0; r < ctx->sumM; ++r) wmax = std::max<i64>(wmax, a->row_windows_us[r]);
+    }
     const i64 sla = a->sla_us;
     const i64 d_cap = sla + wmax + ctx->Tmax + 1;
     RangePlan rp{true, 64, d_cap};
@@ -430,7 +443,8 @@ int configs_per_lane(const smiless_ctx *ctx, const smiless_plan_args *a) {
     const int M = ctx->M[ctx->N - 1], W = a->n_windows;
     int G = 1;
     const char *env = getenv("SMILESS_G");
-    const int want = env ? std::max(1, atoi(env)) : std::max(1, 16 / W);
+    // per-row windows carry a run-time window and Te per variant: fewer variants fit in registers
+    const int want = env ? std::max(1, atoi(env)) : (a->row_windows_us ? 8 : std::max(1, 16 / W));
     for (int g = 1; g <= want; ++g)
         if (M % g == 0 && g * W <= 32) G = g;
     return G;
@@ -479,7 +493,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_K " << rp.K << "\n#define SM_TIME64 " << (rp.time64 ? 1 : 0) << "\n";
     s << "#define SM_OFF_SMEM " << (off_smem ? 1 : 0) << "\n#define SM_THREADS " << kThreads
       << "\n#define SM_MINB " << minb << "\n";
-    s << "#define SM_W0_ZERO " << (a->windows_us[0] == 0 ? 1 : 0) << "\n";
+    s << "#define SM_W0_ZERO " << (!a->row_windows_us && a->windows_us[0] == 0 ? 1 : 0) << "\n";
     s << "#define SM_G " << G << "\n#define SM_UNROLL " << unroll << "\n";
     const char *ck_env = getenv("SMILESS_CHECK");     // SLA early-exit check period (steps)
     const int check = std::max(unroll, ck_env ? atoi(ck_env) : 16);
@@ -487,6 +501,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     const int D = bb_depth(ctx, a);
     s << "#define SM_D " << (D > 0 ? D : N - 1) << "\n#define SMILESS_MAXF " << SMILESS_MAX_FUNCS << "\n";
     s << "#define SM_NSLA " << ctx->nsla << "\n";
+    s << "#define SM_ROWWIN " << (a->row_windows_us ? 1 : 0) << "\n";
     // compile-time window grid (immediates) and a constant-bank copy for runtime indices
     s << "#define SM_WIN(v) (";
     for (int v = 0; v < W; ++v) s << "(v)==" << v << "?" << a->windows_us[v] << ":";
@@ -634,7 +649,7 @@ size_t smem_bytes(const smiless_ctx *ctx, const smiless_plan_args *a, const Rang
     const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
     const size_t padU = (size_t)((ctx->sumM + 1) & ~1);
     const size_t tsz = rp.time64 ? 8 : 4;
-    size_t b = 2 * padI * 4 + padU * 8;
+    size_t b = 3 * padI * 4 + padU * 8;
     b += 8ull * (size_t)(ctx->N - 1 + a->n_windows * configs_per_lane(ctx, a)) * kThreads;
     b += (tsz * (size_t)ctx->N * kThreads + 15) & ~(size_t)15;
     if (off_smem) b += tsz * (size_t)n_off;
@@ -670,7 +685,7 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
         if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound)");
         {
             const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
-            jk.smem_bound = 2 * padI * 4 + (rp.time64 ? 8 : 4) * (size_t)n_off;
+            jk.smem_bound = 3 * padI * 4 + (rp.time64 ? 8 : 4) * (size_t)n_off;
             if (jk.smem_bound <= 227 * 1024) {
                 r = driver().funcSetAttribute(jk.fn_bound, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
                                               (int)jk.smem_bound);
@@ -704,7 +719,19 @@ void fill_exact_params(const smiless_ctx *ctx, const smiless_plan_args *a, const
         ep.row0[k] = ctx->row0[k];
     }
     for (int v = 0; v < a->n_windows; ++v) ep.win[v] = a->windows_us[v];
+    ep.rowwin = a->row_windows_us ? ctx->dW.p : nullptr;
     for (int k = 0; k < a->n_fixed; ++k) ep.fixed[k] = a->fixed_digits[k];
+}
+
+// Per-row windows of this call (row_windows_us) or zeros: the kernels always stage the table.
+int stage_row_windows(smiless_ctx *ctx, const smiless_plan_args *a) {
+    const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
+    std::vector<int> w(padI, 0);
+    if (a->row_windows_us) std::copy(a->row_windows_us, a->row_windows_us + ctx->sumM, w.begin());
+    CK(ctx->dW.ensure(padI), "cudaMalloc row windows");
+    CK(cudaMemcpyAsync(ctx->dW.p, w.data(), padI * sizeof(int), cudaMemcpyHostToDevice, ctx->stream), "H2D windows");
+    CK(cudaStreamSynchronize(ctx->stream), "H2D windows");
+    return SMILESS_OK;
 }
 
 // Upload (host) or adopt (device) the arrival sequence; returns the device pointer.
@@ -765,7 +792,7 @@ void smiless_destroy(smiless_ctx *ctx) {
         ctx->dArr.release(); ctx->dOff.release(); ctx->dScal.release(); ctx->dErr.release();
         ctx->dCounter.release(); ctx->dStats.release(); ctx->dBlk.release(); ctx->dIdxEval.release();
         ctx->dCost.release(); ctx->dLat.release(); ctx->dFeas.release(); ctx->dRes.release(); ctx->dDump.release();
-        ctx->dList.release(); ctx->dListCnt.release();
+        ctx->dList.release(); ctx->dListCnt.release(); ctx->dW.release();
         if (ctx->hRes) cudaFreeHost(ctx->hRes);
         for (auto &ev : ctx->ev)
             if (ev) cudaEventDestroy(ev);
@@ -903,6 +930,7 @@ int smiless_evaluate(smiless_ctx *ctx, const smiless_plan_args *a, const uint64_
     if ((rc = upload_tables(ctx))) return rc;
     const i64 *d_arr = nullptr;
     if ((rc = stage_arrivals(ctx, a, &d_arr))) return rc;
+    if ((rc = stage_row_windows(ctx, a))) return rc;
     CK(ctx->dIdxEval.ensure((size_t)n), "cudaMalloc");
     CK(ctx->dCost.ensure((size_t)n), "cudaMalloc");
     CK(ctx->dLat.ensure((size_t)n), "cudaMalloc");
@@ -962,6 +990,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
 
     const i64 *d_arr = nullptr;
     if ((rc = stage_arrivals(ctx, a, &d_arr))) return rc;
+    if ((rc = stage_row_windows(ctx, a))) return rc;
 
     const RangePlan rp = range_plan(ctx, a);
     const i64 n_steps = a->n_arrivals - 1;
@@ -995,6 +1024,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         memset(&pp, 0, sizeof pp);
         pp.tabI = ctx->dI.p;
         pp.tabNI = ctx->dNI.p;
+        pp.tabW = ctx->dW.p;
         pp.zero = 0;
         pp.tabT = ctx->dT.p;
         pp.tabU = ctx->dU.p;
@@ -1035,6 +1065,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             BoundParamsHost bp;
             memset(&bp, 0, sizeof bp);
             bp.tabNI = ctx->dNI.p;
+            bp.tabW = ctx->dW.p;
             bp.tabT = ctx->dT.p;
             bp.off = ctx->dOff.p;
             bp.counter = ctx->dCounter.p;
@@ -1245,6 +1276,18 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
     if (!a) return fail(ctx, SMILESS_EINVAL, "args is NULL");
     const i64 sla = a->sla_us;
     return plan_impl(ctx, a, &sla, 1, res, config_out, window_out);
+}
+
+int smiless_derive_windows(const smiless_ctx *ctx, int64_t it_us, int32_t *row_windows_out) {
+    if (!ctx || !row_windows_out) return SMILESS_EINVAL;
+    if (!ctx->dag_loaded || !ctx->prof_loaded) return SMILESS_ESTATE;
+    if (it_us < 0) return SMILESS_EINVAL;
+    for (int r = 0; r < ctx->sumM; ++r) {
+        const i64 t = ctx->T[r], i = ctx->I[r];
+        const i64 w = (t + i < it_us) ? it_us - t - i : 0;   // Case I gap, else Case II keep-alive
+        row_windows_out[r] = (int32_t)std::min<i64>(w, (1 << 29) - 1);
+    }
+    return SMILESS_OK;
 }
 
 int smiless_plan_sla_sweep(smiless_ctx *ctx, const smiless_plan_args *a, const int64_t *slas, int32_t n_sla,

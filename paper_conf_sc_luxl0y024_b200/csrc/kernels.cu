@@ -104,7 +104,7 @@ __global__ void eval_exact_kernel(ExactParams p) {
         const int row = p.row0[k] + cfg[k];
         I[k] = p.tabI[row];
         T[k] = p.tabT[row];
-        w[k] = p.win[win[k]];
+        w[k] = p.rowwin ? p.rowwin[row] : p.win[win[k]];
         billed[k] = 0;
         D[k] = 0;
     }

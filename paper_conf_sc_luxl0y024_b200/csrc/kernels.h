@@ -42,6 +42,7 @@ struct ExactParams {
     int row0[SMILESS_DEV_MAX_FUNCS];
     int win[SMILESS_DEV_MAX_WINDOWS];
     int fixed[SMILESS_DEV_MAX_FUNCS];
+    const int *rowwin;           // per-row windows (NULL: the grid)
 };
 
 extern "C" {

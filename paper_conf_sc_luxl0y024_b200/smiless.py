@@ -25,8 +25,8 @@ _NAMES = {0: "OK", 1: "INFEASIBLE", -1: "EINVAL", -2: "ENOTTOPO", -3: "ERANGE", 
 # every symbol include/smiless.h declares (checked by tests/test_abi.py)
 EXPORTS = ("smiless_create", "smiless_set_stream", "smiless_destroy", "smiless_last_error",
            "smiless_load_dag", "smiless_load_profiles", "smiless_space_size", "smiless_plan",
-           "smiless_plan_sla_sweep", "smiless_evaluate", "smiless_decode", "smiless_kernel_source",
-           "smiless_jit_compile")
+           "smiless_plan_sla_sweep", "smiless_derive_windows", "smiless_evaluate", "smiless_decode",
+           "smiless_kernel_source", "smiless_jit_compile")
 
 
 class SmilessError(RuntimeError):
@@ -50,6 +50,7 @@ class PlanArgs(ctypes.Structure):
         ("shard", ctypes.c_int32),
         ("n_shards", ctypes.c_int32),
         ("cost_out", ctypes.c_void_p),
+        ("row_windows_us", ctypes.c_void_p),
     ]
 
 
@@ -113,6 +114,7 @@ def load_library(build_if_missing: bool = True):
     lib.smiless_plan.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.POINTER(PlanResultC), vp, vp]
     lib.smiless_plan_sla_sweep.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i32, ctypes.POINTER(PlanResultC),
                                            vp, vp]
+    lib.smiless_derive_windows.argtypes = [vp, i64, vp]
     lib.smiless_evaluate.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i64, vp, vp, vp]
     lib.smiless_decode.argtypes = [vp, i32, u64, ctypes.POINTER(PlanArgs), vp, vp]
     lib.smiless_kernel_source.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.c_char_p, ctypes.c_size_t,
@@ -176,13 +178,14 @@ class Planner:
 
     def load_profiles(self, n_configs, exec_us, init_us, price_per_us):
         m, e, t = _i32(n_configs), _i32(exec_us), _i32(init_us)
+        self._n_rows = int(m.sum())
         u = np.ascontiguousarray(np.asarray(price_per_us, dtype=np.float64))
         self._check(self._lib.smiless_load_profiles(self._ctx, m.ctypes.data, e.ctypes.data, t.ctypes.data,
                                                     u.ctypes.data))
 
     # ---- args ----------------------------------------------------------------------------
     def _args(self, arrivals, sla_us, windows_us, n_fixed=0, fixed_digits=(), begin=0, end=0, flags=0,
-              shard=0, n_shards=0, cost_out=None):
+              shard=0, n_shards=0, cost_out=None, row_windows=None):
         keep = []
         if _is_device_tensor(arrivals):
             import torch
@@ -203,12 +206,24 @@ class Planner:
                      fixed_digits=fixed.ctypes.data if n_fixed else None, begin=int(begin), end=int(end),
                      flags=int(flags), shard=int(shard), n_shards=int(n_shards),
                      cost_out=cost_out.ctypes.data if cost_out is not None else None)
+        if row_windows is not None:
+            rw = _i32(row_windows)
+            keep.append(rw)
+            a.row_windows_us = rw.ctypes.data
         if cost_out is not None:
             assert cost_out.dtype == np.float64 and cost_out.flags.c_contiguous
             keep.append(cost_out)
         return a, keep
 
     # ---- API -----------------------------------------------------------------------------
+    def derive_windows(self, it_us: int) -> np.ndarray:
+        """The paper's adaptive pre-warm window per (function, config) row for a predicted
+        inter-arrival time (smiless_derive_windows)."""
+        n = int(self._n_rows)
+        out = np.zeros(n, np.int32)
+        self._check(self._lib.smiless_derive_windows(self._ctx, int(it_us), out.ctypes.data))
+        return out
+
     def space_size(self, n_windows: int, n_fixed: int = 0) -> int:
         out = ctypes.c_uint64()
         self._check(self._lib.smiless_space_size(self._ctx, int(n_windows), int(n_fixed), ctypes.byref(out)))

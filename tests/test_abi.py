@@ -211,3 +211,15 @@ def test_library_kernels_have_no_vimnmx3():
     out = subprocess.run(["cuobjdump", "-sass", S.LIB_PATH], capture_output=True, text=True, check=True).stdout
     assert "prep_offsets_kernel" in out and "eval_exact_kernel" in out
     assert "VIMNMX3" not in out
+
+
+def test_derive_windows_is_the_papers_rule():
+    p = W.make_config("C2", n_arrivals=10)
+    pl = S.planner_for(p)
+    for it in (0, 1_000_000, 4_000_000, 20_000_000):
+        rw = pl.derive_windows(it)
+        exp = [it - t - i if t + i < it else 0 for t, i in zip(p.init_us.tolist(), p.exec_us.tolist())]
+        assert rw.tolist() == exp
+    with pytest.raises(S.SmilessError) as e:
+        pl.plan(p.arrivals_us, p.sla_us, [0, 5], row_windows=rw)       # requires n_windows == 1
+    assert e.value.code == S.EINVAL

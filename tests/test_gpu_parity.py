@@ -450,3 +450,50 @@ def test_sla_sweep_random_dags():
         for sla, g in zip(slas, rs):
             o = OracleProblem(p.replace(sla_us=sla))
             assert_same_plan(g, o.plan(), o)
+
+
+# ---------------------------------------------------------------------------------------
+# NEXT-1: config-only search under the paper's derived windows (per-row windows)
+# ---------------------------------------------------------------------------------------
+
+def test_derived_window_plans_match_oracle():
+    rng = np.random.default_rng(61)
+    n_checked = 0
+    for t in range(30):
+        n = int(rng.integers(1, 7))
+        p = W.random_problem(rng, n, 6, 1, int(rng.integers(1, 150)))
+        p = p.replace(windows_us=np.array([0], np.int32))
+        if p.space_size() > 30000:
+            continue
+        pl = S.planner_for(p)
+        it = int(np.diff(p.arrivals_us).mean()) if len(p.arrivals_us) > 1 else 0
+        rw = pl.derive_windows(it)
+        o = OracleProblem(p, row_windows=rw)
+        space = p.space_size()
+        for flags in (0, S.FLAG_NO_PRUNE, S.FLAG_FORCE_INT64):
+            out = np.empty(space)
+            g = pl.plan(p.arrivals_us, p.sla_us, [0], row_windows=rw, flags=flags, cost_out=out)
+            assert_same_plan(g, o.plan(), o)
+            oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
+            assert_dump_matches(out, oc, of)
+        idx = rng.integers(0, space, size=32, dtype=np.uint64)
+        assert_same_eval(*pl.evaluate(idx, p.arrivals_us, p.sla_us, [0], row_windows=rw), *o.evaluate(idx))
+        n_checked += 1
+    assert n_checked > 15
+
+
+def test_derived_window_c2_full_plan_with_bnb():
+    """C2 (J = 10^4) under the paper's derived windows: 16^6 configurations, B&B pre-pass."""
+    p = W.make_config("C2")
+    q = p.replace(windows_us=np.array([0], np.int32))
+    pl = S.planner_for(q)
+    rw = pl.derive_windows(int(np.diff(p.arrivals_us).mean()))
+    g = pl.plan(q.arrivals_us, q.sla_us, [0], row_windows=rw)
+    o = OracleProblem(q, row_windows=rw)
+    assert g.n_decided == 16 ** 6
+    if g.feasible:
+        c, l, f = o.evaluate([g.index])
+        assert f[0] and c[0] == g.cost and l[0] == g.max_latency_us
+        lo = g.index - g.index % 4096
+        ref = o.plan(begin=lo, end=lo + 4096)
+        assert ref[0] == g.index and ref[1] == g.cost

@@ -403,3 +403,40 @@ def test_oracle_rejects_bad_args():
     o.s.n_arrivals = 0
     with pytest.raises(ValueError):
         o.evaluate([0])
+
+
+# ---------------------------------------------------------------------------
+# NEXT-1: the paper's derived (adaptive) pre-warm windows as per-row windows
+# ---------------------------------------------------------------------------
+
+def paper_window(T, I, IT):
+    """Case I (T + I < IT) -> IT - T - I; Case II -> 0 (keep alive)."""
+    return IT - T - I if T + I < IT else 0
+
+
+def test_derived_windows_reproduce_eq5_on_periodic_arrivals():
+    """With the paper's derived windows and periodic arrivals the oracle gives Eq. (5):
+    L = sum of I, C_k = (T_k + I_k) per invocation in Case I and IT per invocation after
+    the first in Case II -- for every config of a random chain."""
+    rng = np.random.default_rng(31)
+    for _ in range(100):
+        n = int(rng.integers(1, 5))
+        M = int(rng.integers(1, 4))
+        IT = int(rng.integers(20_000, 100_000))
+        J = int(rng.integers(2, 25))
+        I = rng.integers(0, IT // (n + 1), size=n * M)          # sum of I over a path < IT: never busy
+        T = rng.integers(0, 2 * IT, size=n * M)
+        p = mk([[]] + [[k - 1] for k in range(1, n)], I, T, np.arange(J, dtype=np.int64) * IT, [0],
+               n_configs=[M] * n, prices=np.ones(n * M))
+        rw = [paper_window(int(T[r]), int(I[r]), IT) for r in range(n * M)]
+        o = OracleProblem(p, row_windows=rw)
+        for _ in range(5):
+            c = [int(rng.integers(0, M)) for _ in range(n)]
+            billed, lat = o.simulate(c, [0] * n)
+            rows = [k * M + c[k] for k in range(n)]
+            assert (lat == sum(int(I[r]) for r in rows)).all()
+            for k, r in enumerate(rows):
+                if T[r] + I[r] < IT:
+                    assert billed[k] == J * int(T[r] + I[r])
+                else:
+                    assert billed[k] == int(T[r] + I[r]) + (J - 1) * IT
