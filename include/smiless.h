@@ -172,6 +172,23 @@ SMILESS_API int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smile
  * Returns OK, ESTATE or EINVAL. */
 SMILESS_API int smiless_derive_windows(const smiless_ctx *ctx, int64_t it_us, int32_t *row_windows_out);
 
+/* NEXT-2: SMIless's own Top-1 path search (Fig. 6, Eq. (6)) -- the heuristic the
+ * paper deploys -- over configurations with per-row pre-warm windows (a->row_windows_us,
+ * n_windows == 1, e.g. from smiless_derive_windows; a->n_fixed must be 0).  Each function's
+ * configs are ranked by the paper's per-invocation cost under adaptive pre-warming,
+ * U * (T + I) in Case I and U * IT in Case II (O(N M log M)).  Root =
+ * every function on its cheapest config; on an SLA miss the search walks the layers
+ * F_1..F_N: in layer k functions < k keep their chosen config, functions > k run on their
+ * fastest config, and F_k takes the next cheapest config until the node meets the SLA
+ * (layer 1 starts at the second cheapest).  Every node is evaluated on the GPU
+ * with model M (the same exact evaluator as smiless_evaluate), one batch per layer.
+ * res / config_out / window_out receive the leaf (index UINT64_MAX, -1 outputs and return
+ * INFEASIBLE if no node of the last layer meets the SLA); *n_nodes the evaluated nodes.
+ * Returns OK, INFEASIBLE or an error. */
+SMILESS_API int smiless_top1_search(smiless_ctx *ctx, const smiless_plan_args *a, int64_t it_us,
+                                    smiless_plan_result *res, int32_t *config_out, int32_t *window_out,
+                                    int64_t *n_nodes);
+
 /* SLA sweep (C4: "impact of SLA settings"): ONE evaluation of the space
  * with one argmin key per SLA in slas[0..n_sla) (1 <= n_sla <= SMILESS_MAX_SLAS); pruning uses
  * their maximum; a->sla_us is ignored and a->cost_out must be NULL.  res[n_sla] and, when not

@@ -1290,6 +1290,103 @@ int smiless_derive_windows(const smiless_ctx *ctx, int64_t it_us, int32_t *row_w
     return SMILESS_OK;
 }
 
+int smiless_top1_search(smiless_ctx *ctx, const smiless_plan_args *a, int64_t it_us, smiless_plan_result *res,
+                        int32_t *config_out, int32_t *window_out, int64_t *n_nodes) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->err.clear();
+    if (!a || !res) return fail(ctx, SMILESS_EINVAL, "args / res is NULL");
+    if (!a->row_windows_us) return fail(ctx, SMILESS_EINVAL, "top1 search needs row_windows_us (n_windows == 1)");
+    if (a->n_fixed != 0) return fail(ctx, SMILESS_EINVAL, "top1 search does not take pinned digits");
+    int rc = validate_args(ctx, a, true);
+    if (rc) return rc;
+    const int N = ctx->N;
+    // per-function ranking by the paper's per-invocation cost (Eq. 5 / Case II), ties: lower config
+    std::vector<std::vector<int>> rank(N);
+    std::vector<int> fastest(N);
+    for (int k = 0; k < N; ++k) {
+        std::vector<std::pair<double, int>> c;
+        int fk = 0;
+        for (int m = 0; m < ctx->M[k]; ++m) {
+            const int row = ctx->row0[k] + m;
+            const i64 t = ctx->T[row], i = ctx->I[row];
+            const double per_inv = (t + i < it_us) ? (double)(t + i) : (double)it_us;
+            c.push_back({ctx->U[row] * per_inv, m});
+            if (ctx->I[row] < ctx->I[ctx->row0[k] + fk]) fk = m;
+        }
+        std::stable_sort(c.begin(), c.end(), [](const std::pair<double, int> &x, const std::pair<double, int> &y) {
+            return x.first < y.first;
+        });
+        for (auto &pr : c) rank[k].push_back(pr.second);
+        fastest[k] = fk;
+    }
+    auto index_of = [&](const std::vector<int> &cfg) {     // W == 1: digit = config
+        u64 idx = 0;
+        for (int k = 0; k < N; ++k) idx = idx * (u64)ctx->M[k] + (u64)cfg[k];
+        return idx;
+    };
+    i64 nodes = 0;
+    std::vector<int> chosen(N, -1);
+    std::vector<u64> batch;
+    std::vector<double> cost;
+    std::vector<int64_t> lat;
+    std::vector<uint8_t> feas;
+    auto eval = [&](const std::vector<std::vector<int>> &cfgs) -> int {
+        batch.clear();
+        for (auto &c : cfgs) batch.push_back(index_of(c));
+        cost.assign(batch.size(), 0.0);
+        lat.assign(batch.size(), 0);
+        feas.assign(batch.size(), 0);
+        nodes += (i64)batch.size();
+        return smiless_evaluate(ctx, a, (const uint64_t *)batch.data(), (int64_t)batch.size(), cost.data(), lat.data(),
+                                feas.data());
+    };
+    // root T^0: every function on its cheapest configuration (Eq. 6)
+    std::vector<int> root(N);
+    for (int k = 0; k < N; ++k) root[k] = rank[k][0];
+    if ((rc = eval({root}))) return rc;
+    std::vector<int> leaf = root;
+    bool ok = feas[0] != 0;
+    if (!ok) {
+        for (int k = 0; k < N; ++k) {
+            std::vector<std::vector<int>> layer;
+            const int r0 = (k == 0) ? 1 : 0;                // T^1_1: F_1 on its second cheapest
+            for (int r = r0; r < ctx->M[k]; ++r) {
+                std::vector<int> c(N);
+                for (int q = 0; q < N; ++q) c[q] = q < k ? chosen[q] : (q == k ? rank[k][r] : fastest[q]);
+                layer.push_back(c);
+            }
+            int pick = -1;
+            if (!layer.empty()) {
+                if ((rc = eval(layer))) return rc;
+                for (size_t i = 0; i < layer.size(); ++i)
+                    if (feas[i]) { pick = (int)i; break; }
+            }
+            chosen[k] = pick >= 0 ? layer[pick][k] : fastest[k];
+        }
+        leaf = chosen;
+        if ((rc = eval({leaf}))) return rc;
+        ok = feas[0] != 0;
+    }
+    memset(res, 0, sizeof *res);
+    res->n_decided = (u64)nodes;
+    res->n_full_evals = (u64)nodes;
+    if (n_nodes) *n_nodes = nodes;
+    for (int k = 0; k < N; ++k) {
+        if (config_out) config_out[k] = ok ? leaf[k] : -1;
+        if (window_out) window_out[k] = ok ? 0 : -1;
+    }
+    if (!ok) {
+        res->index = ~0ull;
+        res->cost = HUGE_VAL;
+        res->max_latency_us = -1;
+        return SMILESS_INFEASIBLE;
+    }
+    res->index = index_of(leaf);
+    res->cost = cost[0];
+    res->max_latency_us = lat[0];
+    return SMILESS_OK;
+}
+
 int smiless_plan_sla_sweep(smiless_ctx *ctx, const smiless_plan_args *a, const int64_t *slas, int32_t n_sla,
                            smiless_plan_result *res, int32_t *config_out, int32_t *window_out) {
     if (!ctx) return SMILESS_EINVAL;

@@ -25,7 +25,8 @@ _NAMES = {0: "OK", 1: "INFEASIBLE", -1: "EINVAL", -2: "ENOTTOPO", -3: "ERANGE", 
 # every symbol include/smiless.h declares (checked by tests/test_abi.py)
 EXPORTS = ("smiless_create", "smiless_set_stream", "smiless_destroy", "smiless_last_error",
            "smiless_load_dag", "smiless_load_profiles", "smiless_space_size", "smiless_plan",
-           "smiless_plan_sla_sweep", "smiless_derive_windows", "smiless_evaluate", "smiless_decode",
+           "smiless_plan_sla_sweep", "smiless_derive_windows", "smiless_top1_search", "smiless_evaluate",
+           "smiless_decode",
            "smiless_kernel_source", "smiless_jit_compile")
 
 
@@ -115,6 +116,8 @@ def load_library(build_if_missing: bool = True):
     lib.smiless_plan_sla_sweep.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i32, ctypes.POINTER(PlanResultC),
                                            vp, vp]
     lib.smiless_derive_windows.argtypes = [vp, i64, vp]
+    lib.smiless_top1_search.argtypes = [vp, ctypes.POINTER(PlanArgs), i64, ctypes.POINTER(PlanResultC), vp, vp,
+                                        ctypes.POINTER(ctypes.c_int64)]
     lib.smiless_evaluate.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i64, vp, vp, vp]
     lib.smiless_decode.argtypes = [vp, i32, u64, ctypes.POINTER(PlanArgs), vp, vp]
     lib.smiless_kernel_source.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.c_char_p, ctypes.c_size_t,
@@ -264,6 +267,22 @@ class Planner:
                                   eval_kernel_ms=float(r.eval_kernel_ms), total_device_ms=float(r.total_device_ms),
                                   int64_path=bool(r.int64_path), launches=int(r.launches)))
         return out
+
+    def top1_search(self, arrivals, sla_us, it_us, row_windows, **kw):
+        """SMIless's Top-1 path search (smiless_top1_search); returns (PlanResult, nodes)."""
+        a, keep = self._args(arrivals, sla_us, [0], row_windows=row_windows, **kw)
+        r = PlanResultC()
+        cfg = np.zeros(max(self.n_funcs, 1), np.int32)
+        win = np.zeros(max(self.n_funcs, 1), np.int32)
+        nodes = ctypes.c_int64()
+        rc = self._check(self._lib.smiless_top1_search(self._ctx, ctypes.byref(a), int(it_us), ctypes.byref(r),
+                                                       cfg.ctypes.data, win.ctypes.data, ctypes.byref(nodes)),
+                         allow=(OK, INFEASIBLE))
+        del keep
+        return PlanResult(status=rc, index=None if rc == INFEASIBLE else int(r.index), cost=float(r.cost),
+                          max_latency_us=int(r.max_latency_us), config=cfg[:self.n_funcs],
+                          window=win[:self.n_funcs], n_decided=int(r.n_decided), n_full_evals=int(r.n_full_evals),
+                          eval_kernel_ms=0.0, total_device_ms=0.0, int64_path=False, launches=0), int(nodes.value)
 
     def evaluate(self, idx, arrivals, sla_us, windows_us, **kw) -> Tuple[np.ndarray, np.ndarray, np.ndarray]:
         a, keep = self._args(arrivals, sla_us, windows_us, **kw)

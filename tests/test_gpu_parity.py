@@ -497,3 +497,42 @@ def test_derived_window_c2_full_plan_with_bnb():
         lo = g.index - g.index % 4096
         ref = o.plan(begin=lo, end=lo + 4096)
         assert ref[0] == g.index and ref[1] == g.cost
+
+
+# ---------------------------------------------------------------------------------------
+# NEXT-2: SMIless's Top-1 path search, GPU-evaluated nodes vs the oracle's walk
+# ---------------------------------------------------------------------------------------
+
+def test_top1_search_matches_oracle_walk():
+    from oracle.top1 import top1_search
+    rng = np.random.default_rng(71)
+    for t in range(30):
+        n = int(rng.integers(1, 7))
+        p = W.random_problem(rng, n, 6, 1, int(rng.integers(2, 120)), sla_us=int(rng.integers(5_000, 40_000)))
+        p = p.replace(windows_us=np.array([0], np.int32))
+        it = int(np.diff(p.arrivals_us).mean()) if len(p.arrivals_us) > 1 else 0
+        pl = S.planner_for(p)
+        rw = pl.derive_windows(it)
+        g, nodes = pl.top1_search(p.arrivals_us, p.sla_us, it, rw)
+        cfg, cost, lat, ok, onodes = top1_search(p, it, rw, OracleProblem)
+        assert nodes == onodes
+        assert g.feasible == ok
+        if ok:
+            assert g.config.tolist() == cfg and g.cost == cost and g.max_latency_us == lat
+
+
+def test_top1_never_beats_exhaustive_opt():
+    """The heuristic's plan is a candidate of the derived-window space, so the exhaustive
+    OPT of that space (and of the full window grid) costs no more."""
+    rng = np.random.default_rng(72)
+    for t in range(20):
+        n = int(rng.integers(2, 6))
+        p = W.random_problem(rng, n, 5, 1, int(rng.integers(10, 100)), sla_us=int(rng.integers(8_000, 40_000)))
+        p = p.replace(windows_us=np.array([0], np.int32))
+        it = int(np.diff(p.arrivals_us).mean())
+        pl = S.planner_for(p)
+        rw = pl.derive_windows(it)
+        h, _ = pl.top1_search(p.arrivals_us, p.sla_us, it, rw)
+        opt = pl.plan(p.arrivals_us, p.sla_us, [0], row_windows=rw)
+        if h.feasible:
+            assert opt.feasible and opt.cost <= h.cost
