@@ -1,0 +1,56 @@
+"""NEXT-1 / NEXT-2 on the BASELINE configs: exhaustive OPT over configs x window grid vs
+exhaustive OPT under the paper's derived windows (NEXT-1) vs SMIless's Top-1 path search
+(NEXT-2, the paper's deployed heuristic), all exact under model M on one GPU.  This is the
+paper's Fig. 8 comparison "SMIless vs OPT (exhaustive search)" on synthetic inputs."""
+import json, sys, time
+sys.path.insert(0, '.')
+import numpy as np
+import torch
+import workloads as W
+from oracle import OracleProblem
+from paper_conf_sc_luxl0y024_b200 import smiless as S
+
+
+def run(name, p, check=True):
+    stream = torch.cuda.current_stream().cuda_stream
+    pl = S.planner_for(p, stream=stream)
+    arr = torch.as_tensor(p.arrivals_us).cuda()
+    it = int(np.diff(p.arrivals_us).mean())
+    out = {"config": name, "J": len(p.arrivals_us), "IT_us": it}
+    t0 = time.perf_counter()
+    full = pl.plan(arr, p.sla_us, p.windows_us)
+    out["opt_grid"] = {"cost": full.cost if full.feasible else None, "s": time.perf_counter() - t0,
+                       "config": full.config.tolist(), "window": full.window.tolist(),
+                       "candidates": pl.space_size(len(p.windows_us))}
+    q = p.replace(windows_us=np.array([0], np.int32))
+    plq = S.planner_for(q, stream=stream)
+    rw = plq.derive_windows(it)
+    t0 = time.perf_counter()
+    der = plq.plan(arr, q.sla_us, [0], row_windows=rw)
+    out["opt_derived_windows"] = {"cost": der.cost if der.feasible else None, "s": time.perf_counter() - t0,
+                                  "config": der.config.tolist(), "candidates": plq.space_size(1)}
+    t0 = time.perf_counter()
+    h, nodes = plq.top1_search(p.arrivals_us, q.sla_us, it, rw)
+    out["top1_search"] = {"cost": h.cost if h.feasible else None, "s": time.perf_counter() - t0, "nodes": nodes,
+                          "config": h.config.tolist()}
+    if full.feasible and h.feasible:
+        out["top1_over_opt"] = h.cost / full.cost
+    if full.feasible and der.feasible:
+        out["derived_over_opt"] = der.cost / full.cost
+    if check and full.feasible:
+        c, l, f = OracleProblem(p).evaluate([full.index])
+        out["opt_grid"]["oracle_check"] = bool(f[0] and c[0] == full.cost and l[0] == full.max_latency_us)
+    return out
+
+
+res = []
+for name in sys.argv[1:] or ["C1", "C2", "C3"]:
+    if name.startswith("C4"):
+        p = W.make_config("C4")
+        for i, w in enumerate(W.c4_replans(int(name[3:] or 6))):
+            for sla in (1_000_000, 2_000_000, 3_000_000):
+                res.append(run(f"C4 window {i} SLA {sla}", p.replace(arrivals_us=w, sla_us=sla)))
+    else:
+        res.append(run(name, W.make_config(name)))
+for r in res:
+    print(json.dumps(r))
