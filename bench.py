@@ -252,10 +252,19 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # SMILESS_BENCH_SAME_GPU=1 (testing the multi-rank flow on a one-GPU box): every rank
+    # uses cuda:0 and the exchange runs on gloo; the real runs use one GPU per rank + NCCL
+    same_gpu = os.environ.get("SMILESS_BENCH_SAME_GPU") == "1"
+    if same_gpu:
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    xdev = torch.device("cpu") if same_gpu else dev           # device of the collective tensors
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if same_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
 
     p, kw = workload(args.workload)
     stream = torch.cuda.current_stream(dev)
@@ -268,7 +277,7 @@ def main():
     def step(arrivals):
         r = pl.plan(arrivals, p.sla_us, p.windows_us, **plan_kw)
         if world > 1:
-            reduce_best(r.cost if r.feasible else None, r.index, r.max_latency_us, r.n_decided, dev)
+            reduce_best(r.cost if r.feasible else None, r.index, r.max_latency_us, r.n_decided, xdev)
         return r
 
     def barrier():
@@ -297,7 +306,7 @@ def main():
             kernel_ms += res.eval_kernel_ms
         torch.cuda.synchronize(dev)
         ms = sum(a.elapsed_time(b) for a, b in evs)
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        t = torch.tensor([ms], dtype=torch.float64, device=xdev)
         if world > 1:
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item()), res, launches, kernel_ms
@@ -312,7 +321,7 @@ def main():
 
     cands = int(res.n_decided)
     if world > 1:
-        t = torch.tensor([cands], dtype=torch.int64, device=dev)
+        t = torch.tensor([cands], dtype=torch.int64, device=xdev)
         dist.all_reduce(t)
         cands = int(t.item())
     steps_e2e = max(1, min(args.steps, 3))
@@ -329,7 +338,7 @@ def main():
         a.record(stream)
         rp = pl.plan(arr_dev, p.sla_us, p.windows_us, **kwp)
         if world > 1:
-            reduce_best(rp.cost if rp.feasible else None, rp.index, rp.max_latency_us, rp.n_decided, dev)
+            reduce_best(rp.cost if rp.feasible else None, rp.index, rp.max_latency_us, rp.n_decided, xdev)
         b.record(stream)
         torch.cuda.synchronize(dev)
         pruned = {"time_to_optimal_ms": a.elapsed_time(b), "index": rp.index, "cost": rp.cost,
@@ -348,13 +357,13 @@ def main():
         rf = pl.plan(arr_dev, p.sla_us, p.windows_us, shard=rank, n_shards=world)
         if world > 1:
             g_cost, g_idx, g_lat, g_dec = reduce_best(rf.cost if rf.feasible else None, rf.index,
-                                                      rf.max_latency_us, rf.n_decided, dev)
+                                                      rf.max_latency_us, rf.n_decided, xdev)
         else:
             g_cost, g_idx, g_lat, g_dec = (rf.cost if rf.feasible else None), rf.index, rf.max_latency_us, rf.n_decided
         b.record(stream)
         torch.cuda.synchronize(dev)
         wall = time.perf_counter() - t0
-        tt = torch.tensor([a.elapsed_time(b)], dtype=torch.float64, device=dev)
+        tt = torch.tensor([a.elapsed_time(b)], dtype=torch.float64, device=xdev)
         if world > 1:
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         full = {"candidates": full_space, "time_to_optimal_s": float(tt.item()) / 1e3, "wall_s": wall,

@@ -502,6 +502,8 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_D " << (D > 0 ? D : N - 1) << "\n#define SMILESS_MAXF " << SMILESS_MAX_FUNCS << "\n";
     s << "#define SM_NSLA " << ctx->nsla << "\n";
     s << "#define SM_ROWWIN " << (a->row_windows_us ? 1 : 0) << "\n";
+    const char *mask_env = getenv("SMILESS_MASK");   // tuning knob, see evaluator.cuh SM_MASK
+    s << "#define SM_MASK " << (mask_env ? atoi(mask_env) : 0) << "\n";
     // compile-time window grid (immediates) and a constant-bank copy for runtime indices
     s << "#define SM_WIN(v) (";
     for (int v = 0; v < W; ++v) s << "(v)==" << v << "?" << a->windows_us[v] << ":";
