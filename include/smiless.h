@@ -189,6 +189,27 @@ SMILESS_API int smiless_top1_search(smiless_ctx *ctx, const smiless_plan_args *a
                                     smiless_plan_result *res, int32_t *config_out, int32_t *window_out,
                                     int64_t *n_nodes);
 
+typedef struct {
+    int32_t config;      /* chosen configuration (-1: none meets the target, or no invocations) */
+    int64_t batch;       /* B: invocations batched per instance                                  */
+    int64_t instances;   /* ceil(G / B)                                                          */
+    double cost;         /* (instances * IT) * U(config): $ per time window; +inf if none         */
+} smiless_autoscale_result;
+
+/* NEXT-4: the paper's auto-scaler (Eq. (7)/(8)) for all functions at once.  For
+ * function k with G_k predicted invocations in the next window of length IT and required
+ * inference time target_k (I_s), choose
+ *     min over (config c, B)  ceil(G_k / B) * IT * U(c)
+ *     s.t.  slope_us[c] * B + intercept_us[c] <= target_k
+ * where slope = lambda (alpha / x + beta) and intercept = gamma are the Eq. (1)/(2) batch model
+ * of row c (x = cores or GPU share).  Per config the largest feasible B in [1, G_k] is found by
+ * bisection (the constraint is monotone in B, the cost non-increasing); ties on cost go to
+ * the lower config.  Doubles: slope * B then + intercept, IEEE, no FMA.  Host-only (the paper
+ * reports < 0.1 ms).  Returns OK, ESTATE or EINVAL. */
+SMILESS_API int smiless_autoscale(const smiless_ctx *ctx, const double *slope_us, const double *intercept_us,
+                                  const int64_t *invocations, int64_t it_us, const int64_t *target_us,
+                                  smiless_autoscale_result *out);
+
 /* SLA sweep (C4: "impact of SLA settings"): ONE evaluation of the space
  * with one argmin key per SLA in slas[0..n_sla) (1 <= n_sla <= SMILESS_MAX_SLAS); pruning uses
  * their maximum; a->sla_us is ignored and a->cost_out must be NULL.  res[n_sla] and, when not

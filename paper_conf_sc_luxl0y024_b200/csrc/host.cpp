@@ -1389,6 +1389,43 @@ int smiless_top1_search(smiless_ctx *ctx, const smiless_plan_args *a, int64_t it
     return SMILESS_OK;
 }
 
+int smiless_autoscale(const smiless_ctx *ctx, const double *slope_us, const double *intercept_us,
+                      const int64_t *invocations, int64_t it_us, const int64_t *target_us,
+                      smiless_autoscale_result *out) {
+    if (!ctx || !slope_us || !intercept_us || !invocations || !target_us || !out) return SMILESS_EINVAL;
+    if (!ctx->dag_loaded || !ctx->prof_loaded) return SMILESS_ESTATE;
+    if (it_us < 0) return SMILESS_EINVAL;
+    for (int k = 0; k < ctx->N; ++k) {
+        smiless_autoscale_result best{-1, 0, 0, HUGE_VAL};
+        const i64 G = invocations[k];
+        if (G <= 0) {
+            out[k] = smiless_autoscale_result{-1, 0, 0, 0.0};
+            continue;
+        }
+        for (int c = 0; c < ctx->M[k]; ++c) {
+            const int row = ctx->row0[k] + c;
+            const double a = slope_us[row], b = intercept_us[row], lim = (double)target_us[k];
+            auto ok = [&](i64 B) {
+                volatile double prod = a * (double)B;   // two rounded operations, never an FMA
+                return prod + b <= lim;
+            };
+            if (!ok(1)) continue;
+            i64 lo = 1, hi = G;                           // bisection: largest feasible B
+            while (lo < hi) {
+                const i64 mid = lo + (hi - lo + 1) / 2;
+                if (ok(mid)) lo = mid;
+                else hi = mid - 1;
+            }
+            const i64 inst = (G + lo - 1) / lo;
+            volatile double inst_it = (double)inst * (double)it_us;
+            const double cost = inst_it * ctx->U[row];
+            if (cost < best.cost) best = smiless_autoscale_result{c, lo, inst, cost};
+        }
+        out[k] = best;
+    }
+    return SMILESS_OK;
+}
+
 int smiless_plan_sla_sweep(smiless_ctx *ctx, const smiless_plan_args *a, const int64_t *slas, int32_t n_sla,
                            smiless_plan_result *res, int32_t *config_out, int32_t *window_out) {
     if (!ctx) return SMILESS_EINVAL;

@@ -25,7 +25,8 @@ _NAMES = {0: "OK", 1: "INFEASIBLE", -1: "EINVAL", -2: "ENOTTOPO", -3: "ERANGE", 
 # every symbol include/smiless.h declares (checked by tests/test_abi.py)
 EXPORTS = ("smiless_create", "smiless_set_stream", "smiless_destroy", "smiless_last_error",
            "smiless_load_dag", "smiless_load_profiles", "smiless_space_size", "smiless_plan",
-           "smiless_plan_sla_sweep", "smiless_derive_windows", "smiless_top1_search", "smiless_evaluate",
+           "smiless_plan_sla_sweep", "smiless_derive_windows", "smiless_top1_search", "smiless_autoscale",
+           "smiless_evaluate",
            "smiless_decode",
            "smiless_kernel_source", "smiless_jit_compile")
 
@@ -116,6 +117,7 @@ def load_library(build_if_missing: bool = True):
     lib.smiless_plan_sla_sweep.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i32, ctypes.POINTER(PlanResultC),
                                            vp, vp]
     lib.smiless_derive_windows.argtypes = [vp, i64, vp]
+    lib.smiless_autoscale.argtypes = [vp, vp, vp, vp, i64, vp, vp]
     lib.smiless_top1_search.argtypes = [vp, ctypes.POINTER(PlanArgs), i64, ctypes.POINTER(PlanResultC), vp, vp,
                                         ctypes.POINTER(ctypes.c_int64)]
     lib.smiless_evaluate.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i64, vp, vp, vp]
@@ -225,6 +227,19 @@ class Planner:
         n = int(self._n_rows)
         out = np.zeros(n, np.int32)
         self._check(self._lib.smiless_derive_windows(self._ctx, int(it_us), out.ctypes.data))
+        return out
+
+    def autoscale(self, slope_us, intercept_us, invocations, it_us, target_us):
+        """The paper's auto-scaler (smiless_autoscale, Eq. (7)/(8)): per function
+        (config, batch B, instances, cost)."""
+        sl = np.ascontiguousarray(np.asarray(slope_us, dtype=np.float64))
+        ic = np.ascontiguousarray(np.asarray(intercept_us, dtype=np.float64))
+        G = np.ascontiguousarray(np.asarray(invocations, dtype=np.int64))
+        tg = np.ascontiguousarray(np.asarray(target_us, dtype=np.int64))
+        out = np.zeros(self.n_funcs, dtype=np.dtype([("config", np.int32), ("batch", np.int64),
+                                                      ("instances", np.int64), ("cost", np.float64)], align=True))
+        self._check(self._lib.smiless_autoscale(self._ctx, sl.ctypes.data, ic.ctypes.data, G.ctypes.data,
+                                                int(it_us), tg.ctypes.data, out.ctypes.data))
         return out
 
     def space_size(self, n_windows: int, n_fixed: int = 0) -> int:

@@ -223,3 +223,36 @@ def test_derive_windows_is_the_papers_rule():
     with pytest.raises(S.SmilessError) as e:
         pl.plan(p.arrivals_us, p.sla_us, [0, 5], row_windows=rw)       # requires n_windows == 1
     assert e.value.code == S.EINVAL
+
+
+def test_autoscale_matches_brute_force_oracle():
+    """NEXT-4 (Eq. (7)/(8)): bisection over B per config == brute force over
+    every (config, B) (host-only, no GPU)."""
+    from oracle.autoscale import autoscale
+    rng = np.random.default_rng(81)
+    for name in ("C1", "C2", "C3"):
+        p = W.make_config(name, n_arrivals=10)
+        pl = S.planner_for(p)
+        for _ in range(20):
+            G = rng.integers(0, 200, size=p.n_funcs)
+            it = int(rng.integers(100_000, 5_000_000))
+            tgt = rng.integers(50_000, 5_000_000, size=p.n_funcs)
+            got = pl.autoscale(p.batch_slope_us, p.batch_intercept_us, G, it, tgt)
+            ref = autoscale(p, p.batch_slope_us, p.batch_intercept_us, G, it, tgt)
+            for k in range(p.n_funcs):
+                c, B, inst, cost = ref[k]
+                assert (int(got[k]["config"]), int(got[k]["batch"]), int(got[k]["instances"])) == (c, B, inst)
+                assert float(got[k]["cost"]) == cost or (c == -1 and G[k] > 0 and np.isinf(got[k]["cost"]))
+
+
+def test_autoscale_paper_properties():
+    """More invocations never cost less; a looser latency target never costs more."""
+    p = W.make_config("C2", n_arrivals=10)
+    pl = S.planner_for(p)
+    it = 1_000_000
+    base = pl.autoscale(p.batch_slope_us, p.batch_intercept_us, [50] * 6, it, [2_000_000] * 6)
+    more = pl.autoscale(p.batch_slope_us, p.batch_intercept_us, [100] * 6, it, [2_000_000] * 6)
+    loose = pl.autoscale(p.batch_slope_us, p.batch_intercept_us, [50] * 6, it, [4_000_000] * 6)
+    for k in range(6):
+        assert more[k]["cost"] >= base[k]["cost"]
+        assert loose[k]["cost"] <= base[k]["cost"]

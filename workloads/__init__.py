@@ -89,6 +89,8 @@ def gen_profiles(rng: np.random.Generator, n_funcs: int, n_configs: int):
     rounded to integer microseconds (reading G14).
     """
     grid = CONFIG_GRIDS[n_configs]
+    slope = np.zeros((n_funcs, n_configs), dtype=np.float64)      # lambda * (alpha / x + beta)
+    icept = np.zeros((n_funcs, n_configs), dtype=np.float64)      # gamma
     ex = np.zeros((n_funcs, n_configs), dtype=np.int64)
     ini = np.zeros((n_funcs, n_configs), dtype=np.int64)
     price = np.zeros((n_funcs, n_configs), dtype=np.float64)
@@ -106,10 +108,12 @@ def gen_profiles(rng: np.random.Generator, n_funcs: int, n_configs: int):
         for c, (kind, amount) in enumerate(grid):
             jitter = rng.uniform(0.97, 1.03)
             if kind == "cpu":
+                slope[k, c], icept[k, c] = l_c * (a_c / amount + b_c), g_c
                 t_inf = l_c * 1 * (a_c / amount + b_c) + g_c          # Eq. (1), B = 1
                 mu = mu_c * jitter
                 p = amount * CPU_PRICE_PER_CORE_H
             else:
+                slope[k, c], icept[k, c] = l_g * (a_g / amount + b_g), g_g
                 t_inf = l_g * 1 * (a_g / amount + b_g) + g_g          # Eq. (2), B = 1
                 mu = mu_g * jitter
                 p = amount * GPU_PRICE_FULL_H
@@ -117,6 +121,7 @@ def gen_profiles(rng: np.random.Generator, n_funcs: int, n_configs: int):
             ex[k, c] = int(round(t_inf))
             ini[k, c] = int(round(mu + 3.0 * sigma))                   # mu + n sigma, n = 3
             price[k, c] = p / US_PER_H
+    gen_profiles.last_batch_model = (slope.reshape(-1), icept.reshape(-1))
     return ex.astype(np.int32), ini.astype(np.int32), price
 
 
@@ -200,6 +205,9 @@ class Problem:
     arrivals_us: np.ndarray   # int64 [J]
     sla_us: int
     windows_us: np.ndarray    # int32 [W]
+    # Eq. (1)/(2) batch model per row: inference time of a batch of B = slope * B + intercept
+    batch_slope_us: Optional[np.ndarray] = None      # f64 [sum M]
+    batch_intercept_us: Optional[np.ndarray] = None  # f64 [sum M]
 
     @property
     def n_funcs(self) -> int:
@@ -224,12 +232,13 @@ def build_problem(name: str, dag: str, m: int, w: int, arrivals: np.ndarray,
     ptr, idx = csr_from_preds(preds)
     n = len(preds)
     ex, ini, pr = gen_profiles(rng, n, m)
+    slope, icept = gen_profiles.last_batch_model
     return Problem(
         name=name, pred_ptr=ptr, pred_idx=idx,
         n_configs=np.full(n, m, dtype=np.int32),
         exec_us=ex.reshape(-1), init_us=ini.reshape(-1), price_per_us=pr.reshape(-1),
         arrivals_us=np.ascontiguousarray(arrivals, dtype=np.int64), sla_us=int(sla_us),
-        windows_us=window_grid(w))
+        windows_us=window_grid(w), batch_slope_us=slope, batch_intercept_us=icept)
 
 
 CONFIG_NUMBER = {"C1": 1, "C2": 2, "C3": 3, "C4": 4, "C5": 5}
