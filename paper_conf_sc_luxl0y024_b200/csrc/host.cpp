@@ -149,10 +149,10 @@ struct PlanParamsHost {
     double *dump;
     const int *tabNI;
     int zero;
-    const unsigned *list_in;
+    const u64 *list_in;
     const unsigned *list_n;
     u64 list_upp;
-    unsigned *list_out;
+    u64 *list_out;
     unsigned *list_cnt;
     u64 list_base;
     i64 horizon;
@@ -168,7 +168,7 @@ struct BoundParamsHost {
     const void *off;
     u64 *counter;
     u64 *stats;
-    unsigned *list_out;
+    u64 *list_out;
     unsigned *list_cnt;
     u64 prefix_begin, prefix_end;
     u64 cands_per_prefix;
@@ -179,6 +179,9 @@ struct BoundParamsHost {
     int sla;
     int prune_check;
     int zero;
+    const u64 *list_in;
+    const unsigned *list_n;
+    u64 list_upp;
     int nimin[SMILESS_MAX_FUNCS];
     const int *tabW;
     int fixed[SMILESS_MAX_FUNCS];
@@ -190,7 +193,7 @@ constexpr int kChunkUnits = 256;     // sharding / claim granularity in units (m
 struct JitKernel {
     CUmodule mod = nullptr;
     CUfunction fn = nullptr;
-    CUfunction fn_bound = nullptr;
+    CUfunction fn_bound = nullptr, fn_bound_a = nullptr;
     size_t smem = 0, smem_bound = 0;
     int blocks_per_sm = 0, blocks_bound = 0;
     int regs = 0;
@@ -253,7 +256,8 @@ struct smiless_ctx {
     DevBuf<i64> dLat;
     DevBuf<unsigned char> dFeas;
     DevBuf<double> dDump;
-    DevBuf<unsigned> dList, dListCnt;
+    DevBuf<u64> dList, dListA;
+    DevBuf<unsigned> dListCnt, dListCntA, dChunkCnt;
     DevBuf<int> dW;                          // per-row windows of the current plan (padded)
     DevBuf<ResBlock> dRes;
     ResBlock *hRes = nullptr;    // pinned [SMILESS_MAX_SLAS]
@@ -473,6 +477,28 @@ int bb_depth(const smiless_ctx *ctx, const smiless_plan_args *a) {
     return best;
 }
 
+// Shallow B&B level (two-level scheme): the deepest depth < D with at most 2^22 prefixes, if
+// the deep level has more than 2^24 prefixes (else 0: single level).  SMILESS_BB_DEPTH_A overrides.
+int bb_depth_a(const smiless_ctx *ctx, const smiless_plan_args *a, int D) {
+    if (D <= 0) return 0;
+    const int nf = a->n_fixed, W = a->n_windows;
+    const char *env = getenv("SMILESS_BB_DEPTH_A");
+    if (env) {
+        const int d = atoi(env);
+        return (d > nf && d < D) ? d : 0;
+    }
+    unsigned __int128 prefD = 1;
+    for (int k = nf; k < D; ++k) prefD *= (u64)ctx->M[k] * (u64)W;
+    if (prefD <= ((unsigned __int128)1 << 24)) return 0;
+    int best = 0;
+    unsigned __int128 pref = 1;
+    for (int d = nf + 1; d < D; ++d) {
+        pref *= (u64)ctx->M[d - 1] * (u64)W;
+        if (pref <= ((unsigned __int128)1 << 22)) best = d;
+    }
+    return best;
+}
+
 u64 cands_per_prefix(const smiless_ctx *ctx, const smiless_plan_args *a, int d) {
     u64 s = 1;
     for (int k = d; k < ctx->N; ++k) s *= (u64)ctx->M[k] * (u64)a->n_windows;
@@ -499,7 +525,9 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     const int check = std::max(unroll, ck_env ? atoi(ck_env) : 16);
     s << "#define SM_CHECK " << check << "\n";
     const int D = bb_depth(ctx, a);
-    s << "#define SM_D " << (D > 0 ? D : N - 1) << "\n#define SMILESS_MAXF " << SMILESS_MAX_FUNCS << "\n";
+    const int DA = bb_depth_a(ctx, a, D);
+    s << "#define SM_D " << (D > 0 ? D : N - 1) << "\n#define SM_DA " << (DA > 0 ? DA : (D > 0 ? D : N - 1))
+      << "\n#define SMILESS_MAXF " << SMILESS_MAX_FUNCS << "\n";
     s << "#define SM_NSLA " << ctx->nsla << "\n";
     s << "#define SM_ROWWIN " << (a->row_windows_us ? 1 : 0) << "\n";
     const char *mask_env = getenv("SMILESS_MASK");   // tuning knob, see evaluator.cuh SM_MASK
@@ -583,12 +611,13 @@ static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
     s << "  (void)NF; (void)o; (void)nlu;\n}\n";
     // ---- B&B pre-pass (smiless_bound_kernel): prefix decode, relaxed first/step ---------------
     {
-        const int Dg = D > 0 ? D : N - 1;
-        s << "static __device__ __forceinline__ void dag_bdecode(u64 u, int (&dig)[SM_N], const int *fixed) {\n";
+        s << "template <int DD> static __device__ __forceinline__ void dag_bdecode(u64 u, int (&dig)[SM_N], "
+             "const int *fixed) {\n";
         for (int k = 0; k < N; ++k) s << "  dig[" << k << "] = 0;\n";
-        for (int k = Dg - 1; k >= nf; --k) {
+        for (int k = N - 1; k >= nf; --k) {
             const u64 radix = (u64)ctx->M[k] * (u64)W;
-            s << "  dig[" << k << "] = (int)(u % " << radix << "ull); u /= " << radix << "ull;\n";
+            s << "  if (" << k << " < DD) { dig[" << k << "] = (int)(u % " << radix << "ull); u /= " << radix
+              << "ull; }\n";
         }
         for (int k = 0; k < nf; ++k) s << "  dig[" << k << "] = fixed[" << k << "];\n";
         s << "  (void)u; (void)fixed;\n}\n";
@@ -599,16 +628,16 @@ static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
         for (int k = 0; k < N; ++k)
             if ((ctx->sinkmask >> k) & 1ull) s << "  nl = vminz(nl, NF[" << k << "], z);\n";
         s << "  (void)z;\n}\n";
-        s << "template <int A> static __device__ __forceinline__ void dag_bstep(tm_t (&NF)[A], const tm_t (&NI)[A], "
-             "const tm_t (&Te)[A], const tm_t (&Wn)[A], const tm_t o, tm_t &nl, const tm_t z) {\n  tm_t su = 0;\n";
+        s << "template <int DD, int A> static __device__ __forceinline__ void dag_bstep(tm_t (&NF)[A], const tm_t "
+             "(&NI)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], const tm_t o, tm_t &nl, const tm_t z) {\n"
+             "  tm_t su = 0;\n";
         for (int k = 0; k < N; ++k) {
             const std::string g = is_src(k) ? "o + NF[" + std::to_string(k) + "]"
                                             : "NF[" + std::to_string(k) + "] - " + nf_min(k);
-            if (k < Dg)
-                s << "  fstep(NF[" << k << "], su, " << g << ", NI[" << k << "], Te[" << k << "], Wn[" << k << "]);\n";
-            else   // relaxed: keep-alive (start - f = max(g, 0)) with the smallest exec time
-                s << "  { const tm_t g = " << g << "; NF[" << k << "] = NF[" << k << "] + NI[" << k
-                  << "] - vmax(g, (tm_t)0); }\n";
+            // assigned (k < DD): model M; relaxed: keep-alive (start - f = max(g, 0)), smallest exec
+            s << "  if (" << k << " < DD) fstep(NF[" << k << "], su, " << g << ", NI[" << k << "], Te[" << k
+              << "], Wn[" << k << "]);\n  else { const tm_t g = " << g << "; NF[" << k << "] = NF[" << k
+              << "] + NI[" << k << "] - vmax(g, (tm_t)0); }\n";
         }
         for (int k = 0; k < N; ++k)
             if ((ctx->sinkmask >> k) & 1ull) s << "  nl = vaddmin(NF[" << k << "], o, nl);\n";
@@ -685,6 +714,8 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
         if (jk.blocks_per_sm < 1) return fail(ctx, SMILESS_ECUDA, "evaluator does not fit on an SM (smem %zu)", jk.smem);
         r = driver().moduleGetFunction(&jk.fn_bound, jk.mod, "smiless_bound_kernel");
         if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound)");
+        r = driver().moduleGetFunction(&jk.fn_bound_a, jk.mod, "smiless_bound_kernel_a");
+        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound_a)");
         {
             const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
             jk.smem_bound = 3 * padI * 4 + (rp.time64 ? 8 : 4) * (size_t)n_off;
@@ -692,6 +723,9 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
                 r = driver().funcSetAttribute(jk.fn_bound, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
                                               (int)jk.smem_bound);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(bound smem)");
+                r = driver().funcSetAttribute(jk.fn_bound_a, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
+                                              (int)jk.smem_bound);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(bound_a smem)");
                 r = driver().occupancy(&jk.blocks_bound, jk.fn_bound, kThreads, jk.smem_bound);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(bound)");
             }
@@ -795,6 +829,7 @@ void smiless_destroy(smiless_ctx *ctx) {
         ctx->dCounter.release(); ctx->dStats.release(); ctx->dBlk.release(); ctx->dIdxEval.release();
         ctx->dCost.release(); ctx->dLat.release(); ctx->dFeas.release(); ctx->dRes.release(); ctx->dDump.release();
         ctx->dList.release(); ctx->dListCnt.release(); ctx->dW.release();
+        ctx->dListA.release(); ctx->dListCntA.release(); ctx->dChunkCnt.release();
         if (ctx->hRes) cudaFreeHost(ctx->hRes);
         for (auto &ev : ctx->ev)
             if (ev) cudaEventDestroy(ev);
@@ -1090,34 +1125,97 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             for (int k = 0; k < a->n_fixed; ++k) bp.fixed[k] = a->fixed_digits[k];
             const int grid_b = jk->blocks_bound * ctx->n_sms;
             CK(cudaEventRecord(ctx->ev[1], st), "event");
-            u64 bi = 0;
-            for (u64 b0 = p_lo; b0 < p_hi; b0 += batch, ++bi) {
-                if (bi % (u64)n_shards != (u64)shard) continue;
-                const u64 b1 = std::min(p_hi, b0 + batch);
-                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
-                bp.prefix_begin = b0;
-                bp.prefix_end = b1;
-                void *bargs[] = {&bp};
-                CUresult r = driver().launchKernel(jk->fn_bound, (unsigned)grid_b, 1, 1, kThreads, 1, 1,
-                                                   (unsigned)jk->smem_bound, (CUstream)st, bargs, nullptr);
-                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "bound launch");
-                ++launches;
+            // evaluator over the deep survivors in dList (absolute depth-D prefix ids)
+            auto run_eval = [&]() -> int {
                 CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
                 pp.claims_begin = 0;
                 pp.claims_end = ~0ull;
                 pp.list_in = ctx->dList.p;
                 pp.list_n = ctx->dListCnt.p;
                 pp.list_upp = upp;
-                pp.list_base = b0 * upp;
+                pp.list_base = 0;
                 pp.list_out = nullptr;
                 pp.list_cnt = nullptr;
                 pp.horizon = 0;
                 void *args[] = {&pp};
-                r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
-                                          (CUstream)st, args, nullptr);
+                CUresult r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
+                                                   (CUstream)st, args, nullptr);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
                 ++launches;
+                return SMILESS_OK;
+            };
+            auto run_bound = [&](CUfunction fn) -> int {
+                void *bargs[] = {&bp};
+                CUresult r = driver().launchKernel(fn, (unsigned)grid_b, 1, 1, kThreads, 1, 1,
+                                                   (unsigned)jk->smem_bound, (CUstream)st, bargs, nullptr);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "bound launch");
+                ++launches;
+                return SMILESS_OK;
+            };
+            const int DA = bb_depth_a(ctx, a, D);
+            if (DA > 0) {
+                // ---- two levels: depth DA over every prefix, depth D over the DA survivors' children --
+                const u64 SA = cands_per_prefix(ctx, a, DA);
+                const u64 R = SA / S;                             // depth-D children per depth-DA prefix
+                const u64 a_lo = cb / SA, a_hi = (ce + SA - 1) / SA;
+                CK(ctx->dListA.ensure((size_t)batch), "cudaMalloc list");
+                CK(ctx->dListCntA.ensure(1), "cudaMalloc");
+                const u64 per_chunk = std::max<u64>(1, batch / R);   // shallow survivors per deep launch
+                u64 bi = 0;
+                for (u64 b0 = a_lo; b0 < a_hi; b0 += batch, ++bi) {
+                    if (bi % (u64)n_shards != (u64)shard) continue;
+                    const u64 b1 = std::min(a_hi, b0 + batch);
+                    CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                    CK(cudaMemsetAsync(ctx->dListCntA.p, 0, sizeof(unsigned), st), "memset list");
+                    bp.list_in = nullptr;
+                    bp.list_n = nullptr;
+                    bp.list_upp = 1;
+                    bp.prefix_begin = b0;
+                    bp.prefix_end = b1;
+                    bp.cands_per_prefix = SA;
+                    bp.list_out = ctx->dListA.p;
+                    bp.list_cnt = ctx->dListCntA.p;
+                    if ((rc = run_bound(jk->fn_bound_a))) return rc;
+                    unsigned n_a = 0;
+                    CK(cudaMemcpyAsync(&n_a, ctx->dListCntA.p, sizeof n_a, cudaMemcpyDeviceToHost, st), "D2H count");
+                    CK(cudaStreamSynchronize(st), "count");
+                    // per-chunk entry counts, uploaded once (no host sync inside the loop)
+                    const u64 n_chunks_a = (n_a + per_chunk - 1) / per_chunk;
+                    std::vector<unsigned> cnts((size_t)std::max<u64>(1, n_chunks_a));
+                    for (u64 i = 0; i < n_chunks_a; ++i)
+                        cnts[i] = (unsigned)std::min<u64>(per_chunk, n_a - i * per_chunk);
+                    CK(ctx->dChunkCnt.ensure(cnts.size()), "cudaMalloc counts");
+                    CK(cudaMemcpy(ctx->dChunkCnt.p, cnts.data(), cnts.size() * sizeof(unsigned), cudaMemcpyHostToDevice),
+                       "H2D counts");
+                    for (u64 i = 0; i < n_chunks_a; ++i) {
+                        const u64 c0 = i * per_chunk;
+                        CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                        CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
+                        bp.list_in = ctx->dListA.p + c0;
+                        bp.list_n = ctx->dChunkCnt.p + i;
+                        bp.list_upp = R;
+                        bp.prefix_begin = 0;
+                        bp.prefix_end = ~0ull;
+                        bp.cands_per_prefix = S;
+                        bp.list_out = ctx->dList.p;
+                        bp.list_cnt = ctx->dListCnt.p;
+                        if ((rc = run_bound(jk->fn_bound))) return rc;
+                        if ((rc = run_eval())) return rc;
+                    }
+                    CK(cudaStreamSynchronize(st), "chunks");      // cnts must outlive its uploads
+                }
+            } else {
+                u64 bi = 0;
+                for (u64 b0 = p_lo; b0 < p_hi; b0 += batch, ++bi) {
+                    if (bi % (u64)n_shards != (u64)shard) continue;
+                    const u64 b1 = std::min(p_hi, b0 + batch);
+                    CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                    CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
+                    bp.prefix_begin = b0;
+                    bp.prefix_end = b1;
+                    if ((rc = run_bound(jk->fn_bound))) return rc;
+                    if ((rc = run_eval())) return rc;
+                }
             }
         } else {
             // split very large ranges into several launches (bounded kernel duration).  Prune mode

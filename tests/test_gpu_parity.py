@@ -536,3 +536,34 @@ def test_top1_never_beats_exhaustive_opt():
         opt = pl.plan(p.arrivals_us, p.sla_us, [0], row_windows=rw)
         if h.feasible:
             assert opt.feasible and opt.cost <= h.cost
+
+
+def test_two_level_branch_and_bound_is_exact(monkeypatch):
+    """Shallow level (depth DA over every prefix) + deep level (depth D over the shallow
+    survivors' children, list mode) + evaluator: same per-candidate results and winners."""
+    rng = np.random.default_rng(53)
+    n_checked = 0
+    for t in range(30):
+        n = int(rng.integers(4, 7))
+        p = W.random_problem(rng, n, 3, int(rng.integers(2, 4)), int(rng.integers(20, 160)),
+                             sla_us=int(rng.integers(15_000, 60_000)))
+        space = p.space_size()
+        if space > 30000:
+            continue
+        o = OracleProblem(p)
+        oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
+        ref = o.plan()
+        for d in range(2, n):
+            for da in range(1, d):
+                monkeypatch.setenv("SMILESS_BB_DEPTH", str(d))
+                monkeypatch.setenv("SMILESS_BB_DEPTH_A", str(da))
+                pl = S.planner_for(p)
+                out = np.empty(space)
+                g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, cost_out=out)
+                assert_dump_matches(out, oc, of)
+                assert_same_plan(g, ref, o)
+                assert g.n_decided == space
+                parts = [pl.plan(p.arrivals_us, p.sla_us, p.windows_us, shard=s_, n_shards=2) for s_ in range(2)]
+                assert sum(r.n_decided for r in parts) == space
+        n_checked += 1
+    assert n_checked > 8
