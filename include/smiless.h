@@ -60,7 +60,7 @@ enum {
     SMILESS_INFEASIBLE = 1,  /* success, but no candidate meets the SLA (reading G13)  */
     SMILESS_EINVAL = -1,     /* bad argument (null, size, range, unsorted arrivals ...) */
     SMILESS_ENOTTOPO = -2,   /* DAG not a topologically ordered predecessor CSR         */
-    SMILESS_ERANGE = -3,     /* candidate space or index exceeds 2^63-1                 */
+    SMILESS_ERANGE = -3,     /* candidate space exceeds 2^63 (indices must fit int64)   */
     SMILESS_ESTATE = -4,     /* call order: plan/evaluate before load_dag+load_profiles */
     SMILESS_ECUDA = -5,      /* CUDA runtime/driver failure or no device                */
     SMILESS_ENOMEM = -6,     /* host or device allocation failed                        */
@@ -153,7 +153,7 @@ typedef struct {
 } smiless_plan_result;
 
 /* Size of the suffix candidate space prod_{k >= n_fixed} M_k * W.
- * Returns OK, ESTATE (profiles not loaded), EINVAL or ERANGE (> 2^63-1). */
+ * Returns OK, ESTATE (profiles not loaded), EINVAL or ERANGE (> 2^63). */
 SMILESS_API int smiless_space_size(const smiless_ctx *ctx, int32_t n_windows, int32_t n_fixed, uint64_t *out);
 
 /* The hot path: exhaustive SLA-constrained min-cost search over [begin, end)

@@ -60,12 +60,12 @@ static int64_t row0(const oracle_problem *P, int k) {
 }
 
 /* Size of the (suffix) candidate space: prod_{k >= n_fixed} M_k * W.
-   Returns 0 on overflow past 2^63-1. */
+   Returns 0 above 2^63 (every index must fit an int64). */
 uint64_t oracle_space_size(const oracle_problem *P) {
     unsigned __int128 s = 1;
     for (int k = P->n_fixed; k < P->n_funcs; ++k) {
         s *= (unsigned __int128)((uint64_t)P->n_configs[k] * (uint64_t)P->n_windows);
-        if (s > (unsigned __int128)INT64_MAX) return 0;
+        if (s > ((unsigned __int128)1 << 63)) return 0;
     }
     return (uint64_t)s;
 }

@@ -359,7 +359,7 @@ bool space_size_of(const smiless_ctx *c, int W, int n_fixed, u64 *out) {
     unsigned __int128 s = 1;
     for (int k = n_fixed; k < c->N; ++k) {
         s *= (unsigned __int128)((u64)c->M[k] * (u64)W);
-        if (s > (unsigned __int128)INT64_MAX) return false;
+        if (s > ((unsigned __int128)1 << 63)) return false;   // indices 0 .. 2^63-1 fit int64
     }
     *out = (u64)s;
     return true;
