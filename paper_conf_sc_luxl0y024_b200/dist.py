@@ -73,3 +73,21 @@ def plan_distributed(planner, arrivals, sla_us, windows_us, group=None, device=N
         return None, None, -1, np.full(n, -1, np.int32), np.full(n, -1, np.int32), decided, r
     c, w = planner.decode(index, len(windows_us), kw.get("n_fixed", 0), kw.get("fixed_digits", ()))
     return cost, index, lat, c, w, decided, r
+
+
+def reduce_lex(keys, payload, device, group=None):
+    """Lexicographic MIN across ranks of an int64 key tuple (e.g. cost bits, pinned digit,
+    suffix index) by successive MIN all-reduces, each over the ranks still tied; `payload`
+    (int64s) comes from the unique owner of the minimum.  Returns (keys, payload)."""
+    BIG = (1 << 63) - 1
+    tied = True
+    out = []
+    for k in keys:
+        t = torch.tensor([int(k) if tied else BIG], dtype=torch.int64, device=device)
+        dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+        v = int(t.item())
+        tied = tied and int(k) == v
+        out.append(v)
+    s = torch.tensor([int(x) if tied else 0 for x in payload], dtype=torch.int64, device=device)
+    dist.all_reduce(s, op=dist.ReduceOp.SUM, group=group)
+    return out, [int(x) for x in s.tolist()]
