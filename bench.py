@@ -177,12 +177,13 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
         if r.feasible and (best is None or (r.cost, d0 or 0, r.index) < best[:3]):
             best = (r.cost, d0 or 0, r.index, r.max_latency_us)
     keys = [cost_bits(best[0]) if best else INF_BITS, best[1] if best else 0, best[2] if best else 0]
-    payload = [best[3] if best else -1, decided]
+    payload = [best[3] if best else -1]
     if world > 1:
         keys, pay = reduce_lex(keys, payload, xdev)
-        tot = torch.tensor([decided], dtype=torch.int64, device=xdev)
-        dist.all_reduce(tot)
-        decided = int(tot.item())
+        # C5 decides 2^70 candidates: exceeds int64, so sum as two int64 halves
+        hi_lo = torch.tensor([decided >> 32, decided & 0xffffffff], dtype=torch.int64, device=xdev)
+        dist.all_reduce(hi_lo)
+        decided = (int(hi_lo[0].item()) << 32) + int(hi_lo[1].item())
         lat = pay[0]
     else:
         lat = payload[0]
