@@ -400,6 +400,7 @@ def main():
     pruned = None
     if not args.no_pruned:
         kwp = dict(kw, flags=0, shard=rank, n_shards=world)
+        pl.plan(arr_dev, p.sla_us, p.windows_us, **kwp)          # NVRTC compile of the prune-mode kernels
         barrier()
         a = torch.cuda.Event(enable_timing=True)
         b = torch.cuda.Event(enable_timing=True)
