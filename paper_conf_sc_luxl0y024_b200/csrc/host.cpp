@@ -187,7 +187,16 @@ struct BoundParamsHost {
     int fixed[SMILESS_MAX_FUNCS];
 };
 
-constexpr int kThreads = 256;
+// CTA size of the evaluator / bound kernels (SMILESS_THREADS tunes it; multiple of 32, <= 1024).
+int threads_per_cta() {
+    static const int t = [] {
+        const char *e = getenv("SMILESS_THREADS");
+        const int v = e ? atoi(e) : 256;
+        return (v >= 64 && v <= 1024 && v % 32 == 0) ? v : 256;
+    }();
+    return t;
+}
+#define kThreads threads_per_cta()
 constexpr int kChunkUnits = 256;     // sharding / claim granularity in units (multiple of 32)
 
 struct JitKernel {
@@ -259,6 +268,7 @@ struct smiless_ctx {
     DevBuf<u64> dList, dListA;
     DevBuf<unsigned> dListCnt, dListCntA, dChunkCnt;
     DevBuf<int> dW;                          // per-row windows of the current plan (padded)
+    std::vector<int> hW;                     // host copy of what dW holds
     DevBuf<ResBlock> dRes;
     ResBlock *hRes = nullptr;    // pinned [SMILESS_MAX_SLAS]
     int nsla = 1;                // argmin keys of the plan being compiled (SLA sweep)
@@ -764,9 +774,10 @@ int stage_row_windows(smiless_ctx *ctx, const smiless_plan_args *a) {
     const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
     std::vector<int> w(padI, 0);
     if (a->row_windows_us) std::copy(a->row_windows_us, a->row_windows_us + ctx->sumM, w.begin());
+    if (ctx->dW.p && ctx->dW.n >= padI && w == ctx->hW && !ctx->tables_dirty) return SMILESS_OK;  // unchanged
     CK(ctx->dW.ensure(padI), "cudaMalloc row windows");
-    CK(cudaMemcpyAsync(ctx->dW.p, w.data(), padI * sizeof(int), cudaMemcpyHostToDevice, ctx->stream), "H2D windows");
-    CK(cudaStreamSynchronize(ctx->stream), "H2D windows");
+    CK(cudaMemcpy(ctx->dW.p, w.data(), padI * sizeof(int), cudaMemcpyHostToDevice), "H2D windows");
+    ctx->hW.swap(w);
     return SMILESS_OK;
 }
 

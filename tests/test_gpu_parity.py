@@ -567,3 +567,35 @@ def test_two_level_branch_and_bound_is_exact(monkeypatch):
                 assert sum(r.n_decided for r in parts) == space
         n_checked += 1
     assert n_checked > 8
+
+
+def test_branch_and_bound_with_pinned_digits(monkeypatch):
+    """B&B levels count from the pinned prefix (n_fixed > 0): per-candidate parity with the
+    oracle on the suffix space, for single and two-level schemes."""
+    rng = np.random.default_rng(59)
+    n_checked = 0
+    for t in range(30):
+        n = int(rng.integers(4, 7))
+        p = W.random_problem(rng, n, 3, int(rng.integers(2, 4)), int(rng.integers(20, 150)),
+                             sla_us=int(rng.integers(15_000, 60_000)))
+        Wn = len(p.windows_us)
+        nf = int(rng.integers(1, 3))
+        fixed = [int(rng.integers(0, p.n_configs[k] * Wn)) for k in range(nf)]
+        o = OracleProblem(p, n_fixed=nf, fixed_digits=fixed)
+        space = o.space_size()
+        if space > 30000 or space < 64:
+            continue
+        oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
+        ref = o.plan()
+        for d in range(nf + 1, n):
+            for da in [0] + list(range(nf + 1, d)):
+                monkeypatch.setenv("SMILESS_BB_DEPTH", str(d))
+                monkeypatch.setenv("SMILESS_BB_DEPTH_A", str(da))
+                pl = S.planner_for(p)
+                out = np.empty(space)
+                g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, n_fixed=nf, fixed_digits=fixed, cost_out=out)
+                assert_dump_matches(out, oc, of)
+                assert_same_plan(g, ref, o)
+                assert g.n_decided == space
+        n_checked += 1
+    assert n_checked > 8
