@@ -1299,13 +1299,13 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         CK(cudaEventRecord(ctx->ev[1], st), "event");
         CK(cudaEventRecord(ctx->ev[2], st), "event");
     }
-    // a10: exact int64 re-evaluation of each winner (also decodes its digits)
-    for (int s_ = 0; s_ < n_sla; ++s_) {
+    // a10: exact int64 re-evaluation of each winner (also decodes its digits), one thread per SLA
+    {
         ExactParams ep;
         fill_exact_params(ctx, a, d_arr, ep);
-        ep.sla = slas[s_];
-        ep.n = 1;
-        ep.res = ctx->dRes.p + s_;
+        for (int s_ = 0; s_ < n_sla; ++s_) ep.slas[s_] = slas[s_];
+        ep.n = n_sla;
+        ep.res = ctx->dRes.p;
         ep.idx_from_res = 1;
         e = smiless_dev_eval_exact(&ep, st);
         if (e) return cuda_fail(ctx, (cudaError_t)e, "eval_exact launch");

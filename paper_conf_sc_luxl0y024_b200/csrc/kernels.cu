@@ -80,9 +80,11 @@ __global__ void reduce_best_kernel(const u64 *__restrict__ slots, int n, int str
 __global__ void eval_exact_kernel(ExactParams p) {
     const i64 t = (i64)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= p.n) return;
-    u64 index = p.idx_from_res ? p.res->best_i : p.idx[t];
+    ResBlock *res = p.idx_from_res ? p.res + t : nullptr;
+    const i64 sla = p.idx_from_res ? p.slas[t] : p.sla;
+    u64 index = p.idx_from_res ? res->best_i : p.idx[t];
     if (index == ~0ull) {
-        if (p.idx_from_res) { p.res->feasible = 0; p.res->cost = 0.0; p.res->maxlat = -1; }
+        if (res) { res->feasible = 0; res->cost = 0.0; res->maxlat = -1; }
         return;
     }
     const int N = p.N, W = p.W;
@@ -148,9 +150,8 @@ __global__ void eval_exact_kernel(ExactParams p) {
         const double term = __dmul_rn(p.tabU[p.row0[k] + cfg[k]], (double)billed[k]);
         cost = (k == 0) ? term : __dadd_rn(cost, term);
     }
-    const unsigned char ok = maxlat <= p.sla ? 1 : 0;
-    if (p.idx_from_res) {
-        ResBlock *res = p.res;
+    const unsigned char ok = maxlat <= sla ? 1 : 0;
+    if (res) {
         res->cost = cost;
         res->maxlat = maxlat;
         res->feasible = ok;

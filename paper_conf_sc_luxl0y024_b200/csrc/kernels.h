@@ -31,9 +31,10 @@ struct ExactParams {
     double *cost;
     long long *maxlat;
     unsigned char *feas;
-    ResBlock *res;               // when idx_from_res: evaluate res->best_i, write into res
+    ResBlock *res;               // when idx_from_res: thread t evaluates res[t].best_i with slas[t]
     int idx_from_res;
     long long sla;
+    long long slas[8];
     int N, W, n_fixed;
     unsigned sinkmask;
     const int *pred_ptr;         // device [N+1]
