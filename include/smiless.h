@@ -210,6 +210,21 @@ SMILESS_API int smiless_autoscale(const smiless_ctx *ctx, const double *slope_us
                                   const int64_t *invocations, int64_t it_us, const int64_t *target_us,
                                   smiless_autoscale_result *out);
 
+/* NEXT-3: SMIless's handling of complex DAGs: decompose the DAG into its
+ * source-to-sink paths (subgraphs with only sequential dependencies), optimise each path
+ * with the Top-1 walk using the paper's O(1) closed-form latency (sum of I along the path,
+ * Eq. (5)) and per-invocation cost (U (T + I) / U IT), then combine: a function on
+ * several paths with different choices takes the fastest of them (the paper's rule for the
+ * start/end F_s, F_e of parallel substructures), and every function on a single path is
+ * moved to its cheapest config that keeps that path's closed-form latency at or below its
+ * latency before combining.  Windows per row from a->row_windows_us (n_windows == 1,
+ * n_fixed == 0).  The combined plan is evaluated on the GPU with model M; res /
+ * config_out / window_out / *n_paths report it (INFEASIBLE if it misses the SLA under
+ * model M).  At most 4096 paths. */
+SMILESS_API int smiless_decompose_search(smiless_ctx *ctx, const smiless_plan_args *a, int64_t it_us,
+                                         smiless_plan_result *res, int32_t *config_out, int32_t *window_out,
+                                         int64_t *n_paths);
+
 /* SLA sweep (C4: "impact of SLA settings"): ONE evaluation of the space
  * with one argmin key per SLA in slas[0..n_sla) (1 <= n_sla <= SMILESS_MAX_SLAS); pruning uses
  * their maximum; a->sla_us is ignored and a->cost_out must be NULL.  res[n_sla] and, when not

@@ -17,6 +17,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <functional>
 #include <map>
 #include <memory>
 #include <mutex>
@@ -1532,6 +1533,130 @@ int smiless_autoscale(const smiless_ctx *ctx, const double *slope_us, const doub
         }
         out[k] = best;
     }
+    return SMILESS_OK;
+}
+
+int smiless_decompose_search(smiless_ctx *ctx, const smiless_plan_args *a, int64_t it_us, smiless_plan_result *res,
+                             int32_t *config_out, int32_t *window_out, int64_t *n_paths) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->err.clear();
+    if (!a || !res) return fail(ctx, SMILESS_EINVAL, "args / res is NULL");
+    if (!a->row_windows_us) return fail(ctx, SMILESS_EINVAL, "decompose search needs row_windows_us (n_windows == 1)");
+    if (a->n_fixed != 0) return fail(ctx, SMILESS_EINVAL, "decompose search does not take pinned digits");
+    int rc = validate_args(ctx, a, true);
+    if (rc) return rc;
+    const int N = ctx->N;
+    // successors and source -> sink paths (DFS)
+    std::vector<std::vector<int>> succ(N);
+    for (int k = 0; k < N; ++k)
+        for (int e = ctx->pred_ptr[k]; e < ctx->pred_ptr[k + 1]; ++e) succ[ctx->pred_idx[e]].push_back(k);
+    std::vector<std::vector<int>> paths;
+    std::vector<int> cur;
+    bool too_many = false;
+    std::function<void(int)> walk = [&](int k) {
+        if (too_many) return;
+        cur.push_back(k);
+        if (succ[k].empty()) {
+            paths.push_back(cur);
+            if (paths.size() > 4096) too_many = true;
+        }
+        for (int s_ : succ[k]) walk(s_);
+        cur.pop_back();
+    };
+    for (int k = 0; k < N; ++k)
+        if (ctx->pred_ptr[k] == ctx->pred_ptr[k + 1]) walk(k);
+    if (too_many) return fail(ctx, SMILESS_EINVAL, "more than 4096 source-to-sink paths");
+    // per-function cost ranking (Eq. 5 / Case II) and fastest config
+    auto per_inv_cost = [&](int k, int m) {
+        const int row = ctx->row0[k] + m;
+        const i64 t = ctx->T[row], i = ctx->I[row];
+        return ctx->U[row] * ((t + i < it_us) ? (double)(t + i) : (double)it_us);
+    };
+    auto I_of = [&](int k, int m) { return (i64)ctx->I[ctx->row0[k] + m]; };
+    std::vector<std::vector<int>> rank(N);
+    std::vector<int> fastest(N);
+    for (int k = 0; k < N; ++k) {
+        std::vector<int> o(ctx->M[k]);
+        for (int m = 0; m < ctx->M[k]; ++m) o[m] = m;
+        std::stable_sort(o.begin(), o.end(), [&](int x, int y) { return per_inv_cost(k, x) < per_inv_cost(k, y); });
+        rank[k] = o;
+        int f = 0;
+        for (int m = 1; m < ctx->M[k]; ++m)
+            if (I_of(k, m) < I_of(k, f)) f = m;
+        fastest[k] = f;
+    }
+    const i64 sla = a->sla_us;
+    // Top-1 per path with the closed-form latency sum(I)
+    std::vector<std::vector<int>> choice(paths.size());
+    for (size_t pi = 0; pi < paths.size(); ++pi) {
+        const auto &P = paths[pi];
+        const size_t L = P.size();
+        std::vector<int> c(L);
+        i64 lat = 0;
+        for (size_t q = 0; q < L; ++q) { c[q] = rank[P[q]][0]; lat += I_of(P[q], c[q]); }
+        if (lat > sla) {
+            std::vector<int> chosen;
+            for (size_t q = 0; q < L; ++q) {
+                int pick = fastest[P[q]];
+                for (int r = (q == 0 ? 1 : 0); r < ctx->M[P[q]]; ++r) {
+                    i64 l = 0;
+                    for (size_t z = 0; z < L; ++z)
+                        l += I_of(P[z], z < q ? chosen[z] : (z == q ? rank[P[q]][r] : fastest[P[z]]));
+                    if (l <= sla) { pick = rank[P[q]][r]; break; }
+                }
+                chosen.push_back(pick);
+            }
+            c = chosen;
+        }
+        choice[pi] = c;
+    }
+    // combine: shared functions take the fastest of the paths' choices ...
+    std::vector<int> cfg(N, -1), n_on(N, 0);
+    std::vector<i64> path_lat(paths.size(), 0);
+    for (size_t pi = 0; pi < paths.size(); ++pi)
+        for (size_t q = 0; q < paths[pi].size(); ++q) {
+            const int k = paths[pi][q], m = choice[pi][q];
+            path_lat[pi] += I_of(k, m);
+            n_on[k] += 1;
+            if (cfg[k] < 0 || I_of(k, m) < I_of(k, cfg[k])) cfg[k] = m;
+        }
+    // ... and functions on a single path move to their cheapest config that keeps that path's
+    // closed-form latency at or below its latency before combining
+    for (size_t pi = 0; pi < paths.size(); ++pi) {
+        const auto &P = paths[pi];
+        for (size_t q = 0; q < P.size(); ++q) {
+            const int k = P[q];
+            if (n_on[k] != 1) continue;
+            i64 others = 0;
+            for (size_t z = 0; z < P.size(); ++z)
+                if (z != q) others += I_of(P[z], cfg[P[z]]);
+            for (int r = 0; r < ctx->M[k]; ++r)
+                if (others + I_of(k, rank[k][r]) <= path_lat[pi]) { cfg[k] = rank[k][r]; break; }
+        }
+    }
+    // evaluate the combined plan with model M on the GPU
+    u64 idx = 0;
+    for (int k = 0; k < N; ++k) idx = idx * (u64)ctx->M[k] + (u64)cfg[k];
+    double cost = 0.0;
+    int64_t lat = 0;
+    uint8_t ok = 0;
+    if ((rc = smiless_evaluate(ctx, a, (const uint64_t *)&idx, 1, &cost, &lat, &ok))) return rc;
+    memset(res, 0, sizeof *res);
+    res->n_decided = res->n_full_evals = 1;
+    if (n_paths) *n_paths = (int64_t)paths.size();
+    for (int k = 0; k < N; ++k) {
+        if (config_out) config_out[k] = ok ? cfg[k] : -1;
+        if (window_out) window_out[k] = ok ? 0 : -1;
+    }
+    if (!ok) {
+        res->index = ~0ull;
+        res->cost = HUGE_VAL;
+        res->max_latency_us = -1;
+        return SMILESS_INFEASIBLE;
+    }
+    res->index = idx;
+    res->cost = cost;
+    res->max_latency_us = lat;
     return SMILESS_OK;
 }
 

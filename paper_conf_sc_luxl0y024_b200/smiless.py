@@ -25,7 +25,8 @@ _NAMES = {0: "OK", 1: "INFEASIBLE", -1: "EINVAL", -2: "ENOTTOPO", -3: "ERANGE", 
 # every symbol include/smiless.h declares (checked by tests/test_abi.py)
 EXPORTS = ("smiless_create", "smiless_set_stream", "smiless_destroy", "smiless_last_error",
            "smiless_load_dag", "smiless_load_profiles", "smiless_space_size", "smiless_plan",
-           "smiless_plan_sla_sweep", "smiless_derive_windows", "smiless_top1_search", "smiless_autoscale",
+           "smiless_plan_sla_sweep", "smiless_derive_windows", "smiless_top1_search", "smiless_decompose_search",
+           "smiless_autoscale",
            "smiless_evaluate",
            "smiless_decode",
            "smiless_kernel_source", "smiless_jit_compile")
@@ -118,6 +119,8 @@ def load_library(build_if_missing: bool = True):
                                            vp, vp]
     lib.smiless_derive_windows.argtypes = [vp, i64, vp]
     lib.smiless_autoscale.argtypes = [vp, vp, vp, vp, i64, vp, vp]
+    lib.smiless_decompose_search.argtypes = [vp, ctypes.POINTER(PlanArgs), i64, ctypes.POINTER(PlanResultC), vp,
+                                             vp, ctypes.POINTER(ctypes.c_int64)]
     lib.smiless_top1_search.argtypes = [vp, ctypes.POINTER(PlanArgs), i64, ctypes.POINTER(PlanResultC), vp, vp,
                                         ctypes.POINTER(ctypes.c_int64)]
     lib.smiless_evaluate.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i64, vp, vp, vp]
@@ -298,6 +301,22 @@ class Planner:
                           max_latency_us=int(r.max_latency_us), config=cfg[:self.n_funcs],
                           window=win[:self.n_funcs], n_decided=int(r.n_decided), n_full_evals=int(r.n_full_evals),
                           eval_kernel_ms=0.0, total_device_ms=0.0, int64_path=False, launches=0), int(nodes.value)
+
+    def decompose_search(self, arrivals, sla_us, it_us, row_windows, **kw):
+        """SMIless's DAG decomposition + combine (smiless_decompose_search); (PlanResult, paths)."""
+        a, keep = self._args(arrivals, sla_us, [0], row_windows=row_windows, **kw)
+        r = PlanResultC()
+        cfg = np.zeros(max(self.n_funcs, 1), np.int32)
+        win = np.zeros(max(self.n_funcs, 1), np.int32)
+        n = ctypes.c_int64()
+        rc = self._check(self._lib.smiless_decompose_search(self._ctx, ctypes.byref(a), int(it_us), ctypes.byref(r),
+                                                            cfg.ctypes.data, win.ctypes.data, ctypes.byref(n)),
+                         allow=(OK, INFEASIBLE))
+        del keep
+        return PlanResult(status=rc, index=None if rc == INFEASIBLE else int(r.index), cost=float(r.cost),
+                          max_latency_us=int(r.max_latency_us), config=cfg[:self.n_funcs],
+                          window=win[:self.n_funcs], n_decided=1, n_full_evals=1, eval_kernel_ms=0.0,
+                          total_device_ms=0.0, int64_path=False, launches=0), int(n.value)
 
     def evaluate(self, idx, arrivals, sla_us, windows_us, **kw) -> Tuple[np.ndarray, np.ndarray, np.ndarray]:
         a, keep = self._args(arrivals, sla_us, windows_us, **kw)

@@ -599,3 +599,24 @@ def test_branch_and_bound_with_pinned_digits(monkeypatch):
                 assert g.n_decided == space
         n_checked += 1
     assert n_checked > 8
+
+
+# ---------------------------------------------------------------------------------------
+# NEXT-3: DAG decomposition into sequential paths + combine
+# ---------------------------------------------------------------------------------------
+
+def test_decompose_search_matches_oracle_steps():
+    from oracle.decompose import decompose_search
+    rng = np.random.default_rng(91)
+    for t in range(30):
+        n = int(rng.integers(1, 8))
+        p = W.random_problem(rng, n, 6, 1, int(rng.integers(2, 80)), sla_us=int(rng.integers(5_000, 40_000)))
+        p = p.replace(windows_us=np.array([0], np.int32))
+        it = int(np.diff(p.arrivals_us).mean()) if len(p.arrivals_us) > 1 else 0
+        pl = S.planner_for(p)
+        rw = pl.derive_windows(it)
+        g, n_paths = pl.decompose_search(p.arrivals_us, p.sla_us, it, rw)
+        cfg, cost, lat, ok, onp = decompose_search(p, it, rw, OracleProblem)
+        assert n_paths == onp and g.feasible == ok
+        if ok:
+            assert g.config.tolist() == cfg and g.cost == cost and g.max_latency_us == lat
