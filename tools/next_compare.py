@@ -1,4 +1,4 @@
-"""NEXT-1 / NEXT-2 on the BASELINE configs: exhaustive OPT over configs x window grid vs
+"""NEXT-1 / NEXT-2 / NEXT-3 on the BASELINE configs: exhaustive OPT over configs x window grid vs
 exhaustive OPT under the paper's derived windows (NEXT-1) vs SMIless's Top-1 path search
 (NEXT-2, the paper's deployed heuristic), all exact under model M on one GPU.  This is the
 paper's Fig. 8 comparison "SMIless vs OPT (exhaustive search)" on synthetic inputs."""
@@ -18,10 +18,21 @@ def run(name, p, check=True):
     it = int(np.diff(p.arrivals_us).mean())
     out = {"config": name, "J": len(p.arrivals_us), "IT_us": it}
     t0 = time.perf_counter()
-    full = pl.plan(arr, p.sla_us, p.windows_us)
+    Wn = len(p.windows_us)
+    try:
+        full = pl.plan(arr, p.sla_us, p.windows_us)
+        space = pl.space_size(Wn)
+        fixed = {}
+    except S.SmilessError:                       # > 2^63 (C5): pin function 0's digit, 128 sub-plans
+        best, space = None, 0
+        for d0 in range(int(p.n_configs[0]) * Wn):
+            r = pl.plan(arr, p.sla_us, p.windows_us, n_fixed=1, fixed_digits=[d0])
+            space += r.n_decided
+            if r.feasible and (best is None or (r.cost, d0, r.index) < (best[0].cost, best[1], best[0].index)):
+                best = (r, d0)
+        full, fixed = best[0], dict(n_fixed=1, fixed_digits=[best[1]])
     out["opt_grid"] = {"cost": full.cost if full.feasible else None, "s": time.perf_counter() - t0,
-                       "config": full.config.tolist(), "window": full.window.tolist(),
-                       "candidates": pl.space_size(len(p.windows_us))}
+                       "config": full.config.tolist(), "window": full.window.tolist(), "candidates": space}
     q = p.replace(windows_us=np.array([0], np.int32))
     plq = S.planner_for(q, stream=stream)
     rw = plq.derive_windows(it)
@@ -33,12 +44,18 @@ def run(name, p, check=True):
     h, nodes = plq.top1_search(p.arrivals_us, q.sla_us, it, rw)
     out["top1_search"] = {"cost": h.cost if h.feasible else None, "s": time.perf_counter() - t0, "nodes": nodes,
                           "config": h.config.tolist()}
+    t0 = time.perf_counter()
+    dc, n_paths = plq.decompose_search(p.arrivals_us, q.sla_us, it, rw)
+    out["decompose_search"] = {"cost": dc.cost if dc.feasible else None, "s": time.perf_counter() - t0,
+                               "paths": n_paths, "config": dc.config.tolist()}
+    if full.feasible and dc.feasible:
+        out["decompose_over_opt"] = dc.cost / full.cost
     if full.feasible and h.feasible:
         out["top1_over_opt"] = h.cost / full.cost
     if full.feasible and der.feasible:
         out["derived_over_opt"] = der.cost / full.cost
     if check and full.feasible:
-        c, l, f = OracleProblem(p).evaluate([full.index])
+        c, l, f = OracleProblem(p, **fixed).evaluate([full.index])
         out["opt_grid"]["oracle_check"] = bool(f[0] and c[0] == full.cost and l[0] == full.max_latency_us)
     return out
 
