@@ -162,6 +162,32 @@ struct PlanParamsHost {
     int fixed[SMILESS_MAX_FUNCS];  // evaluator uses SM_NFIXED_ALLOC <= SMILESS_MAX_FUNCS; extra tail is ignored
 };
 
+// Mirror of MemoParams (evaluator.cuh, prefix memoisation kernels).
+struct MemoParamsHost {
+    const int *tabNI, *tabT, *tabW;
+    const double *tabU;
+    const void *off;
+    const i64 *scal;
+    u64 *counter;
+    u64 *stats;
+    u64 *blk_best;
+    void *xbuf;
+    void *rec_nx;
+    double *rec_pre;
+    void *rec_nlu;
+    double *dump;
+    u64 pref_begin, pref_end;
+    u64 unit_begin, unit_end;
+    u64 cand_begin, cand_end;
+    i64 n_steps;
+    i64 n_off;
+    int sumM;
+    int sla;
+    int zero;
+    int slas[8];
+    int fixed[SMILESS_MAX_FUNCS];
+};
+
 // Mirror of BoundParams (evaluator.cuh, B&B pre-pass kernel).
 struct BoundParamsHost {
     const int *tabNI;
@@ -203,7 +229,9 @@ constexpr int kChunkUnits = 256;     // sharding / claim granularity in units (m
 struct JitKernel {
     CUmodule mod = nullptr;
     CUfunction fn = nullptr;
-    CUfunction fn_bound = nullptr, fn_bound_a = nullptr;
+    CUfunction fn_bound = nullptr, fn_bound_a = nullptr, fn_up = nullptr, fn_var = nullptr;
+    size_t smem_up = 0, smem_var = 0;
+    int blocks_up = 0, blocks_var = 0;
     size_t smem = 0, smem_bound = 0;
     int blocks_per_sm = 0, blocks_bound = 0;
     int regs = 0;
@@ -269,6 +297,9 @@ struct smiless_ctx {
     DevBuf<u64> dList, dListA;
     DevBuf<unsigned> dListCnt, dListCntA, dChunkCnt;
     DevBuf<int> dW;                          // per-row windows of the current plan (padded)
+    DevBuf<unsigned char> dX;                // memoised last-function inputs [prefix][n_off]
+    DevBuf<i64> dRecNx, dRecNlu;             // per-prefix records (int32 or int64 time)
+    DevBuf<double> dRecPre;
     std::vector<int> hW;                     // host copy of what dW holds
     DevBuf<ResBlock> dRes;
     ResBlock *hRes = nullptr;    // pinned [SMILESS_MAX_SLAS]
@@ -532,6 +563,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
       << "\n#define SM_MINB " << minb << "\n";
     s << "#define SM_W0_ZERO " << (!a->row_windows_us && a->windows_us[0] == 0 ? 1 : 0) << "\n";
     s << "#define SM_G " << G << "\n#define SM_UNROLL " << unroll << "\n";
+    s << "#define SM_UPP " << (ctx->M[N - 1] / G) << "\n";   // units (config groups) per upstream prefix
     const char *ck_env = getenv("SMILESS_CHECK");     // SLA early-exit check period (steps)
     const int check = std::max(unroll, ck_env ? atoi(ck_env) : 16);
     s << "#define SM_CHECK " << check << "\n";
@@ -727,6 +759,29 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
         if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound)");
         r = driver().moduleGetFunction(&jk.fn_bound_a, jk.mod, "smiless_bound_kernel_a");
         if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound_a)");
+        r = driver().moduleGetFunction(&jk.fn_up, jk.mod, "smiless_upstream_kernel");
+        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(upstream)");
+        r = driver().moduleGetFunction(&jk.fn_var, jk.mod, "smiless_variants_kernel");
+        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(variants)");
+        {
+            const size_t padI = (size_t)((ctx->sumM + 3) & ~3), padU = (size_t)((ctx->sumM + 1) & ~1);
+            const size_t tsz = rp.time64 ? 8 : 4;
+            const size_t base = 3 * padI * 4 + padU * 8 + tsz * (size_t)n_off;
+            jk.smem_up = base + 8ull * (size_t)std::max(ctx->N - 1, 1) * kThreads +
+                         ((tsz * (size_t)ctx->N * kThreads + 15) & ~(size_t)15);
+            jk.smem_var = base + 8ull * (size_t)(a->n_windows * configs_per_lane(ctx, a)) * kThreads;
+            if (jk.smem_up <= 227 * 1024 && jk.smem_var <= 227 * 1024) {
+                r = driver().funcSetAttribute(jk.fn_up, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)jk.smem_up);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(upstream smem)");
+                r = driver().funcSetAttribute(jk.fn_var, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
+                                              (int)jk.smem_var);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(variants smem)");
+                r = driver().occupancy(&jk.blocks_up, jk.fn_up, kThreads, jk.smem_up);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(upstream)");
+                r = driver().occupancy(&jk.blocks_var, jk.fn_var, kThreads, jk.smem_var);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(variants)");
+            }
+        }
         {
             const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
             jk.smem_bound = 3 * padI * 4 + (rp.time64 ? 8 : 4) * (size_t)n_off;
@@ -842,6 +897,7 @@ void smiless_destroy(smiless_ctx *ctx) {
         ctx->dCost.release(); ctx->dLat.release(); ctx->dFeas.release(); ctx->dRes.release(); ctx->dDump.release();
         ctx->dList.release(); ctx->dListCnt.release(); ctx->dW.release();
         ctx->dListA.release(); ctx->dListCntA.release(); ctx->dChunkCnt.release();
+        ctx->dX.release(); ctx->dRecNx.release(); ctx->dRecNlu.release(); ctx->dRecPre.release();
         if (ctx->hRes) cudaFreeHost(ctx->hRes);
         for (auto &ev : ctx->ev)
             if (ev) cudaEventDestroy(ev);
@@ -1066,6 +1122,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         const u64 my_chunks = n_chunks > (u64)shard ? (n_chunks - 1 - (u64)shard) / (u64)n_shards + 1 : 0;
         const u64 claims_total = my_chunks * (u64)kChunkUnits;
         const int grid = jk->blocks_per_sm * ctx->n_sms;
+        int grid_used = grid;                        // CTAs whose argmin slots the reduce reads
         CK(ctx->dBlk.ensure((size_t)grid * 2 * n_sla), "cudaMalloc");
         CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid * 16 * n_sla, st), "memset");
         CK(cudaMemsetAsync(ctx->dStats.p, 0, 16, st), "memset");
@@ -1103,7 +1160,76 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         }
         const int D = bb_depth(ctx, a);
         pp.list_upp = 1;
-        if (D > 0 && jk->blocks_bound > 0) {
+        const char *memo_env = getenv("SMILESS_MEMO");
+        const bool memo = !pp.prune && a->n_fixed < ctx->N && (!memo_env || atoi(memo_env) != 0) &&
+                          jk->blocks_up > 0 && jk->blocks_var > 0;
+        if (memo) {
+            // ---- prefix memoisation: upstream once per prefix, then the variants per unit ---------
+            const u64 upp = (u64)(ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
+            const u64 pl0 = ub / upp, ph0 = (ue + upp - 1) / upp;
+            const size_t tsz2 = rp.time64 ? 8 : 4;
+            const size_t row_bytes = tsz2 * (size_t)n_off;
+            const u64 max_batch = std::max<u64>(1, std::min<u64>((u64)1 << 16, ((u64)4 << 30) / row_bytes));
+            const u64 batch_p = std::min<u64>(max_batch, ph0 - pl0);
+            CK(ctx->dX.ensure((size_t)batch_p * row_bytes), "cudaMalloc memo buffer");
+            CK(ctx->dRecNx.ensure((size_t)batch_p), "cudaMalloc");
+            CK(ctx->dRecNlu.ensure((size_t)batch_p), "cudaMalloc");
+            CK(ctx->dRecPre.ensure((size_t)batch_p), "cudaMalloc");
+            MemoParamsHost mp;
+            memset(&mp, 0, sizeof mp);
+            mp.tabNI = ctx->dNI.p;
+            mp.tabT = ctx->dT.p;
+            mp.tabW = ctx->dW.p;
+            mp.tabU = ctx->dU.p;
+            mp.off = ctx->dOff.p;
+            mp.scal = ctx->dScal.p;
+            mp.counter = ctx->dCounter.p;
+            mp.stats = ctx->dStats.p;
+            mp.blk_best = ctx->dBlk.p;
+            mp.xbuf = ctx->dX.p;
+            mp.rec_nx = ctx->dRecNx.p;
+            mp.rec_pre = ctx->dRecPre.p;
+            mp.rec_nlu = ctx->dRecNlu.p;
+            mp.dump = pp.dump;
+            mp.cand_begin = cb;
+            mp.cand_end = ce;
+            mp.n_steps = n_steps;
+            mp.n_off = n_off;
+            mp.sumM = ctx->sumM;
+            mp.sla = (int)a->sla_us;
+            mp.zero = 0;
+            for (int s_ = 0; s_ < n_sla; ++s_) mp.slas[s_] = (int)slas[s_];
+            for (int k = 0; k < a->n_fixed; ++k) mp.fixed[k] = a->fixed_digits[k];
+            const int grid_up = jk->blocks_up * ctx->n_sms;
+            const int grid_var = jk->blocks_var * ctx->n_sms;
+            if (grid_var > grid) {     // per-CTA argmin slots of the variants kernel
+                CK(ctx->dBlk.ensure((size_t)grid_var * 2 * n_sla), "cudaMalloc");
+                CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid_var * 16 * n_sla, st), "memset");
+                mp.blk_best = ctx->dBlk.p;
+            }
+            CK(cudaEventRecord(ctx->ev[1], st), "event");
+            u64 bi = 0;
+            for (u64 b0 = pl0; b0 < ph0; b0 += batch_p, ++bi) {
+                if (bi % (u64)n_shards != (u64)shard) continue;
+                const u64 b1 = std::min(ph0, b0 + batch_p);
+                mp.pref_begin = b0;
+                mp.pref_end = b1;
+                mp.unit_begin = std::max(ub, b0 * upp);
+                mp.unit_end = std::min(ue, b1 * upp);
+                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                void *args[] = {&mp};
+                CUresult r = driver().launchKernel(jk->fn_up, (unsigned)grid_up, 1, 1, kThreads, 1, 1,
+                                                   (unsigned)jk->smem_up, (CUstream)st, args, nullptr);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "upstream launch");
+                ++launches;
+                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                r = driver().launchKernel(jk->fn_var, (unsigned)grid_var, 1, 1, kThreads, 1, 1, (unsigned)jk->smem_var,
+                                          (CUstream)st, args, nullptr);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "variants launch");
+                ++launches;
+            }
+            grid_used = std::max(grid, grid_var);
+        } else if (D > 0 && jk->blocks_bound > 0) {
             // ---- exact branch-and-bound: prefixes of functions n_fixed..D-1, then list mode ----
             const u64 S = cands_per_prefix(ctx, a, D);
             const u64 upp = S / V;                            // evaluator units per prefix
@@ -1283,7 +1409,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         }
         CK(cudaEventRecord(ctx->ev[2], st), "event");
         for (int s_ = 0; s_ < n_sla; ++s_) {
-            e = smiless_dev_reduce_best(ctx->dBlk.p + 2 * s_, grid, n_sla, ctx->dRes.p + s_, st);
+            e = smiless_dev_reduce_best(ctx->dBlk.p + 2 * s_, grid_used, n_sla, ctx->dRes.p + s_, st);
             if (e) return cuda_fail(ctx, (cudaError_t)e, "reduce launch");
             ++launches;
         }

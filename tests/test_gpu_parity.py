@@ -620,3 +620,30 @@ def test_decompose_search_matches_oracle_steps():
         assert n_paths == onp and g.feasible == ok
         if ok:
             assert g.config.tolist() == cfg and g.cost == cost and g.max_latency_us == lat
+
+
+@pytest.mark.parametrize("memo", ["0", "1"])
+def test_throughput_mode_with_and_without_prefix_memoisation(memo, monkeypatch):
+    """Throughput mode runs the upstream once per prefix (memo = 1: upstream + variants
+    kernels) or per unit (memo = 0): per-candidate parity with the oracle either way."""
+    monkeypatch.setenv("SMILESS_MEMO", memo)
+    rng = np.random.default_rng(97)
+    n_checked = 0
+    for t in range(40):
+        n = int(rng.integers(1, 7))
+        p = W.random_problem(rng, n, 4, int(rng.integers(1, 6)), int(rng.integers(1, 200)))
+        space = p.space_size()
+        if space > 30000:
+            continue
+        flags = S.FLAG_NO_PRUNE | (S.FLAG_FORCE_INT64 if rng.random() < 0.3 else 0)
+        pl = S.planner_for(p)
+        b = int(rng.integers(0, space // 3 + 1))
+        out = np.empty(space - b)
+        g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=flags, begin=b, cost_out=out)
+        o = OracleProblem(p)
+        oc, ol, of = o.evaluate(np.arange(b, space, dtype=np.uint64))
+        assert_dump_matches(out, oc, of)
+        assert_same_plan(g, o.plan(begin=b), o)
+        assert g.n_full_evals == g.n_decided == space - b
+        n_checked += 1
+    assert n_checked > 20
