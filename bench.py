@@ -67,25 +67,26 @@ def configs_per_lane(p) -> int:
     return G
 
 
-def algorithmic_ops_per_candidate(p) -> float:
+def algorithmic_ops_per_candidate(p, memo: bool = True) -> float:
     """Integer ops per candidate over the whole horizon for the algorithm as implemented
-    (DESIGN.md "Roofline"): per invocation j >= 1 a lane-unit (one upstream prefix x G
-    configs x W windows of the last function) executes
-      7 per upstream function-step (g, u, delta, busy mask, masked update, +I, sum u),
-      +1 per extra join input, +1 per upstream sink latency check,
-      per last-function config 3 shared (x + CN, CN += -I, o + CN),
-      7 per window variant (g, u, delta, mask, update, sum u, latency) or 4 for keep-alive,
-    divided by the G*W candidates of the unit."""
+    (DESIGN.md "Roofline").  Per invocation j >= 1:
+      upstream, once per prefix (memo) or per lane-unit: 7 per function-step (g, u, delta,
+        busy mask, masked update, +I, sum u), +1 per extra join input, +1 per upstream sink;
+      per last-function config 3 shared ops (x + CN, CN += -I, o + CN);
+      per window variant 7 (g, u, delta, mask, update, sum u, latency), 4 for keep-alive;
+    divided by the candidates sharing each part (prefix: M_{N-1} x W, unit: G x W)."""
     n = p.n_funcs
     Wn = len(p.windows_us)
     G = configs_per_lane(p)
-    joins = sum(max(0, len(p.preds(k)) - 1) for k in range(n - 1))
+    joins = sum(max(0, len(p.preds(k)) - 1) for k in range(n))
     listed = set(int(v) for v in p.pred_idx)
     up_sinks = sum(1 for k in range(n - 1) if k not in listed)
     w0 = 1 if int(p.windows_us[0]) == 0 else 0
-    per_unit_step = 7 * (n - 1) + joins + max(0, len(p.preds(n - 1)) - 1) + up_sinks + \
-        G * (3 + 4 * w0 + 7 * (Wn - w0))
-    return per_unit_step * (len(p.arrivals_us) - 1) / (G * Wn)
+    upstream = 7 * (n - 1) + joins + up_sinks
+    per_unit = G * (3 + 4 * w0 + 7 * (Wn - w0))
+    up_share = int(p.n_configs[-1]) * Wn if memo else G * Wn
+    per_cand_step = upstream / up_share + per_unit / (G * Wn)
+    return per_cand_step * (len(p.arrivals_us) - 1)
 
 
 class ClockSampler:
@@ -457,7 +458,7 @@ def main():
     clocks = clk.summary()
     sm_mhz = clocks["sm_mhz"] or peaks.get("sm_max_mhz", 1965.0)
     peak_ops = props.multi_processor_count * ISSUE_LANES_PER_CLK_PER_SM * float(clocks["sm_max_mhz"] or 1965.0) * 1e6
-    ops_per_cand = algorithmic_ops_per_candidate(p)
+    ops_per_cand = algorithmic_ops_per_candidate(p, memo=os.environ.get("SMILESS_MEMO", "1") != "0")
     ops = ops_per_cand * res.n_decided
     kernel_ms_per_step = kernel_ms / args.steps
     achieved = ops / (kernel_ms_per_step / 1e3)
@@ -478,7 +479,9 @@ def main():
         "clocks": clocks,
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_ops, "unit": "int-ops/s",
                      "frac": achieved / peak_ops, "traffic": ncu_traffic(),
-                     "kernel": "smiless_plan_kernel", "kernel_ms_per_launch": kernel_ms_per_step,
+                     "kernel": ("smiless_variants_kernel + smiless_upstream_kernel (prefix memoisation)"
+                                if os.environ.get("SMILESS_MEMO", "1") != "0" else "smiless_plan_kernel"),
+                     "kernel_ms_per_launch": kernel_ms_per_step,
                      "int_ops_per_candidate": ops_per_cand, "configs_per_lane": configs_per_lane(p),
                      "peak_basis": "issue peak: SMs x 4 SMSP x 32 lanes x sm_max_mhz (DESIGN.md Roofline)"},
         "kernel_share_of_step": kernel_ms_per_step / (ms / args.steps),

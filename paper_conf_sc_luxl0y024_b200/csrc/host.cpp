@@ -224,6 +224,16 @@ int threads_per_cta() {
     return t;
 }
 #define kThreads threads_per_cta()
+// CTA size of the memoised variants kernel (fewer registers than the fused evaluator: 384
+// threads fit 168 registers per thread; SMILESS_VTHREADS tunes it)
+int vthreads_per_cta() {
+    static const int t = [] {
+        const char *e = getenv("SMILESS_VTHREADS");
+        const int v = e ? atoi(e) : 384;
+        return (v >= 64 && v <= 1024 && v % 32 == 0) ? v : 384;
+    }();
+    return t;
+}
 constexpr int kChunkUnits = 256;     // sharding / claim granularity in units (multiple of 32)
 
 struct JitKernel {
@@ -564,6 +574,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_W0_ZERO " << (!a->row_windows_us && a->windows_us[0] == 0 ? 1 : 0) << "\n";
     s << "#define SM_G " << G << "\n#define SM_UNROLL " << unroll << "\n";
     s << "#define SM_UPP " << (ctx->M[N - 1] / G) << "\n";   // units (config groups) per upstream prefix
+    s << "#define SM_VTHREADS " << vthreads_per_cta() << "\n";
     const char *ck_env = getenv("SMILESS_CHECK");     // SLA early-exit check period (steps)
     const int check = std::max(unroll, ck_env ? atoi(ck_env) : 16);
     s << "#define SM_CHECK " << check << "\n";
@@ -769,7 +780,7 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
             const size_t base = 3 * padI * 4 + padU * 8 + tsz * (size_t)n_off;
             jk.smem_up = base + 8ull * (size_t)std::max(ctx->N - 1, 1) * kThreads +
                          ((tsz * (size_t)ctx->N * kThreads + 15) & ~(size_t)15);
-            jk.smem_var = base + 8ull * (size_t)(a->n_windows * configs_per_lane(ctx, a)) * kThreads;
+            jk.smem_var = base + 8ull * (size_t)(a->n_windows * configs_per_lane(ctx, a)) * vthreads_per_cta();
             if (jk.smem_up <= 227 * 1024 && jk.smem_var <= 227 * 1024) {
                 r = driver().funcSetAttribute(jk.fn_up, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)jk.smem_up);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(upstream smem)");
@@ -778,7 +789,7 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(variants smem)");
                 r = driver().occupancy(&jk.blocks_up, jk.fn_up, kThreads, jk.smem_up);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(upstream)");
-                r = driver().occupancy(&jk.blocks_var, jk.fn_var, kThreads, jk.smem_var);
+                r = driver().occupancy(&jk.blocks_var, jk.fn_var, vthreads_per_cta(), jk.smem_var);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(variants)");
             }
         }
@@ -1223,8 +1234,8 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "upstream launch");
                 ++launches;
                 CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                r = driver().launchKernel(jk->fn_var, (unsigned)grid_var, 1, 1, kThreads, 1, 1, (unsigned)jk->smem_var,
-                                          (CUstream)st, args, nullptr);
+                r = driver().launchKernel(jk->fn_var, (unsigned)grid_var, 1, 1, vthreads_per_cta(), 1, 1,
+                                          (unsigned)jk->smem_var, (CUstream)st, args, nullptr);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "variants launch");
                 ++launches;
             }
