@@ -557,8 +557,10 @@ u64 cands_per_prefix(const smiless_ctx *ctx, const smiless_plan_args *a, int d) 
     return s;
 }
 
+enum { FAM_PLAN = 1, FAM_BOUND = 2, FAM_MEMO = 4, FAM_ALL = 7 };   // kernel families of a module
+
 std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, bool off_smem,
-                            int minb) {
+                            int minb, int families) {
     const int N = ctx->N, W = a->n_windows, NU = N - 1, nf = a->n_fixed;
     const int G = configs_per_lane(ctx, a);
     const char *un_env = getenv("SMILESS_UNROLL");
@@ -575,6 +577,8 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_G " << G << "\n#define SM_UNROLL " << unroll << "\n";
     s << "#define SM_UPP " << (ctx->M[N - 1] / G) << "\n";   // units (config groups) per upstream prefix
     s << "#define SM_VTHREADS " << vthreads_per_cta() << "\n";
+    s << "#define SM_BUILD_PLAN " << ((families & FAM_PLAN) ? 1 : 0) << "\n#define SM_BUILD_BOUND "
+      << ((families & FAM_BOUND) ? 1 : 0) << "\n#define SM_BUILD_MEMO " << ((families & FAM_MEMO) ? 1 : 0) << "\n";
     const char *ck_env = getenv("SMILESS_CHECK");     // SLA early-exit check period (steps)
     const int check = std::max(unroll, ck_env ? atoi(ck_env) : 16);
     s << "#define SM_CHECK " << check << "\n";
@@ -701,8 +705,21 @@ static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
 }
 
 std::string full_source(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, bool off_smem,
-                        int minb) {
-    return dag_spec_source(ctx, a, rp, off_smem, minb) + "\n" + smiless_evaluator_src;
+                        int minb, int families = FAM_ALL) {
+    return dag_spec_source(ctx, a, rp, off_smem, minb, families) + "\n" + smiless_evaluator_src;
+}
+
+// shared-memory bytes of the memo kernels / bound kernel (host-side, to pick a path before compiling)
+size_t smem_memo_up(const smiless_ctx *ctx, const RangePlan &rp, i64 n_off) {
+    const size_t padI = (size_t)((ctx->sumM + 3) & ~3), padU = (size_t)((ctx->sumM + 1) & ~1);
+    const size_t tsz = rp.time64 ? 8 : 4;
+    return 3 * padI * 4 + padU * 8 + tsz * (size_t)n_off + 8ull * (size_t)std::max(ctx->N - 1, 1) * kThreads +
+           ((tsz * (size_t)ctx->N * kThreads + 15) & ~(size_t)15);
+}
+size_t smem_memo_var(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off);
+size_t smem_bound_bytes(const smiless_ctx *ctx, const RangePlan &rp, i64 n_off) {
+    const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
+    return 3 * padI * 4 + (rp.time64 ? 8 : 4) * (size_t)n_off;
 }
 
 int nvrtc_compile(smiless_ctx *ctx, const std::string &src, std::vector<char> &cubin, std::string &log) {
@@ -741,13 +758,21 @@ size_t smem_bytes(const smiless_ctx *ctx, const smiless_plan_args *a, const Rang
     return b;
 }
 
-int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off, JitKernel **out) {
+size_t smem_memo_var(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off) {
+    const size_t padI = (size_t)((ctx->sumM + 3) & ~3), padU = (size_t)((ctx->sumM + 1) & ~1);
+    const size_t tsz = rp.time64 ? 8 : 4;
+    return 3 * padI * 4 + padU * 8 + tsz * (size_t)n_off +
+           8ull * (size_t)(a->n_windows * configs_per_lane(ctx, a)) * vthreads_per_cta();
+}
+
+int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off, int families,
+               JitKernel **out) {
     // offsets in shared memory when they fit next to the per-thread accumulators
     const size_t max_smem = 227 * 1024;
     bool off_smem = smem_bytes(ctx, a, rp, n_off, true) <= max_smem;
     const char *mb_env = getenv("SMILESS_MINB");     // tuning knob: min CTAs/SM for __launch_bounds__
     const int minb = mb_env ? std::max(1, atoi(mb_env)) : 1;
-    std::string src = full_source(ctx, a, rp, off_smem, minb);
+    std::string src = full_source(ctx, a, rp, off_smem, minb, families);
     auto it = ctx->jit_cache.find(src);
     if (it == ctx->jit_cache.end()) {
         std::vector<char> cubin;
@@ -757,24 +782,31 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
         JitKernel jk;
         CUresult r = driver().moduleLoadData(&jk.mod, cubin.data());
         if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleLoadData");
-        r = driver().moduleGetFunction(&jk.fn, jk.mod, "smiless_plan_kernel");
-        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction");
-        jk.smem = smem_bytes(ctx, a, rp, n_off, off_smem);
-        r = driver().funcSetAttribute(jk.fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)jk.smem);
-        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(smem)");
-        driver().funcGetAttribute(&jk.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, jk.fn);
-        r = driver().occupancy(&jk.blocks_per_sm, jk.fn, kThreads, jk.smem);
-        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuOccupancyMaxActiveBlocksPerMultiprocessor");
-        if (jk.blocks_per_sm < 1) return fail(ctx, SMILESS_ECUDA, "evaluator does not fit on an SM (smem %zu)", jk.smem);
-        r = driver().moduleGetFunction(&jk.fn_bound, jk.mod, "smiless_bound_kernel");
-        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound)");
-        r = driver().moduleGetFunction(&jk.fn_bound_a, jk.mod, "smiless_bound_kernel_a");
-        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound_a)");
-        r = driver().moduleGetFunction(&jk.fn_up, jk.mod, "smiless_upstream_kernel");
-        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(upstream)");
-        r = driver().moduleGetFunction(&jk.fn_var, jk.mod, "smiless_variants_kernel");
-        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(variants)");
-        {
+        if (families & FAM_PLAN) {
+            r = driver().moduleGetFunction(&jk.fn, jk.mod, "smiless_plan_kernel");
+            if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction");
+            jk.smem = smem_bytes(ctx, a, rp, n_off, off_smem);
+            r = driver().funcSetAttribute(jk.fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)jk.smem);
+            if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(smem)");
+            driver().funcGetAttribute(&jk.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, jk.fn);
+            r = driver().occupancy(&jk.blocks_per_sm, jk.fn, kThreads, jk.smem);
+            if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuOccupancyMaxActiveBlocksPerMultiprocessor");
+            if (jk.blocks_per_sm < 1)
+                return fail(ctx, SMILESS_ECUDA, "evaluator does not fit on an SM (smem %zu)", jk.smem);
+        }
+        if (families & FAM_BOUND) {
+            r = driver().moduleGetFunction(&jk.fn_bound, jk.mod, "smiless_bound_kernel");
+            if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound)");
+            r = driver().moduleGetFunction(&jk.fn_bound_a, jk.mod, "smiless_bound_kernel_a");
+            if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound_a)");
+        }
+        if (families & FAM_MEMO) {
+            r = driver().moduleGetFunction(&jk.fn_up, jk.mod, "smiless_upstream_kernel");
+            if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(upstream)");
+            r = driver().moduleGetFunction(&jk.fn_var, jk.mod, "smiless_variants_kernel");
+            if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(variants)");
+        }
+        if (families & FAM_MEMO) {
             const size_t padI = (size_t)((ctx->sumM + 3) & ~3), padU = (size_t)((ctx->sumM + 1) & ~1);
             const size_t tsz = rp.time64 ? 8 : 4;
             const size_t base = 3 * padI * 4 + padU * 8 + tsz * (size_t)n_off;
@@ -793,7 +825,7 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(variants)");
             }
         }
-        {
+        if (families & FAM_BOUND) {
             const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
             jk.smem_bound = 3 * padI * 4 + (rp.time64 ? 8 : 4) * (size_t)n_off;
             if (jk.smem_bound <= 227 * 1024) {
@@ -1124,8 +1156,16 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     double eval_ms = 0.0;
     u64 n_decided = 0, n_full = 0;
     if (!single && ce > cb) {
+        // pick the path first, then compile only the kernel families it needs
+        const bool prune_mode = !(a->flags & SMILESS_FLAG_NO_PRUNE);
+        const char *memo_env0 = getenv("SMILESS_MEMO");
+        const bool memo_path = !prune_mode && a->n_fixed < ctx->N && (!memo_env0 || atoi(memo_env0) != 0) &&
+                               smem_memo_up(ctx, rp, n_off) <= 227 * 1024 &&
+                               smem_memo_var(ctx, a, rp, n_off) <= 227 * 1024;
+        const bool bnb_path = !memo_path && bb_depth(ctx, a) > 0 && smem_bound_bytes(ctx, rp, n_off) <= 227 * 1024;
+        const int families = memo_path ? (FAM_MEMO | FAM_PLAN) : (bnb_path ? (FAM_PLAN | FAM_BOUND) : FAM_PLAN);
         JitKernel *jk = nullptr;
-        if ((rc = get_kernel(ctx, a, rp, n_off, &jk))) return rc;
+        if ((rc = get_kernel(ctx, a, rp, n_off, families, &jk))) return rc;
         const u64 V = (u64)a->n_windows * (u64)configs_per_lane(ctx, a);   // candidates per unit
         const u64 ub = cb / V, ue = (ce + V - 1) / V;
         const u64 U = ue - ub;
@@ -1171,9 +1211,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         }
         const int D = bb_depth(ctx, a);
         pp.list_upp = 1;
-        const char *memo_env = getenv("SMILESS_MEMO");
-        const bool memo = !pp.prune && a->n_fixed < ctx->N && (!memo_env || atoi(memo_env) != 0) &&
-                          jk->blocks_up > 0 && jk->blocks_var > 0;
+        const bool memo = memo_path && jk->blocks_up > 0 && jk->blocks_var > 0;
         if (memo) {
             // ---- prefix memoisation: upstream once per prefix, then the variants per unit ---------
             const u64 upp = (u64)(ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
@@ -1240,7 +1278,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 ++launches;
             }
             grid_used = std::max(grid, grid_var);
-        } else if (D > 0 && jk->blocks_bound > 0) {
+        } else if (bnb_path && D > 0 && jk->blocks_bound > 0) {
             // ---- exact branch-and-bound: prefixes of functions n_fixed..D-1, then list mode ----
             const u64 S = cands_per_prefix(ctx, a, D);
             const u64 upp = S / V;                            // evaluator units per prefix
