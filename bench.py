@@ -219,9 +219,16 @@ def measured_peaks():
         return {}
 
 
-def ncu_traffic():
-    """DRAM bytes per launch of the evaluator from the committed ncu --set full summary."""
+def ncu_traffic(memo: bool, plan_launches: int):
+    """DRAM bytes of the timed kernels per plan call (the unit `achieved` uses), from the
+    committed ncu --set full summaries.  Memo path: one plan call = prep + B x (upstream,
+    variants) + reduce + exact, so B = (launches - 3) / 2 pairs, each pair moving the
+    upstream kernel's x-buffer write and the variants kernel's read of it."""
     try:
+        if memo:
+            d = json.load(open(os.path.join(ROOT, "profiles", "ncu_memo_summary.json")))
+            pair = sum(k["dram_bytes_per_launch"] for k in d["launches"])
+            return pair * max(1, (plan_launches - 3) // 2)
         d = json.load(open(os.path.join(ROOT, "profiles", "ncu_evaluator_summary.json")))
         return d.get("dram_bytes_per_launch")
     except Exception:
@@ -458,7 +465,8 @@ def main():
     clocks = clk.summary()
     sm_mhz = clocks["sm_mhz"] or peaks.get("sm_max_mhz", 1965.0)
     peak_ops = props.multi_processor_count * ISSUE_LANES_PER_CLK_PER_SM * float(clocks["sm_max_mhz"] or 1965.0) * 1e6
-    ops_per_cand = algorithmic_ops_per_candidate(p, memo=os.environ.get("SMILESS_MEMO", "1") != "0")
+    memo = os.environ.get("SMILESS_MEMO", "1") != "0"
+    ops_per_cand = algorithmic_ops_per_candidate(p, memo=memo)
     ops = ops_per_cand * res.n_decided
     kernel_ms_per_step = kernel_ms / args.steps
     achieved = ops / (kernel_ms_per_step / 1e3)
@@ -478,9 +486,10 @@ def main():
                 "d2h_bytes_per_step": 312},
         "clocks": clocks,
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_ops, "unit": "int-ops/s",
-                     "frac": achieved / peak_ops, "traffic": ncu_traffic(),
+                     "frac": achieved / peak_ops, "traffic": ncu_traffic(memo, res.launches),
+                     "traffic_basis": "ncu dram__bytes_read+write per plan call (profiles/ncu_memo_summary.json)",
                      "kernel": ("smiless_variants_kernel + smiless_upstream_kernel (prefix memoisation)"
-                                if os.environ.get("SMILESS_MEMO", "1") != "0" else "smiless_plan_kernel"),
+                                if memo else "smiless_plan_kernel"),
                      "kernel_ms_per_launch": kernel_ms_per_step,
                      "int_ops_per_candidate": ops_per_cand, "configs_per_lane": configs_per_lane(p),
                      "peak_basis": "issue peak: SMs x 4 SMSP x 32 lanes x sm_max_mhz (DESIGN.md Roofline)"},

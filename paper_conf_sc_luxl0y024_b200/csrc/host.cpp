@@ -224,15 +224,23 @@ int threads_per_cta() {
     return t;
 }
 #define kThreads threads_per_cta()
-// CTA size of the memoised variants kernel (fewer registers than the fused evaluator: 384
-// threads fit 168 registers per thread; SMILESS_VTHREADS tunes it)
+// CTA size and min CTAs/SM of the memoised variants kernel.  2 x 256 threads (128 registers)
+// measured best on C2 (profiles/r01f_sweep_variants.md; SMILESS_VTHREADS / SMILESS_VMINB tune it)
 int vthreads_per_cta() {
     static const int t = [] {
         const char *e = getenv("SMILESS_VTHREADS");
-        const int v = e ? atoi(e) : 384;
-        return (v >= 64 && v <= 1024 && v % 32 == 0) ? v : 384;
+        const int v = e ? atoi(e) : 256;
+        return (v >= 64 && v <= 1024 && v % 32 == 0) ? v : 256;
     }();
     return t;
+}
+int vmin_blocks() {
+    static const int b = [] {
+        const char *e = getenv("SMILESS_VMINB");
+        const int v = e ? atoi(e) : 2;
+        return (v >= 1 && v <= 8) ? v : 2;
+    }();
+    return b;
 }
 constexpr int kChunkUnits = 256;     // sharding / claim granularity in units (multiple of 32)
 
@@ -307,7 +315,7 @@ struct smiless_ctx {
     DevBuf<u64> dList, dListA;
     DevBuf<unsigned> dListCnt, dListCntA, dChunkCnt;
     DevBuf<int> dW;                          // per-row windows of the current plan (padded)
-    DevBuf<unsigned char> dX;                // memoised last-function inputs [prefix][n_off]
+    DevBuf<unsigned char> dX;                // memoised last-function inputs [n_off/4][prefix][4]
     DevBuf<i64> dRecNx, dRecNlu;             // per-prefix records (int32 or int64 time)
     DevBuf<double> dRecPre;
     std::vector<int> hW;                     // host copy of what dW holds
@@ -576,7 +584,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_W0_ZERO " << (!a->row_windows_us && a->windows_us[0] == 0 ? 1 : 0) << "\n";
     s << "#define SM_G " << G << "\n#define SM_UNROLL " << unroll << "\n";
     s << "#define SM_UPP " << (ctx->M[N - 1] / G) << "\n";   // units (config groups) per upstream prefix
-    s << "#define SM_VTHREADS " << vthreads_per_cta() << "\n";
+    s << "#define SM_VTHREADS " << vthreads_per_cta() << "\n#define SM_VMINB " << vmin_blocks() << "\n";
     s << "#define SM_BUILD_PLAN " << ((families & FAM_PLAN) ? 1 : 0) << "\n#define SM_BUILD_BOUND "
       << ((families & FAM_BOUND) ? 1 : 0) << "\n#define SM_BUILD_MEMO " << ((families & FAM_MEMO) ? 1 : 0) << "\n";
     const char *ck_env = getenv("SMILESS_CHECK");     // SLA early-exit check period (steps)
@@ -590,6 +598,9 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_ROWWIN " << (a->row_windows_us ? 1 : 0) << "\n";
     const char *mask_env = getenv("SMILESS_MASK");   // tuning knob, see evaluator.cuh SM_MASK
     s << "#define SM_MASK " << (mask_env ? atoi(mask_env) : 0) << "\n";
+    // tuning knob, see evaluator.cuh SM_SELMASK; default: window variants 1 and 2 use select
+    const char *sel_env = getenv("SMILESS_SELMASK");
+    s << "#define SM_SELMASK " << (sel_env ? atoi(sel_env) : 6) << "\n";
     // compile-time window grid (immediates) and a constant-bank copy for runtime indices
     s << "#define SM_WIN(v) (";
     for (int v = 0; v < W; ++v) s << "(v)==" << v << "?" << a->windows_us[v] << ":";
@@ -765,14 +776,18 @@ size_t smem_memo_var(const smiless_ctx *ctx, const smiless_plan_args *a, const R
            8ull * (size_t)(a->n_windows * configs_per_lane(ctx, a)) * vthreads_per_cta();
 }
 
+// tuning knob: min CTAs/SM for __launch_bounds__ of the evaluator / variants kernels
+int min_blocks() {
+    const char *mb_env = getenv("SMILESS_MINB");
+    return mb_env ? std::max(1, atoi(mb_env)) : 1;
+}
+
 int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off, int families,
                JitKernel **out) {
     // offsets in shared memory when they fit next to the per-thread accumulators
     const size_t max_smem = 227 * 1024;
     bool off_smem = smem_bytes(ctx, a, rp, n_off, true) <= max_smem;
-    const char *mb_env = getenv("SMILESS_MINB");     // tuning knob: min CTAs/SM for __launch_bounds__
-    const int minb = mb_env ? std::max(1, atoi(mb_env)) : 1;
-    std::string src = full_source(ctx, a, rp, off_smem, minb, families);
+    std::string src = full_source(ctx, a, rp, off_smem, min_blocks(), families);
     auto it = ctx->jit_cache.find(src);
     if (it == ctx->jit_cache.end()) {
         std::vector<char> cubin;
@@ -1878,7 +1893,7 @@ int smiless_jit_compile(smiless_ctx *ctx, const smiless_plan_args *a, char *log,
     const bool off_smem = smem_bytes(ctx, a, rp, n_off, true) <= 227 * 1024;
     std::vector<char> cubin;
     std::string lg;
-    rc = nvrtc_compile(ctx, full_source(ctx, a, rp, off_smem, 1), cubin, lg);
+    rc = nvrtc_compile(ctx, full_source(ctx, a, rp, off_smem, min_blocks()), cubin, lg);
     if (log && logcap) {
         const size_t n = std::min(logcap - 1, lg.size());
         memcpy(log, lg.data(), n);

@@ -653,3 +653,30 @@ def test_throughput_mode_with_and_without_prefix_memoisation(memo, monkeypatch):
         assert g.n_full_evals == g.n_decided == space - b
         n_checked += 1
     assert n_checked > 20
+
+
+@pytest.mark.parametrize("g,selmask", [("1", "0"), ("1", "2"), ("2", "255"), ("4", "6")])
+def test_memo_variants_shapes_are_exact(g, selmask, monkeypatch):
+    """The variants kernel's tuning knobs (configs per lane G, select vs IMAD.HI busy mask
+    per window variant) change only the instruction mix: per-candidate parity with the
+    oracle for each."""
+    monkeypatch.setenv("SMILESS_MEMO", "1")
+    monkeypatch.setenv("SMILESS_G", g)
+    monkeypatch.setenv("SMILESS_SELMASK", selmask)
+    rng = np.random.default_rng(131 + int(g) * 7 + int(selmask))
+    n_checked = 0
+    for t in range(30):
+        n = int(rng.integers(2, 6))
+        p = W.random_problem(rng, n, 4, int(rng.integers(2, 5)), int(rng.integers(2, 300)))
+        space = p.space_size()
+        if space > 30000:
+            continue
+        pl = S.planner_for(p)
+        out = np.empty(space)
+        g_ = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=S.FLAG_NO_PRUNE, cost_out=out)
+        o = OracleProblem(p)
+        oc, ol, of = o.evaluate(np.arange(0, space, dtype=np.uint64))
+        assert_dump_matches(out, oc, of)
+        assert_same_plan(g_, o.plan(), o)
+        n_checked += 1
+    assert n_checked > 10
