@@ -234,6 +234,12 @@ int vthreads_per_cta() {
     }();
     return t;
 }
+// L2 prefetch distance (4-step groups) of the variants kernel's x stream (SMILESS_XPF tunes it)
+int xpf_groups() {
+    const char *e = getenv("SMILESS_XPF");
+    return e ? std::min(64, std::max(1, atoi(e))) : 8;
+}
+
 int vmin_blocks() {
     static const int b = [] {
         const char *e = getenv("SMILESS_VMINB");
@@ -598,6 +604,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_ROWWIN " << (a->row_windows_us ? 1 : 0) << "\n";
     const char *mask_env = getenv("SMILESS_MASK");   // tuning knob, see evaluator.cuh SM_MASK
     s << "#define SM_MASK " << (mask_env ? atoi(mask_env) : 0) << "\n";
+    s << "#define SM_XPF " << xpf_groups() << "\n";
     // tuning knob, see evaluator.cuh SM_SELMASK; default: window variants 1 and 2 use select
     const char *sel_env = getenv("SMILESS_SELMASK");
     s << "#define SM_SELMASK " << (sel_env ? atoi(sel_env) : 6) << "\n";
@@ -1232,7 +1239,8 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             const u64 upp = (u64)(ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
             const u64 pl0 = ub / upp, ph0 = (ue + upp - 1) / upp;
             const size_t tsz2 = rp.time64 ? 8 : 4;
-            const size_t row_bytes = tsz2 * (size_t)n_off;
+            // + SM_XPF + 1 groups of 4 steps of read-ahead slack for the variants kernel
+            const size_t row_bytes = tsz2 * (size_t)(n_off + 4 * (xpf_groups() + 1));
             const u64 max_batch = std::max<u64>(1, std::min<u64>((u64)1 << 16, ((u64)4 << 30) / row_bytes));
             const u64 batch_p = std::min<u64>(max_batch, ph0 - pl0);
             CK(ctx->dX.ensure((size_t)batch_p * row_bytes), "cudaMalloc memo buffer");
