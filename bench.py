@@ -170,7 +170,11 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
         if pinned:
             if i % world != rank:
                 continue
-            r = pl.plan(arr, p.sla_us, p.windows_us, n_fixed=1, fixed_digits=[d0])
+            # the cheapest feasible cost found so far caps the next sub-plan: its cost bound then
+            # prunes from the first launch (a cap >= OPT keeps the result exact; ties resolve on
+            # (cost, digit, index) below)
+            cap = {"cost_cap": best[0]} if best is not None else {}
+            r = pl.plan(arr, p.sla_us, p.windows_us, n_fixed=1, fixed_digits=[d0], **cap)
         else:
             r = pl.plan(arr, p.sla_us, p.windows_us, shard=rank, n_shards=world)
         decided += r.n_decided

@@ -71,7 +71,9 @@ enum {
 enum {
     SMILESS_FLAG_NO_PRUNE = 1u,            /* throughput mode: walk every candidate to j = J-1 */
     SMILESS_FLAG_ARRIVALS_ON_DEVICE = 2u,  /* arrivals_us is a device pointer (HBM-resident)   */
-    SMILESS_FLAG_FORCE_INT64 = 4u          /* use the int64 evaluator even if int32 is exact   */
+    SMILESS_FLAG_FORCE_INT64 = 4u,         /* use the int64 evaluator even if int32 is exact   */
+    SMILESS_FLAG_COST_CAP = 8u             /* only candidates with cost <= cost_cap are eligible
+                                              (prune mode, smiless_plan only)                  */
 };
 
 #define SMILESS_MAX_FUNCS 32
@@ -137,6 +139,13 @@ typedef struct {
                                      paper's adaptive pre-warming; see
                                      smiless_derive_windows); requires n_windows == 1 (windows_us
                                      is then ignored); 0 <= w < 2^29                               */
+    double cost_cap;              /* with SMILESS_FLAG_COST_CAP: the plan is the argmin over the
+                                     feasible candidates whose cost is <= cost_cap (INFEASIBLE if
+                                     none), so a cap >= OPT returns OPT exactly.  Passing the cost of
+                                     a plan known to be feasible (a heuristic's, the previous
+                                     re-plan's) lets the evaluator's cost bound prune from the first
+                                     launch (DESIGN.md section 5 item 11).  cost_cap >= 0, not NaN;
+                                     EINVAL with SMILESS_FLAG_NO_PRUNE or in smiless_plan_sla_sweep */
 } smiless_plan_args;
 
 typedef struct {

@@ -159,6 +159,11 @@ struct PlanParamsHost {
     i64 horizon;
     int slas[8];
     const int *tabW;               // [sumM] per-row windows (SM_ROWWIN) or a dummy table
+    u64 *inc;                      // incumbent cost bits (cost-bound pruning)
+    const i64 *rrem;               // [chunks] r_{J-1} - r_{(q+1)K}
+    u64 cap;                       // cost cap bits (~0: none)
+    int cost_prune;
+    int pad0;
     int fixed[SMILESS_MAX_FUNCS];  // evaluator uses SM_NFIXED_ALLOC <= SMILESS_MAX_FUNCS; extra tail is ignored
 };
 
@@ -211,6 +216,11 @@ struct BoundParamsHost {
     u64 list_upp;
     int nimin[SMILESS_MAX_FUNCS];
     const int *tabW;
+    const double *tabU;
+    const i64 *scal;
+    u64 *inc;                      // incumbent cost bits shared with the evaluator
+    int cost_prune;
+    int pad0;
     int fixed[SMILESS_MAX_FUNCS];
 };
 
@@ -312,8 +322,9 @@ struct smiless_ctx {
     DevBuf<i64> dArr;
     DevBuf<unsigned char> dOff;
     DevBuf<i64> dScal;
+    DevBuf<i64> dRrem;                       // real time left after each chunk (cost bound)
     DevBuf<int> dErr;
-    DevBuf<u64> dCounter, dStats, dBlk, dIdxEval;
+    DevBuf<u64> dCounter, dStats, dBlk, dIdxEval, dInc;
     DevBuf<double> dCost;
     DevBuf<i64> dLat;
     DevBuf<unsigned char> dFeas;
@@ -385,6 +396,7 @@ int ensure_device(smiless_ctx *ctx) {
     CK(ctx->dErr.ensure(1), "cudaMalloc");
     CK(ctx->dCounter.ensure(1), "cudaMalloc");
     CK(ctx->dStats.ensure(2), "cudaMalloc");
+    CK(ctx->dInc.ensure(1), "cudaMalloc");
     ctx->dev_ready = true;
     return SMILESS_OK;
 }
@@ -472,6 +484,10 @@ int validate_args(smiless_ctx *ctx, const smiless_plan_args *a, bool need_arriva
         return fail(ctx, SMILESS_ERANGE, "candidate space exceeds 2^63-1; pin leading digits with n_fixed");
     if (a->n_shards < 0 || (a->n_shards > 0 && (a->shard < 0 || a->shard >= a->n_shards)))
         return fail(ctx, SMILESS_EINVAL, "bad shard/n_shards");
+    if (a->flags & SMILESS_FLAG_COST_CAP) {
+        if (!(a->cost_cap >= 0.0)) return fail(ctx, SMILESS_EINVAL, "cost_cap must be >= 0 (not NaN)");
+        if (a->flags & SMILESS_FLAG_NO_PRUNE) return fail(ctx, SMILESS_EINVAL, "FLAG_COST_CAP requires prune mode");
+    }
     return SMILESS_OK;
 }
 
@@ -573,6 +589,9 @@ u64 cands_per_prefix(const smiless_ctx *ctx, const smiless_plan_args *a, int d) 
 
 enum { FAM_PLAN = 1, FAM_BOUND = 2, FAM_MEMO = 4, FAM_ALL = 7 };   // kernel families of a module
 
+// static cost-bound terms of every (row, window) staged in shared memory when small
+bool bound_lb_table(const smiless_ctx *ctx, int W) { return (size_t)ctx->sumM * (size_t)W <= 8192; }
+
 std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, bool off_smem,
                             int minb, int families) {
     const int N = ctx->N, W = a->n_windows, NU = N - 1, nf = a->n_fixed;
@@ -602,6 +621,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
       << "\n#define SMILESS_MAXF " << SMILESS_MAX_FUNCS << "\n";
     s << "#define SM_NSLA " << ctx->nsla << "\n";
     s << "#define SM_ROWWIN " << (a->row_windows_us ? 1 : 0) << "\n";
+    s << "#define SM_LBT " << (bound_lb_table(ctx, W) ? 1 : 0) << "\n";
     const char *mask_env = getenv("SMILESS_MASK");   // tuning knob, see evaluator.cuh SM_MASK
     s << "#define SM_MASK " << (mask_env ? atoi(mask_env) : 0) << "\n";
     s << "#define SM_XPF " << xpf_groups() << "\n";
@@ -617,6 +637,9 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "};\n#define SM_WINV(i) c_win[(i)]\n";
     s << "#define SM_ROW0(k) (";
     for (int k = 0; k < N; ++k) s << "(k)==" << k << "?" << ctx->row0[k] << ":";
+    s << "0)\n";
+    s << "#define SM_MK(k) (";
+    for (int k = 0; k < N; ++k) s << "(k)==" << k << "?" << ctx->M[k] << ":";
     s << "0)\n";
     s << R"(
 typedef long long i64;
@@ -735,9 +758,10 @@ size_t smem_memo_up(const smiless_ctx *ctx, const RangePlan &rp, i64 n_off) {
            ((tsz * (size_t)ctx->N * kThreads + 15) & ~(size_t)15);
 }
 size_t smem_memo_var(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off);
-size_t smem_bound_bytes(const smiless_ctx *ctx, const RangePlan &rp, i64 n_off) {
+size_t smem_bound_bytes(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off) {
     const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
-    return 3 * padI * 4 + (rp.time64 ? 8 : 4) * (size_t)n_off;
+    const size_t lbt = bound_lb_table(ctx, a->n_windows) ? 8 * (size_t)((ctx->sumM * a->n_windows + 1) & ~1) : 0;
+    return 3 * padI * 4 + 8 * (size_t)((ctx->sumM + 1) & ~1) + lbt + (rp.time64 ? 8 : 4) * (size_t)n_off;
 }
 
 int nvrtc_compile(smiless_ctx *ctx, const std::string &src, std::vector<char> &cubin, std::string &log) {
@@ -848,8 +872,7 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
             }
         }
         if (families & FAM_BOUND) {
-            const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
-            jk.smem_bound = 3 * padI * 4 + (rp.time64 ? 8 : 4) * (size_t)n_off;
+            jk.smem_bound = smem_bound_bytes(ctx, a, rp, n_off);
             if (jk.smem_bound <= 227 * 1024) {
                 r = driver().funcSetAttribute(jk.fn_bound, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
                                               (int)jk.smem_bound);
@@ -957,8 +980,8 @@ void smiless_destroy(smiless_ctx *ctx) {
         for (auto &kv : ctx->jit_cache)
             if (kv.second.mod) driver().moduleUnload(kv.second.mod);
         ctx->dI.release(); ctx->dNI.release(); ctx->dT.release(); ctx->dU.release(); ctx->dPtr.release(); ctx->dIdx.release();
-        ctx->dArr.release(); ctx->dOff.release(); ctx->dScal.release(); ctx->dErr.release();
-        ctx->dCounter.release(); ctx->dStats.release(); ctx->dBlk.release(); ctx->dIdxEval.release();
+        ctx->dArr.release(); ctx->dOff.release(); ctx->dScal.release(); ctx->dRrem.release(); ctx->dErr.release();
+        ctx->dCounter.release(); ctx->dStats.release(); ctx->dInc.release(); ctx->dBlk.release(); ctx->dIdxEval.release();
         ctx->dCost.release(); ctx->dLat.release(); ctx->dFeas.release(); ctx->dRes.release(); ctx->dDump.release();
         ctx->dList.release(); ctx->dListCnt.release(); ctx->dW.release();
         ctx->dListA.release(); ctx->dListCntA.release(); ctx->dChunkCnt.release();
@@ -1141,6 +1164,8 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     if (rc) return rc;
     for (int s_ = 0; s_ < n_sla; ++s_)
         if (slas[s_] < 0 || slas[s_] >= (1ll << 29)) return fail(ctx, SMILESS_EINVAL, "sla out of [0, 2^29)");
+    if (n_sla > 1 && (a->flags & SMILESS_FLAG_COST_CAP))
+        return fail(ctx, SMILESS_EINVAL, "FLAG_COST_CAP is not supported by the SLA sweep");
     ctx->nsla = n_sla;
     struct NslaReset { smiless_ctx *c; ~NslaReset() { c->nsla = 1; } } nsla_reset{ctx};
     u64 space;
@@ -1169,8 +1194,9 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     CK(ctx->dOff.ensure((size_t)n_off * tsz), "cudaMalloc offsets");
     CK(cudaMemsetAsync(ctx->dErr.p, 0, sizeof(int), st), "memset");
     CK(cudaMemsetAsync(ctx->dRes.p, 0xff, sizeof(ResBlock) * n_sla, st), "memset");
+    CK(ctx->dRrem.ensure((size_t)(n_off / rp.K + 1)), "cudaMalloc rrem");
     int e = smiless_dev_prep_offsets(d_arr, a->n_arrivals, rp.d_cap, rp.K, rp.time64 ? 1 : 0, ctx->dOff.p, n_off,
-                                     ctx->dScal.p, ctx->dErr.p, st);
+                                     ctx->dScal.p, ctx->dErr.p, ctx->dRrem.p, st);
     if (e) return cuda_fail(ctx, (cudaError_t)e, "prep_offsets launch");
     ++launches;
 
@@ -1184,7 +1210,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         const bool memo_path = !prune_mode && a->n_fixed < ctx->N && (!memo_env0 || atoi(memo_env0) != 0) &&
                                smem_memo_up(ctx, rp, n_off) <= 227 * 1024 &&
                                smem_memo_var(ctx, a, rp, n_off) <= 227 * 1024;
-        const bool bnb_path = !memo_path && bb_depth(ctx, a) > 0 && smem_bound_bytes(ctx, rp, n_off) <= 227 * 1024;
+        const bool bnb_path = !memo_path && bb_depth(ctx, a) > 0 && smem_bound_bytes(ctx, a, rp, n_off) <= 227 * 1024;
         const int families = memo_path ? (FAM_MEMO | FAM_PLAN) : (bnb_path ? (FAM_PLAN | FAM_BOUND) : FAM_PLAN);
         JitKernel *jk = nullptr;
         if ((rc = get_kernel(ctx, a, rp, n_off, families, &jk))) return rc;
@@ -1222,6 +1248,20 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         pp.sla = (int)a->sla_us;
         for (int s_ = 0; s_ < n_sla; ++s_) pp.slas[s_] = (int)slas[s_];
         pp.prune = (a->flags & SMILESS_FLAG_NO_PRUNE) ? 0 : 1;
+        // cost-bound pruning against a running incumbent (one SLA, no per-candidate dump);
+        // SMILESS_COST_PRUNE=0 disables it
+        {
+            const char *cp_env = getenv("SMILESS_COST_PRUNE");
+            pp.cost_prune = (pp.prune && n_sla == 1 && !a->cost_out && (!cp_env || atoi(cp_env) != 0)) ? 1 : 0;
+            pp.inc = ctx->dInc.p;
+            pp.rrem = ctx->dRrem.p;
+            pp.cap = ~0ull;
+            if (a->flags & SMILESS_FLAG_COST_CAP) {
+                double c = a->cost_cap + 0.0;               // -0.0 -> +0.0: bits order like the costs
+                memcpy(&pp.cap, &c, 8);
+            }
+            CK(cudaMemcpyAsync(ctx->dInc.p, &pp.cap, 8, cudaMemcpyHostToDevice, st), "H2D incumbent");
+        }
         pp.shard = shard;
         pp.n_shards = n_shards;
         pp.chunk_units = kChunkUnits;
@@ -1314,6 +1354,10 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             bp.tabNI = ctx->dNI.p;
             bp.tabW = ctx->dW.p;
             bp.tabT = ctx->dT.p;
+            bp.tabU = ctx->dU.p;
+            bp.scal = ctx->dScal.p;
+            bp.inc = ctx->dInc.p;
+            bp.cost_prune = pp.cost_prune;
             bp.off = ctx->dOff.p;
             bp.counter = ctx->dCounter.p;
             bp.stats = ctx->dStats.p;
@@ -1531,7 +1575,8 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     int status = SMILESS_INFEASIBLE;
     for (int s_ = 0; s_ < n_sla; ++s_) {
         const ResBlock &h = ctx->hRes[s_];
-        const bool found = h.best_i != ~0ull && h.feasible == 1;
+        const bool found = h.best_i != ~0ull && h.feasible == 1 &&
+                           !((a->flags & SMILESS_FLAG_COST_CAP) && !(h.cost <= a->cost_cap + 0.0));
         if (!single && h.best_i != ~0ull && h.feasible != 1)
             return fail(ctx, SMILESS_ECUDA, "internal: evaluator winner %llu not feasible on exact re-evaluation",
                         (unsigned long long)h.best_i);

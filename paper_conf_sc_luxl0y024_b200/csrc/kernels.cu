@@ -19,13 +19,16 @@ namespace smiless_dev {
 // One thread per chunk of K steps; step s (0-based) is arrival j = s + 1.
 // off[s] = sum_{i = chunk start}^{s} min(r_{i+1} - r_i, d_cap), i.e. the clamped arrival
 // time of j = s + 1 relative to the chunk base (the arrival just before the chunk).
+// rrem[q] = r_{J-1} - r_{(q+1)K}: the real (unclamped) time left after chunk q, used by the
+// evaluator's cost bound (0 past the last full chunk).
 template <typename T>
 __global__ void prep_offsets_kernel(const i64 *__restrict__ arr, i64 J, i64 d_cap, int K, T *__restrict__ off,
-                                    i64 n_off, i64 *__restrict__ scal, int *__restrict__ err) {
+                                    i64 n_off, i64 *__restrict__ scal, int *__restrict__ err, i64 *__restrict__ rrem) {
     const i64 n_steps = J - 1;
     const i64 q = (i64)blockIdx.x * blockDim.x + threadIdx.x;
     const i64 s0 = q * K;
     if (s0 >= n_off) return;
+    rrem[q] = (q + 1) * K <= n_steps ? arr[J - 1] - arr[(q + 1) * K] : 0;
     i64 acc = 0;
     const i64 LIM = (i64)1 << 62;
     for (i64 s = s0; s < s0 + K && s < n_off; ++s) {
@@ -76,87 +79,128 @@ __global__ void reduce_best_kernel(const u64 *__restrict__ slots, int n, int str
     }
 }
 
-// Exact evaluation, absolute int64 times, generic DAG (runtime CSR in device memory).
+// Exact evaluation, absolute int64 times, generic DAG (runtime CSR in device memory), the
+// plain case split of model M with per-step billing -- independent of the
+// NVRTC evaluator's reformulations.  One WARP per candidate, lane k = function k: within an
+// invocation the functions run level by level of the DAG (a function's level = 1 + the
+// highest level of its predecessors), a predecessor's done time comes over a shuffle, so an
+// invocation costs (levels x max in-degree) shuffles instead of N dependent local-memory
+// walks.  Arrivals are read 32 at a time (one coalesced load) and broadcast by shuffle.
+__device__ __forceinline__ long long shfl64(long long v, int src) {
+    return (long long)__shfl_sync(0xffffffffu, (unsigned long long)v, src);
+}
+
 __global__ void eval_exact_kernel(ExactParams p) {
-    const i64 t = (i64)blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= p.n) return;
+    const unsigned FULL = 0xffffffffu;
+    const int lane = threadIdx.x & 31;
+    const i64 t = ((i64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;   // candidate of this warp
+    if (t >= p.n) return;                                                // warp-uniform
     ResBlock *res = p.idx_from_res ? p.res + t : nullptr;
     const i64 sla = p.idx_from_res ? p.slas[t] : p.sla;
-    u64 index = p.idx_from_res ? res->best_i : p.idx[t];
+    const u64 index = p.idx_from_res ? res->best_i : p.idx[t];
     if (index == ~0ull) {
-        if (res) { res->feasible = 0; res->cost = 0.0; res->maxlat = -1; }
+        if (res && lane == 0) { res->feasible = 0; res->cost = 0.0; res->maxlat = -1; }
         return;
     }
     const int N = p.N, W = p.W;
-    int cfg[SMILESS_DEV_MAX_FUNCS], win[SMILESS_DEV_MAX_FUNCS];
-    for (int k = N - 1; k >= p.n_fixed; --k) {
-        const u64 radix = (u64)p.M[k] * (u64)W;
-        const u64 d = index % radix;
-        index /= radix;
-        cfg[k] = (int)(d / (u64)W);
-        win[k] = (int)(d % (u64)W);
+    const bool act = lane < N;
+    const int k = act ? lane : 0;
+    // ---- decode this lane's digit: index = sum_k d_k S_k over functions n_fixed..N-1 --------
+    int cfg = 0, win = 0;
+    if (lane < p.n_fixed) {
+        cfg = p.fixed[lane] / W;
+        win = p.fixed[lane] % W;
+    } else if (act) {
+        u64 stride = 1;
+        for (int q = N - 1; q > k; --q) stride *= (u64)p.M[q] * (u64)W;
+        const u64 d = (index / stride) % ((u64)p.M[k] * (u64)W);
+        cfg = (int)(d / (u64)W);
+        win = (int)(d % (u64)W);
     }
-    for (int k = 0; k < p.n_fixed; ++k) {
-        cfg[k] = p.fixed[k] / W;
-        win[k] = p.fixed[k] % W;
+    const int row = p.row0[k] + cfg;
+    const i64 I = act ? p.tabI[row] : 0, T = act ? p.tabT[row] : 0;
+    const i64 w = act ? (p.rowwin ? p.rowwin[row] : p.win[win]) : 0;
+    const int e0 = act ? p.pred_ptr[k] : 0, deg = act ? p.pred_ptr[k + 1] - e0 : 0;
+    const bool sink = act && ((p.sinkmask >> k) & 1u);
+    int pc[4];                                            // first predecessors in registers
+#pragma unroll
+    for (int e = 0; e < 4; ++e) pc[e] = e < deg ? p.pred_idx[e0 + e] : lane;
+    int maxdeg = deg;
+#pragma unroll
+    for (int m = 16; m > 0; m >>= 1) maxdeg = max(maxdeg, __shfl_xor_sync(FULL, maxdeg, m));
+    // ---- topological levels (Bellman-Ford over the warp, N passes at most) -----------------
+    int lvl = act ? 0 : -1;
+    for (int pass = 0; pass < N; ++pass) {
+        int l2 = act ? 0 : -1;
+        for (int e = 0; e < maxdeg; ++e) {
+            const int src = e < deg ? (e < 4 ? pc[e] : p.pred_idx[e0 + e]) : lane;
+            const int lp = __shfl_sync(FULL, lvl, src);
+            if (e < deg) l2 = max(l2, lp + 1);
+        }
+        lvl = l2;
     }
-    i64 I[SMILESS_DEV_MAX_FUNCS], T[SMILESS_DEV_MAX_FUNCS], w[SMILESS_DEV_MAX_FUNCS];
-    i64 D[SMILESS_DEV_MAX_FUNCS], billed[SMILESS_DEV_MAX_FUNCS];
-    for (int k = 0; k < N; ++k) {
-        const int row = p.row0[k] + cfg[k];
-        I[k] = p.tabI[row];
-        T[k] = p.tabT[row];
-        w[k] = p.rowwin ? p.rowwin[row] : p.win[win[k]];
-        billed[k] = 0;
-        D[k] = 0;
-    }
-    i64 maxlat = INT64_MIN;
-    for (i64 j = 0; j < p.J; ++j) {
-        const i64 r = p.arr[j];
-        i64 lat = INT64_MIN;
-        for (int k = 0; k < N; ++k) {
-            i64 x;
-            const int e0 = p.pred_ptr[k], e1 = p.pred_ptr[k + 1];
-            if (e0 == e1) {
-                x = r;
-            } else {
-                x = D[p.pred_idx[e0]];
-                for (int e = e0 + 1; e < e1; ++e) x = max(x, D[p.pred_idx[e]]);
-            }
-            i64 start, bill;
-            if (j == 0) {
-                start = x;
-                bill = T[k];
-            } else {
-                const i64 f = D[k], g = x - f;
-                if (g <= 0) {
-                    start = f;
-                    bill = 0;
-                } else {
-                    const i64 te = w[k] == 0 ? 0 : T[k];
-                    const i64 u = min(g, w[k]);
-                    start = f + max(u + te, g);
-                    bill = max(te, g - w[k]);
+    int nlev = lvl + 1;
+#pragma unroll
+    for (int m = 16; m > 0; m >>= 1) nlev = max(nlev, __shfl_xor_sync(FULL, nlev, m));
+
+    i64 D = 0, billed = 0, maxlat = INT64_MIN;
+    for (i64 j0 = 0; j0 < p.J; j0 += 32) {
+        const i64 rb = j0 + lane < p.J ? p.arr[j0 + lane] : 0;
+        const int jn = (int)min((i64)32, p.J - j0);
+        for (int jj = 0; jj < jn; ++jj) {
+            const i64 r = shfl64(rb, jj);
+            for (int l = 0; l < nlev; ++l) {
+                i64 x = r;                                // sources: the request's arrival
+                for (int e = 0; e < maxdeg; ++e) {        // AND-join: max over predecessors
+                    const int src = e < deg ? (e < 4 ? pc[e] : p.pred_idx[e0 + e]) : lane;
+                    const i64 d = shfl64(D, src);
+                    if (e < deg) x = e == 0 ? d : max(x, d);
+                }
+                if (lvl == l) {
+                    i64 start, bill;
+                    if (j0 + jj == 0) {                   // first invocation pre-warmed (G5)
+                        start = x;
+                        bill = T;
+                    } else {
+                        const i64 f = D, g = x - f;
+                        if (g <= 0) {                     // busy: FIFO, stays warm (G6)
+                            start = f;
+                            bill = 0;
+                        } else if (w == 0) {              // keep-alive (Case II)
+                            start = x;
+                            bill = g;
+                        } else if (x < f + w) {           // pre-warm not begun: cold (G3)
+                            start = x + T;
+                            bill = T;
+                        } else if (x < f + w + T) {       // init partly covered (G4)
+                            start = f + w + T;
+                            bill = T;
+                        } else {                          // covered (Case I)
+                            start = x;
+                            bill = x - (f + w);
+                        }
+                    }
+                    D = start + I;
+                    billed += bill + I;
                 }
             }
-            D[k] = start + I[k];
-            billed[k] += bill + I[k];
-            if ((p.sinkmask >> k) & 1u) lat = max(lat, D[k] - r);
+            if (sink) maxlat = max(maxlat, D - r);
         }
-        maxlat = max(maxlat, lat);
     }
+#pragma unroll
+    for (int m = 16; m > 0; m >>= 1) maxlat = max(maxlat, shfl64(maxlat, lane ^ m));
+    // cost = ((U_0 E_0 + U_1 E_1) + ...) left to right, IEEE mul/add, no FMA (G15)
+    const double term = act ? __dmul_rn(p.tabU[row], (double)billed) : 0.0;
     double cost = 0.0;
-    for (int k = 0; k < N; ++k) {
-        const double term = __dmul_rn(p.tabU[p.row0[k] + cfg[k]], (double)billed[k]);
-        cost = (k == 0) ? term : __dadd_rn(cost, term);
+    for (int q = 0; q < N; ++q) {
+        const double tq = __shfl_sync(FULL, term, q);
+        cost = (q == 0) ? tq : __dadd_rn(cost, tq);
     }
     const unsigned char ok = maxlat <= sla ? 1 : 0;
     if (res) {
-        res->cost = cost;
-        res->maxlat = maxlat;
-        res->feasible = ok;
-        for (int k = 0; k < N; ++k) { res->cfg[k] = cfg[k]; res->win[k] = win[k]; }
-    } else {
+        if (act) { res->cfg[k] = cfg; res->win[k] = win; }
+        if (lane == 0) { res->cost = cost; res->maxlat = maxlat; res->feasible = ok; }
+    } else if (lane == 0) {
         p.cost[t] = cost;
         p.maxlat[t] = maxlat;
         p.feas[t] = ok;
@@ -168,15 +212,16 @@ __global__ void eval_exact_kernel(ExactParams p) {
 extern "C" {
 
 int smiless_dev_prep_offsets(const long long *arr, long long J, long long d_cap, int K, int time64, void *off,
-                             long long n_off, long long *scal, int *err, cudaStream_t st) {
+                             long long n_off, long long *scal, int *err, long long *rrem, cudaStream_t st) {
     const long long n_threads = (n_off + K - 1) / K;
     const int bs = 128;
     const unsigned grid = (unsigned)((n_threads + bs - 1) / bs);
     if (grid == 0) return 0;
     if (time64)
-        smiless_dev::prep_offsets_kernel<long long><<<grid, bs, 0, st>>>(arr, J, d_cap, K, (long long *)off, n_off, scal, err);
+        smiless_dev::prep_offsets_kernel<long long><<<grid, bs, 0, st>>>(arr, J, d_cap, K, (long long *)off, n_off, scal, err,
+                                                                         rrem);
     else
-        smiless_dev::prep_offsets_kernel<int><<<grid, bs, 0, st>>>(arr, J, d_cap, K, (int *)off, n_off, scal, err);
+        smiless_dev::prep_offsets_kernel<int><<<grid, bs, 0, st>>>(arr, J, d_cap, K, (int *)off, n_off, scal, err, rrem);
     return (int)cudaGetLastError();
 }
 
@@ -186,8 +231,8 @@ int smiless_dev_reduce_best(const unsigned long long *slots, int n, int stride, 
 }
 
 int smiless_dev_eval_exact(const ExactParams *p, cudaStream_t st) {
-    const int bs = 128;
-    const unsigned grid = (unsigned)((p->n + bs - 1) / bs);
+    const int bs = 128;                                   // 4 candidates (warps) per CTA
+    const unsigned grid = (unsigned)((p->n * 32 + bs - 1) / bs);
     if (grid == 0) return 0;
     smiless_dev::eval_exact_kernel<<<grid, bs, 0, st>>>(*p);
     return (int)cudaGetLastError();

@@ -48,7 +48,7 @@ struct ExactParams {
 
 extern "C" {
 int smiless_dev_prep_offsets(const long long *arr, long long J, long long d_cap, int K, int time64, void *off,
-                             long long n_off, long long *scal, int *err, cudaStream_t st);
+                             long long n_off, long long *scal, int *err, long long *rrem, cudaStream_t st);
 int smiless_dev_reduce_best(const unsigned long long *slots, int n, int stride, ResBlock *res, cudaStream_t st);
 int smiless_dev_eval_exact(const ExactParams *p, cudaStream_t st);
 }

@@ -18,7 +18,7 @@ LIB_PATH = os.path.join(_PKG, "libsmiless.so")
 
 OK, INFEASIBLE = 0, 1
 EINVAL, ENOTTOPO, ERANGE, ESTATE, ECUDA, ENOMEM, EJIT = -1, -2, -3, -4, -5, -6, -7
-FLAG_NO_PRUNE, FLAG_ARRIVALS_ON_DEVICE, FLAG_FORCE_INT64 = 1, 2, 4
+FLAG_NO_PRUNE, FLAG_ARRIVALS_ON_DEVICE, FLAG_FORCE_INT64, FLAG_COST_CAP = 1, 2, 4, 8
 _NAMES = {0: "OK", 1: "INFEASIBLE", -1: "EINVAL", -2: "ENOTTOPO", -3: "ERANGE", -4: "ESTATE",
           -5: "ECUDA", -6: "ENOMEM", -7: "EJIT"}
 
@@ -54,6 +54,7 @@ class PlanArgs(ctypes.Structure):
         ("n_shards", ctypes.c_int32),
         ("cost_out", ctypes.c_void_p),
         ("row_windows_us", ctypes.c_void_p),
+        ("cost_cap", ctypes.c_double),
     ]
 
 
@@ -193,7 +194,7 @@ class Planner:
 
     # ---- args ----------------------------------------------------------------------------
     def _args(self, arrivals, sla_us, windows_us, n_fixed=0, fixed_digits=(), begin=0, end=0, flags=0,
-              shard=0, n_shards=0, cost_out=None, row_windows=None):
+              shard=0, n_shards=0, cost_out=None, row_windows=None, cost_cap=None):
         keep = []
         if _is_device_tensor(arrivals):
             import torch
@@ -214,6 +215,9 @@ class Planner:
                      fixed_digits=fixed.ctypes.data if n_fixed else None, begin=int(begin), end=int(end),
                      flags=int(flags), shard=int(shard), n_shards=int(n_shards),
                      cost_out=cost_out.ctypes.data if cost_out is not None else None)
+        if cost_cap is not None:
+            a.flags |= FLAG_COST_CAP
+            a.cost_cap = float(cost_cap)
         if row_windows is not None:
             rw = _i32(row_windows)
             keep.append(rw)

@@ -116,6 +116,9 @@ def test_plan_argument_validation_before_any_gpu_work():
         (dict(n_fixed=4), S.EINVAL),
         (dict(n_fixed=1, fixed_digits=[16]), S.EINVAL),             # digit >= M*W
         (dict(n_shards=2, shard=2), S.EINVAL),
+        (dict(cost_cap=float("nan")), S.EINVAL),
+        (dict(cost_cap=-1.0), S.EINVAL),
+        (dict(cost_cap=1.0, flags=S.FLAG_NO_PRUNE), S.EINVAL),      # the cap is a prune-mode argument
     ]
     for over, code in cases:
         kw = dict(ok)

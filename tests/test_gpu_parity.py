@@ -680,3 +680,116 @@ def test_memo_variants_shapes_are_exact(g, selmask, monkeypatch):
         assert_same_plan(g_, o.plan(), o)
         n_checked += 1
     assert n_checked > 10
+
+
+# ---------------------------------------------------------------------------------------
+# Cost-bound pruning against an incumbent, and the caller's cost cap (DESIGN.md section 5
+# item 11): only candidates costing strictly more than a real feasible candidate (or the
+# cap) are dropped, so the argmin and its lowest-index tie-break are unchanged
+# ---------------------------------------------------------------------------------------
+
+def _lex_min(oc, of, cap=np.inf):
+    elig = np.nonzero(of & (oc <= cap))[0]
+    if len(elig) == 0:
+        return None
+    best = elig[np.lexsort((elig, oc[elig]))[0]]
+    return int(best), float(oc[best])
+
+
+def test_cost_bound_and_cost_cap_are_exact(monkeypatch):
+    rng = np.random.default_rng(61)
+    checked = fewer = 0
+    for t in range(120):
+        if checked == 12:
+            break
+        n = int(rng.integers(2, 6))
+        p = W.random_problem(rng, n, 4, int(rng.integers(2, 5)), int(rng.integers(150, 400)),
+                             sla_us=int(rng.integers(15_000, 60_000)))
+        space = p.space_size()
+        if space > 40000:
+            continue
+        o = OracleProblem(p)
+        oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
+        ref = o.plan()
+        assert (None if ref is None else (ref[0], ref[1])) == _lex_min(oc, of)
+        pl = S.planner_for(p)
+        args = (p.arrivals_us, p.sla_us, p.windows_us)
+        assert_same_plan(pl.plan(*args), ref, o)                     # running incumbent
+        monkeypatch.setenv("SMILESS_COST_PRUNE", "0")
+        off = pl.plan(*args)
+        monkeypatch.delenv("SMILESS_COST_PRUNE")
+        assert_same_plan(off, ref, o)
+        if ref is None:
+            continue
+        # the tightest valid cap is OPT itself: candidates tying it must survive; with the B&B
+        # pre-pass at every depth the static prefix bound prunes against the cap as well
+        for d in [None] + list(range(1, n)):
+            if d is None:
+                monkeypatch.delenv("SMILESS_BB_DEPTH", raising=False)
+            else:
+                monkeypatch.setenv("SMILESS_BB_DEPTH", str(d))
+            for cap in (ref[1], float(np.nextafter(ref[1], np.inf)), 2 * ref[1] + 1e-3, np.inf):
+                g = pl.plan(*args, cost_cap=cap)
+                assert_same_plan(g, ref, o)
+                assert g.n_decided == space
+            g = pl.plan(*args)
+            assert_same_plan(g, ref, o)
+        monkeypatch.delenv("SMILESS_BB_DEPTH", raising=False)
+        g = pl.plan(*args, cost_cap=ref[1])
+        fewer += g.n_full_evals < off.n_full_evals
+        # a cap below OPT leaves nothing eligible
+        g = pl.plan(*args, cost_cap=float(np.nextafter(ref[1], 0)))
+        assert g.status == S.INFEASIBLE and g.index is None
+        # sub-ranges and shards with a cap between two feasible costs
+        costs = np.unique(oc[of])
+        if len(costs) > 1:
+            cap = float(costs[len(costs) // 2])
+            b, e = int(rng.integers(0, space // 2)), int(rng.integers(space // 2, space + 1))
+            want = _lex_min(oc[b:e], of[b:e], cap)
+            g = pl.plan(*args, begin=b, end=e, cost_cap=cap)
+            assert (None if want is None else (want[0] + b, want[1])) == \
+                (None if g.index is None else (g.index, g.cost))
+            parts = [pl.plan(*args, shard=s_, n_shards=3, cost_cap=cap) for s_ in range(3)]
+            feas = [(r.cost, r.index) for r in parts if r.feasible]
+            want = _lex_min(oc, of, cap)
+            assert (min(feas) if feas else None) == (None if want is None else (want[1], want[0]))
+        checked += 1
+    assert checked >= 8 and fewer >= 1
+
+
+def test_cost_cap_ties_and_single_candidate():
+    """Zero prices: every candidate costs 0, a cap of 0 keeps them all and the winner is the
+    lowest feasible index; a fully pinned (single-candidate) plan honours the cap too."""
+    rng = np.random.default_rng(3)
+    p = W.random_problem(rng, 3, 3, 3, 20, sla_us=10**8)
+    p = p.replace(price_per_us=np.zeros_like(p.price_per_us))
+    pl = S.planner_for(p)
+    g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, cost_cap=0.0)
+    assert g.index == 0 and g.cost == 0.0
+    p2 = p.replace(price_per_us=np.ones_like(p.price_per_us) / 1024)
+    o = OracleProblem(p2, n_fixed=3, fixed_digits=[0, 0, 0])
+    c, l, f = o.evaluate([0])
+    pl2 = S.planner_for(p2)
+    kw = dict(n_fixed=3, fixed_digits=[0, 0, 0])
+    g = pl2.plan(p2.arrivals_us, p2.sla_us, p2.windows_us, cost_cap=float(c[0]), **kw)
+    assert g.index == 0 and g.cost == c[0]
+    g = pl2.plan(p2.arrivals_us, p2.sla_us, p2.windows_us, cost_cap=float(np.nextafter(c[0], 0)), **kw)
+    assert g.status == S.INFEASIBLE
+
+
+def test_exact_evaluator_wide_dags():
+    """The warp-per-candidate exact evaluator (lane k = function k, DAG levels in parallel) at
+    the ABI limits: 32 functions, joins of up to 8 predecessors (past its 4 register-cached
+    ones), several sinks; evaluated indices and a plan sub-range against the oracle."""
+    rng = np.random.default_rng(71)
+    for t in range(3):
+        p = W.random_problem(rng, 32, 2, 1 + t % 2, 300, max_preds=8, sla_us=10**9)
+        space = p.space_size()
+        o = OracleProblem(p)
+        idx = rng.integers(0, space, size=96, dtype=np.uint64)
+        pl = S.planner_for(p)
+        gc, gl, gf = pl.evaluate(idx, p.arrivals_us, p.sla_us, p.windows_us)
+        assert_same_eval(gc, gl, gf, *o.evaluate(idx))
+        b = int(rng.integers(0, space - 4096))
+        g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, begin=b, end=b + 4096)
+        assert_same_plan(g, o.plan(begin=b, end=b + 4096), o)
