@@ -56,7 +56,9 @@ NvrtcApi &nvrtc() {
     static std::once_flag once;
     std::call_once(once, [] {
         const char *env = getenv("SMILESS_NVRTC");
-        const char *cands[] = {env, "libnvrtc.so.12", "/usr/local/cuda/lib64/libnvrtc.so.12", "libnvrtc.so"};
+        // the toolkit's own NVRTC first: a bare soname may resolve to an older copy another
+        // library (e.g. a framework's bundled runtime) already loaded into the process
+        const char *cands[] = {env, "/usr/local/cuda/lib64/libnvrtc.so.12", "libnvrtc.so.12", "libnvrtc.so"};
         void *h = nullptr;
         for (const char *c : cands) {
             if (!c) continue;
@@ -1433,16 +1435,27 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                     unsigned n_a = 0;
                     CK(cudaMemcpyAsync(&n_a, ctx->dListCntA.p, sizeof n_a, cudaMemcpyDeviceToHost, st), "D2H count");
                     CK(cudaStreamSynchronize(st), "count");
-                    // per-chunk entry counts, uploaded once (no host sync inside the loop)
-                    const u64 n_chunks_a = (n_a + per_chunk - 1) / per_chunk;
-                    std::vector<unsigned> cnts((size_t)std::max<u64>(1, n_chunks_a));
-                    for (u64 i = 0; i < n_chunks_a; ++i)
-                        cnts[i] = (unsigned)std::min<u64>(per_chunk, n_a - i * per_chunk);
+                    // per-chunk entry counts, uploaded once (no host sync inside the loop).  With the
+                    // cost bound on, the first chunk is small: its evaluation sets the incumbent the
+                    // static prefix bound of every later chunk prunes against.
+                    const char *first_env = getenv("SMILESS_BB_FIRST");
+                    const u64 first = std::max<u64>(1, std::min<u64>(per_chunk, pp.cost_prune ? (first_env ? (u64)atoll(first_env) : 64)
+                                                                                             : per_chunk));
+                    std::vector<unsigned> cnts;
+                    std::vector<u64> starts;
+                    for (u64 c0 = 0; c0 < n_a;) {
+                        const u64 len = std::min<u64>(c0 == 0 ? first : per_chunk, n_a - c0);
+                        starts.push_back(c0);
+                        cnts.push_back((unsigned)len);
+                        c0 += len;
+                    }
+                    const u64 n_chunks_a = cnts.size();
+                    if (cnts.empty()) cnts.push_back(0);
                     CK(ctx->dChunkCnt.ensure(cnts.size()), "cudaMalloc counts");
                     CK(cudaMemcpy(ctx->dChunkCnt.p, cnts.data(), cnts.size() * sizeof(unsigned), cudaMemcpyHostToDevice),
                        "H2D counts");
                     for (u64 i = 0; i < n_chunks_a; ++i) {
-                        const u64 c0 = i * per_chunk;
+                        const u64 c0 = starts[i];
                         CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
                         CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
                         bp.list_in = ctx->dListA.p + c0;

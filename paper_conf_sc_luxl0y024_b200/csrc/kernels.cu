@@ -81,18 +81,19 @@ __global__ void reduce_best_kernel(const u64 *__restrict__ slots, int n, int str
 
 // Exact evaluation, absolute int64 times, generic DAG (runtime CSR in device memory), the
 // plain case split of model M with per-step billing -- independent of the
-// NVRTC evaluator's reformulations.  One WARP per candidate, lane k = function k: within an
-// invocation the functions run level by level of the DAG (a function's level = 1 + the
-// highest level of its predecessors), a predecessor's done time comes over a shuffle, so an
-// invocation costs (levels x max in-degree) shuffles instead of N dependent local-memory
-// walks.  Arrivals are read 32 at a time (one coalesced load) and broadcast by shuffle.
-__device__ __forceinline__ long long shfl64(long long v, int src) {
-    return (long long)__shfl_sync(0xffffffffu, (unsigned long long)v, src);
-}
+// NVRTC evaluator's reformulations.  One WARP per candidate, lane k = function k, run as a
+// wavefront: a function's level is 1 + the highest level of its predecessors, and at
+// iteration t lane k handles invocation j = t - level_k.  Its predecessors (lower levels)
+// finished invocation j in earlier iterations and left D[p][j] in a per-warp shared ring of
+// 32 invocations (level gaps are <= 31, so a slot is never overwritten before it is read);
+// one __syncwarp per iteration orders the ring.  A whole invocation of the DAG thus costs
+// one iteration of the warp instead of N dependent steps of one thread.
+#define EXACT_WARPS 4
 
-__global__ void eval_exact_kernel(ExactParams p) {
+__global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParams p) {
+    __shared__ long long ring[EXACT_WARPS][SMILESS_DEV_MAX_FUNCS][32];   // [warp][function][j % 32]
     const unsigned FULL = 0xffffffffu;
-    const int lane = threadIdx.x & 31;
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const i64 t = ((i64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;   // candidate of this warp
     if (t >= p.n) return;                                                // warp-uniform
     ResBlock *res = p.idx_from_res ? p.res + t : nullptr;
@@ -122,73 +123,72 @@ __global__ void eval_exact_kernel(ExactParams p) {
     const i64 w = act ? (p.rowwin ? p.rowwin[row] : p.win[win]) : 0;
     const int e0 = act ? p.pred_ptr[k] : 0, deg = act ? p.pred_ptr[k + 1] - e0 : 0;
     const bool sink = act && ((p.sinkmask >> k) & 1u);
-    int pc[4];                                            // first predecessors in registers
-#pragma unroll
-    for (int e = 0; e < 4; ++e) pc[e] = e < deg ? p.pred_idx[e0 + e] : lane;
     int maxdeg = deg;
 #pragma unroll
     for (int m = 16; m > 0; m >>= 1) maxdeg = max(maxdeg, __shfl_xor_sync(FULL, maxdeg, m));
     // ---- topological levels (Bellman-Ford over the warp, N passes at most) -----------------
-    int lvl = act ? 0 : -1;
+    int lvl = 0;
     for (int pass = 0; pass < N; ++pass) {
-        int l2 = act ? 0 : -1;
+        int l2 = 0;
         for (int e = 0; e < maxdeg; ++e) {
-            const int src = e < deg ? (e < 4 ? pc[e] : p.pred_idx[e0 + e]) : lane;
+            const int src = e < deg ? p.pred_idx[e0 + e] : lane;
             const int lp = __shfl_sync(FULL, lvl, src);
             if (e < deg) l2 = max(l2, lp + 1);
         }
         lvl = l2;
     }
-    int nlev = lvl + 1;
+    int nlev = act ? lvl + 1 : 1;
 #pragma unroll
     for (int m = 16; m > 0; m >>= 1) nlev = max(nlev, __shfl_xor_sync(FULL, nlev, m));
 
+    long long (*rg)[32] = ring[wib];
+    const i64 J = p.J;
     i64 D = 0, billed = 0, maxlat = INT64_MIN;
-    for (i64 j0 = 0; j0 < p.J; j0 += 32) {
-        const i64 rb = j0 + lane < p.J ? p.arr[j0 + lane] : 0;
-        const int jn = (int)min((i64)32, p.J - j0);
-        for (int jj = 0; jj < jn; ++jj) {
-            const i64 r = shfl64(rb, jj);
-            for (int l = 0; l < nlev; ++l) {
-                i64 x = r;                                // sources: the request's arrival
-                for (int e = 0; e < maxdeg; ++e) {        // AND-join: max over predecessors
-                    const int src = e < deg ? (e < 4 ? pc[e] : p.pred_idx[e0 + e]) : lane;
-                    const i64 d = shfl64(D, src);
-                    if (e < deg) x = e == 0 ? d : max(x, d);
-                }
-                if (lvl == l) {
-                    i64 start, bill;
-                    if (j0 + jj == 0) {                   // first invocation pre-warmed (G5)
-                        start = x;
-                        bill = T;
-                    } else {
-                        const i64 f = D, g = x - f;
-                        if (g <= 0) {                     // busy: FIFO, stays warm (G6)
-                            start = f;
-                            bill = 0;
-                        } else if (w == 0) {              // keep-alive (Case II)
-                            start = x;
-                            bill = g;
-                        } else if (x < f + w) {           // pre-warm not begun: cold (G3)
-                            start = x + T;
-                            bill = T;
-                        } else if (x < f + w + T) {       // init partly covered (G4)
-                            start = f + w + T;
-                            bill = T;
-                        } else {                          // covered (Case I)
-                            start = x;
-                            bill = x - (f + w);
-                        }
-                    }
-                    D = start + I;
-                    billed += bill + I;
+    i64 rcur = act ? p.arr[0] : 0;                        // r_j of this lane's next invocation
+    for (i64 it = 0; it < J + nlev - 1; ++it) {
+        const i64 j = it - lvl;
+        const bool on = act && j >= 0 && j < J;
+        const i64 r = rcur;
+        if (on && j + 1 < J) rcur = p.arr[j + 1];          // prefetch for the next iteration
+        if (on) {
+            i64 x = r;                                    // sources: the request's arrival
+            for (int e = 0; e < deg; ++e) {               // AND-join: max over predecessors
+                const i64 d = rg[p.pred_idx[e0 + e]][j & 31];
+                x = e == 0 ? d : max(x, d);
+            }
+            i64 start, bill;
+            if (j == 0) {                                 // first invocation pre-warmed (G5)
+                start = x;
+                bill = T;
+            } else {
+                const i64 f = D, g = x - f;
+                if (g <= 0) {                             // busy: FIFO, stays warm (G6)
+                    start = f;
+                    bill = 0;
+                } else if (w == 0) {                      // keep-alive (Case II)
+                    start = x;
+                    bill = g;
+                } else if (x < f + w) {                   // pre-warm not begun: cold (G3)
+                    start = x + T;
+                    bill = T;
+                } else if (x < f + w + T) {               // init partly covered (G4)
+                    start = f + w + T;
+                    bill = T;
+                } else {                                  // covered (Case I)
+                    start = x;
+                    bill = x - (f + w);
                 }
             }
+            D = start + I;
+            billed += bill + I;
+            rg[k][j & 31] = D;
             if (sink) maxlat = max(maxlat, D - r);
         }
+        __syncwarp();
     }
 #pragma unroll
-    for (int m = 16; m > 0; m >>= 1) maxlat = max(maxlat, shfl64(maxlat, lane ^ m));
+    for (int m = 16; m > 0; m >>= 1)
+        maxlat = max(maxlat, (i64)__shfl_xor_sync(FULL, (unsigned long long)maxlat, m));
     // cost = ((U_0 E_0 + U_1 E_1) + ...) left to right, IEEE mul/add, no FMA (G15)
     const double term = act ? __dmul_rn(p.tabU[row], (double)billed) : 0.0;
     double cost = 0.0;
@@ -231,7 +231,7 @@ int smiless_dev_reduce_best(const unsigned long long *slots, int n, int stride, 
 }
 
 int smiless_dev_eval_exact(const ExactParams *p, cudaStream_t st) {
-    const int bs = 128;                                   // 4 candidates (warps) per CTA
+    const int bs = 32 * EXACT_WARPS;                      // one candidate (warp) each
     const unsigned grid = (unsigned)((p->n * 32 + bs - 1) / bs);
     if (grid == 0) return 0;
     smiless_dev::eval_exact_kernel<<<grid, bs, 0, st>>>(*p);

@@ -569,6 +569,16 @@ def test_two_level_branch_and_bound_is_exact(monkeypatch):
                 assert g.n_decided == space
                 parts = [pl.plan(p.arrivals_us, p.sla_us, p.windows_us, shard=s_, n_shards=2) for s_ in range(2)]
                 assert sum(r.n_decided for r in parts) == space
+                # one shallow survivor per deep chunk: every later chunk's static prefix bound
+                # prunes against the incumbent the earlier chunks set (cost bound on)
+                monkeypatch.setenv("SMILESS_BB_FIRST", "1")
+                g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us)
+                assert_same_plan(g, ref, o)
+                assert g.n_decided == space
+                if ref is not None:
+                    g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, cost_cap=ref[1])
+                    assert_same_plan(g, ref, o)
+                monkeypatch.delenv("SMILESS_BB_FIRST")
         n_checked += 1
     assert n_checked > 8
 
@@ -783,7 +793,7 @@ def test_exact_evaluator_wide_dags():
     ones), several sinks; evaluated indices and a plan sub-range against the oracle."""
     rng = np.random.default_rng(71)
     for t in range(3):
-        p = W.random_problem(rng, 32, 2, 1 + t % 2, 300, max_preds=8, sla_us=10**9)
+        p = W.random_problem(rng, 32, 2, 1 + t % 2, 300, max_preds=8, sla_us=5 * 10**8)
         space = p.space_size()
         o = OracleProblem(p)
         idx = rng.integers(0, space, size=96, dtype=np.uint64)
