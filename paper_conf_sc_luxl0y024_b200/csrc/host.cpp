@@ -627,9 +627,10 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     const char *mask_env = getenv("SMILESS_MASK");   // tuning knob, see evaluator.cuh SM_MASK
     s << "#define SM_MASK " << (mask_env ? atoi(mask_env) : 0) << "\n";
     s << "#define SM_XPF " << xpf_groups() << "\n";
-    // tuning knob, see evaluator.cuh SM_SELMASK; default: window variants 1 and 2 use select
+    // tuning knob, see evaluator.cuh SM_SELMASK; default: every window variant uses the IMAD.HI
+    // busy mask (measured best once the x stream is prefetched, profiles/r01k_sweep_variants.md)
     const char *sel_env = getenv("SMILESS_SELMASK");
-    s << "#define SM_SELMASK " << (sel_env ? atoi(sel_env) : 6) << "\n";
+    s << "#define SM_SELMASK " << (sel_env ? atoi(sel_env) : 0) << "\n";
     // compile-time window grid (immediates) and a constant-bank copy for runtime indices
     s << "#define SM_WIN(v) (";
     for (int v = 0; v < W; ++v) s << "(v)==" << v << "?" << a->windows_us[v] << ":";

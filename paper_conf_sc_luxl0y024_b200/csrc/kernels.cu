@@ -123,6 +123,9 @@ __global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParam
     const i64 w = act ? (p.rowwin ? p.rowwin[row] : p.win[win]) : 0;
     const int e0 = act ? p.pred_ptr[k] : 0, deg = act ? p.pred_ptr[k + 1] - e0 : 0;
     const bool sink = act && ((p.sinkmask >> k) & 1u);
+    int pc[4];                                            // first predecessors, in registers
+#pragma unroll
+    for (int e = 0; e < 4; ++e) pc[e] = e < deg ? p.pred_idx[e0 + e] : 0;
     int maxdeg = deg;
 #pragma unroll
     for (int m = 16; m > 0; m >>= 1) maxdeg = max(maxdeg, __shfl_xor_sync(FULL, maxdeg, m));
@@ -152,10 +155,15 @@ __global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParam
         if (on && j + 1 < J) rcur = p.arr[j + 1];          // prefetch for the next iteration
         if (on) {
             i64 x = r;                                    // sources: the request's arrival
-            for (int e = 0; e < deg; ++e) {               // AND-join: max over predecessors
-                const i64 d = rg[p.pred_idx[e0 + e]][j & 31];
-                x = e == 0 ? d : max(x, d);
+            const int sl = (int)(j & 31);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {                 // AND-join: max over predecessors
+                if (e < deg) {
+                    const i64 d = rg[pc[e]][sl];
+                    x = e == 0 ? d : max(x, d);
+                }
             }
+            for (int e = 4; e < deg; ++e) x = max(x, rg[p.pred_idx[e0 + e]][sl]);
             i64 start, bill;
             if (j == 0) {                                 // first invocation pre-warmed (G5)
                 start = x;

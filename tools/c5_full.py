@@ -19,18 +19,22 @@ arr = torch.as_tensor(p.arrivals_us).cuda()
 pl.plan(arr, p.sla_us, p.windows_us, n_fixed=2, fixed_digits=[0, 0], end=1 << 20)   # JIT warm-up
 torch.cuda.synchronize()
 t0 = time.perf_counter()
-best, per = None, []
+best, per, dev, launches = None, [], [], 0
 decided = 0
 for d0 in range(n_dig):
     t1 = time.perf_counter()
-    r = pl.plan(arr, p.sla_us, p.windows_us, n_fixed=1, fixed_digits=[d0])
+    cap = {"cost_cap": best[0]} if best is not None else {}        # cheapest feasible so far
+    r = pl.plan(arr, p.sla_us, p.windows_us, n_fixed=1, fixed_digits=[d0], **cap)
     per.append(time.perf_counter() - t1)
+    dev.append(r.total_device_ms)
+    launches += r.launches
     decided += r.n_decided
     if r.feasible and (best is None or (r.cost, d0, r.index) < best[:3]):
         best = (r.cost, d0, r.index, r.max_latency_us, r.config.tolist(), r.window.tolist())
 dt = time.perf_counter() - t0
 out = {"config": "C5", "digits_planned": n_dig, "candidates": decided, "time_to_optimal_s": dt,
        "per_subplan_s": {"mean": float(np.mean(per)), "max": float(np.max(per))},
+       "per_subplan_device_ms": {"mean": float(np.mean(dev)), "max": float(np.max(dev))}, "launches": launches,
        "decided_per_s": decided / dt}
 if best:
     cost, d0, idx, lat, cfg, win = best

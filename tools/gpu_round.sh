@@ -19,3 +19,12 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:"smi
     > $O/${TAG}_ncu_full.log 2>&1
 echo "ncu full exit $?"
 ls -la $O | tail -20
+# multi-rank flow on the one GPU (gloo collectives, SMILESS_BENCH_SAME_GPU): sharded slice,
+# full-space plans and the C5 cross-rank incumbent exchange, oracle-checked winners
+SMILESS_BENCH_SAME_GPU=1 timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 \
+    --master-port 29533 bench.py --gpus 2 --steps 2 --warmup 3 --no-cpu-baseline --no-c4 > $O/${TAG}_bench_2rank.log 2>&1
+echo "2-rank exit $?"; python -c "
+import json,sys
+d=json.loads([l for l in open(sys.argv[1]) if l.startswith('{')][-1])
+print('2rank value %.4g' % d['value'], {k: (v['time_to_optimal_s'], v.get('oracle_check'), v['cost']) for k, v in d['time_to_optimal_full_space'].items()})
+" $O/${TAG}_bench_2rank.log || tail -20 $O/${TAG}_bench_2rank.log
