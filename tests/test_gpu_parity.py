@@ -665,14 +665,17 @@ def test_throughput_mode_with_and_without_prefix_memoisation(memo, monkeypatch):
     assert n_checked > 20
 
 
-@pytest.mark.parametrize("g,selmask", [("1", "0"), ("1", "2"), ("2", "255"), ("4", "6")])
-def test_memo_variants_shapes_are_exact(g, selmask, monkeypatch):
+@pytest.mark.parametrize("g,selmask,alu", [("1", "0", "0 0"), ("1", "2", "255 255"), ("2", "255", "42 0"),
+                                            ("4", "6", "0 170")])
+def test_memo_variants_shapes_are_exact(g, selmask, alu, monkeypatch):
     """The variants kernel's tuning knobs (configs per lane G, select vs IMAD.HI busy mask
-    per window variant) change only the instruction mix: per-candidate parity with the
-    oracle for each."""
+    per window variant, adds pinned to the ALU pipe) change only the instruction mix:
+    per-candidate parity with the oracle for each."""
     monkeypatch.setenv("SMILESS_MEMO", "1")
     monkeypatch.setenv("SMILESS_G", g)
     monkeypatch.setenv("SMILESS_SELMASK", selmask)
+    monkeypatch.setenv("SMILESS_ALUG", alu.split()[0])
+    monkeypatch.setenv("SMILESS_ALUSUL", alu.split()[1])
     rng = np.random.default_rng(131 + int(g) * 7 + int(selmask))
     n_checked = 0
     for t in range(30):
