@@ -20,6 +20,20 @@ os.environ["SMILESS_BB_DEPTH"] = "0"
 os.environ["SMILESS_HORIZON"] = "64"
 plq.plan(q.arrivals_us, q.sla_us, q.windows_us)
 plq.plan_sla_sweep(q.arrivals_us, [20_000, 40_000], q.windows_us)
+# cost bound: two-level B&B with one shallow survivor per deep chunk and a cost cap
+os.environ.pop("SMILESS_HORIZON")
+os.environ.update(SMILESS_BB_DEPTH="3", SMILESS_BB_DEPTH_A="1", SMILESS_BB_FIRST="1")
+r = plq.plan(q.arrivals_us, q.sla_us, q.windows_us)
+if r.feasible:
+    plq.plan(q.arrivals_us, q.sla_us, q.windows_us, cost_cap=r.cost)
+for k in ("SMILESS_BB_DEPTH", "SMILESS_BB_DEPTH_A", "SMILESS_BB_FIRST"):
+    os.environ.pop(k)
+# prefix memoisation (throughput mode) and the wavefront exact evaluator on a 32-function DAG
+os.environ["SMILESS_MEMO"] = "1"
+plq.plan(q.arrivals_us, q.sla_us, q.windows_us, flags=S.FLAG_NO_PRUNE)
+w = W.random_problem(rng, 32, 2, 2, 100, max_preds=8, sla_us=5 * 10**8)
+S.planner_for(w).evaluate(rng.integers(0, w.space_size(), size=8, dtype=np.uint64), w.arrivals_us, w.sla_us,
+                          w.windows_us)
 print("sanitize workload done")
 PY
 for tool in memcheck racecheck synccheck initcheck; do
