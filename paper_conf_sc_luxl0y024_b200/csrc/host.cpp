@@ -13,6 +13,7 @@
 #include <nvrtc.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -1156,11 +1157,36 @@ int smiless_evaluate(smiless_ctx *ctx, const smiless_plan_args *a, const uint64_
 
 namespace {
 
+// SMILESS_PROFILE_HOST=1: host-side stage timestamps of every plan call on stderr (tuning aid)
+struct HostProf {
+    bool on;
+    std::chrono::steady_clock::time_point t0, last;
+    std::string line;
+    HostProf() : on(getenv("SMILESS_PROFILE_HOST") != nullptr) {
+        if (on) t0 = last = std::chrono::steady_clock::now();
+    }
+    void mark(const char *what) {
+        if (!on) return;
+        const auto now = std::chrono::steady_clock::now();
+        char b[96];
+        snprintf(b, sizeof b, " %s=%.0fus", what, std::chrono::duration<double, std::micro>(now - last).count());
+        line += b;
+        last = now;
+    }
+    ~HostProf() {
+        if (on)
+            fprintf(stderr, "[smiless host] total=%.0fus%s\n",
+                    std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - t0).count(),
+                    line.c_str());
+    }
+};
+
 // The hot path.  n_sla = 1: an ordinary plan with a->sla_us.  n_sla > 1: one evaluation of the
 // space, one argmin key per SLA in slas[] (pruning against their maximum); a->sla_us is ignored.
 int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, int n_sla, smiless_plan_result *res,
               int32_t *config_out, int32_t *window_out) {
     if (!a_in) return fail(ctx, SMILESS_EINVAL, "args is NULL");
+    HostProf hp;
     smiless_plan_args a_copy = *a_in;
     i64 sla_max = slas[0];
     for (int s_ = 1; s_ < n_sla; ++s_) sla_max = std::max<i64>(sla_max, slas[s_]);
@@ -1218,8 +1244,10 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                                smem_memo_var(ctx, a, rp, n_off) <= 227 * 1024;
         const bool bnb_path = !memo_path && bb_depth(ctx, a) > 0 && smem_bound_bytes(ctx, a, rp, n_off) <= 227 * 1024;
         const int families = memo_path ? (FAM_MEMO | FAM_PLAN) : (bnb_path ? (FAM_PLAN | FAM_BOUND) : FAM_PLAN);
+        hp.mark("setup");
         JitKernel *jk = nullptr;
         if ((rc = get_kernel(ctx, a, rp, n_off, families, &jk))) return rc;
+        hp.mark("get_kernel");
         const u64 V = (u64)a->n_windows * (u64)configs_per_lane(ctx, a);   // candidates per unit
         const u64 ub = cb / V, ue = (ce + V - 1) / V;
         const u64 U = ue - ub;
@@ -1437,8 +1465,10 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                     bp.list_cnt = ctx->dListCntA.p;
                     if ((rc = run_bound(jk->fn_bound_a))) return rc;
                     unsigned n_a = 0;
+                    hp.mark("launch_a");
                     CK(cudaMemcpyAsync(&n_a, ctx->dListCntA.p, sizeof n_a, cudaMemcpyDeviceToHost, st), "D2H count");
                     CK(cudaStreamSynchronize(st), "count");
+                    hp.mark("sync_a");
                     // per-chunk entry counts, uploaded once (no host sync inside the loop).  With the
                     // cost bound on, the first chunk is small: its evaluation sets the incumbent the
                     // static prefix bound of every later chunk prunes against.
@@ -1473,7 +1503,9 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                         if ((rc = run_bound(jk->fn_bound))) return rc;
                         if ((rc = run_eval())) return rc;
                     }
+                    hp.mark("chunks_launched");
                     CK(cudaStreamSynchronize(st), "chunks");      // cnts must outlive its uploads
+                    hp.mark("sync_chunks");
                 }
             } else {
                 u64 bi = 0;
@@ -1574,7 +1606,9 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     CK(cudaMemcpyAsync(&ctx->dRes.p->err, ctx->dErr.p, sizeof(int), cudaMemcpyDeviceToDevice, st), "D2D err");
     CK(cudaMemcpyAsync(ctx->hRes, ctx->dRes.p, sizeof(ResBlock) * n_sla, cudaMemcpyDeviceToHost, st), "D2H result");
     CK(cudaEventRecord(ctx->ev[3], st), "event");
+    hp.mark("tail_launched");
     CK(cudaStreamSynchronize(st), "plan");
+    hp.mark("sync_final");
     float ms = 0.f, tot = 0.f;
     cudaEventElapsedTime(&ms, ctx->ev[1], ctx->ev[2]);
     cudaEventElapsedTime(&tot, ctx->ev[0], ctx->ev[3]);
