@@ -164,28 +164,18 @@ __global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParam
                 }
             }
             for (int e = 4; e < deg; ++e) x = max(x, rg[p.pred_idx[e0 + e]][sl]);
-            i64 start, bill;
+            // the case split of model M as selects (lanes of one warp take different cases;
+            // straight-line code keeps them converged)
+            const i64 f = D, g = x - f, s = f + w;
+            const bool busy = g <= 0;                     // busy: FIFO, stays warm (G6)
+            const bool keep = w == 0;                     // keep-alive (Case II)
+            const bool cold = x < s;                      // pre-warm not begun: cold (G3)
+            const bool part = x < s + T;                  // init partly covered (G4); else covered (Case I)
+            i64 start = busy ? f : keep ? x : cold ? x + T : part ? s + T : x;
+            i64 bill = busy ? 0 : keep ? g : (cold || part) ? T : x - s;
             if (j == 0) {                                 // first invocation pre-warmed (G5)
                 start = x;
                 bill = T;
-            } else {
-                const i64 f = D, g = x - f;
-                if (g <= 0) {                             // busy: FIFO, stays warm (G6)
-                    start = f;
-                    bill = 0;
-                } else if (w == 0) {                      // keep-alive (Case II)
-                    start = x;
-                    bill = g;
-                } else if (x < f + w) {                   // pre-warm not begun: cold (G3)
-                    start = x + T;
-                    bill = T;
-                } else if (x < f + w + T) {               // init partly covered (G4)
-                    start = f + w + T;
-                    bill = T;
-                } else {                                  // covered (Case I)
-                    start = x;
-                    bill = x - (f + w);
-                }
             }
             D = start + I;
             billed += bill + I;
