@@ -375,9 +375,21 @@ def main():
             dist.barrier()
         torch.cuda.synchronize(dev)
 
-    for _ in range(args.warmup):
+    t_first = time.perf_counter()
+    first_call_s = None
+    for w_ in range(args.warmup):
         r = step(arr_dev)
+        if w_ == 0:
+            torch.cuda.synchronize(dev)
+            first_call_s = time.perf_counter() - t_first      # includes the NVRTC specialisation
     barrier()
+    # NVRTC compile of the DAG-specialised module, timed on its own (SURVEY 8(d) ii): a fresh
+    # planner for the same DAG compiles once on its first call
+    t_c = time.perf_counter()
+    pl_c = S.planner_for(p, device=local, stream=stream.cuda_stream)
+    pl_c.jit_compile(p.arrivals_us, p.sla_us, p.windows_us, **dict(kw, flags=S.FLAG_NO_PRUNE))
+    nvrtc_s = time.perf_counter() - t_c
+    del pl_c
 
     def timed(arrivals, n):
         evs = []
@@ -508,6 +520,11 @@ def main():
                      "int_ops_per_candidate": ops_per_cand, "configs_per_lane": configs_per_lane(p),
                      "peak_basis": "issue peak: SMs x 4 SMSP x 32 lanes x sm_max_mhz (DESIGN.md Roofline)"},
         "kernel_share_of_step": kernel_ms_per_step / (ms / args.steps),
+        # SURVEY 8(d) i/ii: function-steps/s (N functions x (J-1) transitions per candidate) and
+        # the NVRTC specialisation, reported apart from the timed steps
+        "function_steps_per_s": value * p.n_funcs * (len(p.arrivals_us) - 1),
+        "nvrtc_compile_s": nvrtc_s,
+        "first_call_s": first_call_s,
     }
     if world == 1 and not args.no_cpu_baseline:
         rate, n, dt, threads = cpu_oracle_rate(p, kw)
