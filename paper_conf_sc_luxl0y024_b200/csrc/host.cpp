@@ -632,6 +632,8 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     // busy mask (measured best once the x stream is prefetched, profiles/r01k_sweep_variants.md)
     const char *sel_env = getenv("SMILESS_SELMASK");
     s << "#define SM_SELMASK " << (sel_env ? atoi(sel_env) : 0) << "\n";
+    const char *vun_env = getenv("SMILESS_VUNROLL");
+    s << "#define SM_VUNROLL " << (vun_env ? atoi(vun_env) : 4) << "\n";
     const char *alusul_env = getenv("SMILESS_ALUSUL"), *alug_env = getenv("SMILESS_ALUG");
     s << "#define SM_ALUSUL " << (alusul_env ? atoi(alusul_env) : 0) << "\n#define SM_ALUG "
       << (alug_env ? atoi(alug_env) : 0) << "\n";
