@@ -528,8 +528,11 @@ def main():
     }
     if world == 1 and not args.no_cpu_baseline:
         rate, n, dt, threads = cpu_oracle_rate(p, kw)
+        rate1, n1, dt1, _ = cpu_oracle_rate(p, kw, seconds=2.0, threads=1)       # SURVEY 8(d) iii
         line["cpu_baseline"] = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle",
-                                "sample": f"first {n} candidates of the slice ({dt:.1f} s, J={len(p.arrivals_us)})"}
+                                "sample": f"first {n} candidates of the slice ({dt:.1f} s, J={len(p.arrivals_us)})",
+                                "single_core_value": rate1,
+                                "single_core_sample": f"first {n1} candidates, 1 thread ({dt1:.1f} s)"}
         if full:
             for name, f in full.items():          # what the same exhaustive search costs on the oracle
                 f["oracle_extrapolated_s"] = f["candidates"] / rate
