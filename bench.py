@@ -151,7 +151,7 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
     reduced lexicographically on (cost bits, digit, index) across ranks."""
     import torch
     import torch.distributed as dist
-    from paper_conf_sc_luxl0y024_b200.dist import cost_bits, bits_cost, reduce_lex, INF_BITS
+    from paper_conf_sc_luxl0y024_b200.dist import cost_bits, bits_cost, reduce_lex, plan_pinned_rounds, INF_BITS
     p = W.make_config(name)
     Wn = len(p.windows_us)
     pl = S.planner_for(p, device=local, stream=stream.cuda_stream)
@@ -165,32 +165,15 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
     b = torch.cuda.Event(enable_timing=True)
     t0 = time.perf_counter()
     a.record(stream)
-    best, decided, full_evals = None, 0, 0
-    cap_bits = INF_BITS                  # cheapest feasible cost found so far on ANY rank
-    n_rounds = (len(digits) + world - 1) // world if pinned else 1
-    for rnd in range(n_rounds):
-        i = rnd * world + rank if pinned else 0
-        if i < len(digits):
-            d0 = digits[i]
-            if pinned:
-                # the global incumbent caps the next sub-plan: its cost bound then prunes from
-                # the first launch (a cap >= OPT keeps the result exact; ties resolve on
-                # (cost, digit, index) below)
-                cap = {"cost_cap": bits_cost(cap_bits)} if cap_bits != INF_BITS else {}
-                r = pl.plan(arr, p.sla_us, p.windows_us, n_fixed=1, fixed_digits=[d0], **cap)
-            else:
-                r = pl.plan(arr, p.sla_us, p.windows_us, shard=rank, n_shards=world)
-            decided += r.n_decided
-            full_evals += r.n_full_evals
-            if r.feasible and (best is None or (r.cost, d0 or 0, r.index) < best[:3]):
-                best = (r.cost, d0 or 0, r.index, r.max_latency_us)
-        if best is not None:
-            cap_bits = min(cap_bits, cost_bits(best[0]))
-        if pinned and world > 1 and rnd + 1 < n_rounds:
-            # one 8-byte MIN all-reduce per round: every rank prunes against the global best
-            t = torch.tensor([cap_bits], dtype=torch.int64, device=xdev)
-            dist.all_reduce(t, op=dist.ReduceOp.MIN)
-            cap_bits = int(t.item())
+    if pinned:
+        best, decided, full_evals, _ = plan_pinned_rounds(
+            lambda d0, cap: pl.plan(arr, p.sla_us, p.windows_us, n_fixed=1, fixed_digits=[d0],
+                                    **({"cost_cap": cap} if cap is not None else {})),
+            digits, rank, world, xdev)
+    else:
+        r = pl.plan(arr, p.sla_us, p.windows_us, shard=rank, n_shards=world)
+        decided, full_evals = r.n_decided, r.n_full_evals
+        best = (r.cost, 0, r.index, r.max_latency_us) if r.feasible else None
     keys = [cost_bits(best[0]) if best else INF_BITS, best[1] if best else 0, best[2] if best else 0]
     payload = [best[3] if best else -1]
     if world > 1:

@@ -91,3 +91,38 @@ def reduce_lex(keys, payload, device, group=None):
     s = torch.tensor([int(x) if tied else 0 for x in payload], dtype=torch.int64, device=device)
     dist.all_reduce(s, op=dist.ReduceOp.SUM, group=group)
     return out, [int(x) for x in s.tolist()]
+
+
+def plan_pinned_rounds(plan_digit, digits, rank, world, device, group=None):
+    """Plan sub-spaces (one per value of a pinned leading digit) round-robin over the ranks:
+    round r gives digit r*world + rank to this rank.  After every round the ranks MIN-all-
+    reduce their cheapest feasible cost (8 bytes) and the next sub-plan gets it as its cost
+    cap, so every rank's cost bound prunes against the global incumbent.  A cap is always a
+    real feasible candidate's cost, i.e. >= OPT, so each sub-plan still returns its own best
+    candidate among those costing <= the cap, and the global (cost, digit, index) minimum is
+    OPT with the lowest-index tie-break.
+
+    plan_digit(d, cap) -> result with .feasible, .cost, .index, .max_latency_us, .n_decided,
+    .n_full_evals (cap None = no cap).  Returns (best, decided, full_evals, caps) where best
+    = (cost, digit, index, max_latency) of this rank or None and caps = the caps it passed."""
+    best, decided, full_evals, caps = None, 0, 0, []
+    cap_bits = INF_BITS
+    n_rounds = (len(digits) + world - 1) // world
+    for rnd in range(n_rounds):
+        i = rnd * world + rank
+        if i < len(digits):
+            d0 = digits[i]
+            cap = bits_cost(cap_bits) if cap_bits != INF_BITS else None
+            caps.append(cap)
+            r = plan_digit(d0, cap)
+            decided += r.n_decided
+            full_evals += r.n_full_evals
+            if r.feasible and (best is None or (r.cost, d0, r.index) < best[:3]):
+                best = (r.cost, d0, r.index, r.max_latency_us)
+        if best is not None:
+            cap_bits = min(cap_bits, cost_bits(best[0]))
+        if world > 1 and rnd + 1 < n_rounds:
+            t = torch.tensor([cap_bits], dtype=torch.int64, device=device)
+            dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+            cap_bits = int(t.item())
+    return best, decided, full_evals, caps

@@ -133,3 +133,72 @@ def test_sharded_plan_reduces_to_global_opt(world):
     for r in range(world):
         cost, idx, lat, dec = out[r]
         assert (idx, cost, lat) == ref and dec == 4096
+
+
+class _Res:
+    def __init__(self, feasible, cost, index, lat, n):
+        self.feasible, self.cost, self.index, self.max_latency_us = feasible, cost, index, lat
+        self.n_decided, self.n_full_evals = n, n
+
+
+def _pinned_worker(rank, world, port, zero_prices, out_q):
+    """C1 as 16 sub-spaces of function 0's digit (256 candidates each), planned round-robin
+    with the global incumbent as cost cap; a sub-plan is emulated with the library's
+    semantics (lowest (cost, index) among feasible candidates costing <= cap) on the oracle's
+    per-candidate costs."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import workloads as W
+    from oracle import OracleProblem
+    from paper_conf_sc_luxl0y024_b200.dist import plan_pinned_rounds, reduce_lex
+    p = W.make_config("C1", n_arrivals=40)
+    if zero_prices:
+        p = p.replace(price_per_us=np.zeros_like(p.price_per_us))
+    c, l, f = OracleProblem(p).evaluate(np.arange(4096, dtype=np.uint64))
+
+    def plan_digit(d, cap):
+        s = np.arange(256)
+        g = d * 256 + s
+        ok = f[g] & (c[g] <= (np.inf if cap is None else cap))
+        if not ok.any():
+            return _Res(False, float("inf"), None, -1, 256)
+        k = s[ok][np.lexsort((s[ok], c[g][ok]))[0]]
+        return _Res(True, float(c[d * 256 + k]), int(k), int(l[d * 256 + k]), 256)
+
+    best, dec, _, caps = plan_pinned_rounds(plan_digit, list(range(16)), rank, world, "cpu")
+    keys = [cost_bits(best[0]) if best else INF_BITS, best[1] if best else 0, best[2] if best else 0]
+    keys, pay = reduce_lex(keys, [best[3] if best else -1], "cpu")
+    out_q.put((rank, (keys, pay, dec, caps)))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,zero_prices", [(2, False), (3, False), (2, True)])
+def test_pinned_rounds_with_global_cost_cap(world, zero_prices):
+    """bench.py's C5 driver (dist.plan_pinned_rounds): the caps exchanged between rounds are
+    real feasible costs (>= OPT), so the reduced (cost, digit, index) equals the oracle's
+    global OPT, ties included (zero prices: every candidate costs 0, lowest index wins)."""
+    import workloads as W
+    from oracle import OracleProblem
+    p = W.make_config("C1", n_arrivals=40)
+    if zero_prices:
+        p = p.replace(price_per_us=np.zeros_like(p.price_per_us))
+    ref_idx, ref_cost, ref_lat = OracleProblem(p).plan()
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_pinned_worker, args=(r, world, port, zero_prices, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    out = dict(q.get(timeout=180) for _ in range(world))
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    n_caps = 0
+    for r in range(world):
+        keys, pay, dec, caps = out[r]
+        assert bits_cost(keys[0]) == ref_cost and keys[1] * 256 + keys[2] == ref_idx and pay[0] == ref_lat
+        assert all(cp is None or cp >= ref_cost for cp in caps)
+        n_caps += sum(cp is not None for cp in caps)
+    assert n_caps > 0                     # later rounds did run under a cap
