@@ -193,6 +193,8 @@ struct MemoParamsHost {
     int sla;
     int zero;
     int slas[8];
+    u64 *cost_list;                // split cost: units holding a feasible candidate
+    unsigned *cost_n;
     int fixed[SMILESS_MAX_FUNCS];
 };
 
@@ -266,7 +268,7 @@ constexpr int kChunkUnits = 256;     // sharding / claim granularity in units (m
 struct JitKernel {
     CUmodule mod = nullptr;
     CUfunction fn = nullptr;
-    CUfunction fn_bound = nullptr, fn_bound_a = nullptr, fn_up = nullptr, fn_var = nullptr;
+    CUfunction fn_bound = nullptr, fn_bound_a = nullptr, fn_up = nullptr, fn_var = nullptr, fn_varc = nullptr;
     size_t smem_up = 0, smem_var = 0;
     int blocks_up = 0, blocks_var = 0;
     size_t smem = 0, smem_bound = 0;
@@ -332,7 +334,8 @@ struct smiless_ctx {
     DevBuf<i64> dLat;
     DevBuf<unsigned char> dFeas;
     DevBuf<double> dDump;
-    DevBuf<u64> dList, dListA;
+    DevBuf<u64> dList, dListA, dCostList;
+    DevBuf<unsigned> dCostN;
     DevBuf<unsigned> dListCnt, dListCntA, dChunkCnt;
     DevBuf<int> dW;                          // per-row windows of the current plan (padded)
     DevBuf<unsigned char> dX;                // memoised last-function inputs [n_off/4][prefix][4]
@@ -592,6 +595,15 @@ u64 cands_per_prefix(const smiless_ctx *ctx, const smiless_plan_args *a, int d) 
 
 enum { FAM_PLAN = 1, FAM_BOUND = 2, FAM_MEMO = 4, FAM_ALL = 7 };   // kernel families of a module
 
+// Throughput mode with prefix memoisation, SMILESS_SPLITCOST=1: walk every unit without the
+// sum-of-u accumulators and re-walk only the units holding a feasible candidate to finish
+// their costs (DESIGN.md section 5 item 12).  Off by default (measured +3 % candidates/s on
+// the C2 slice, profiles/r01k_sweep_variants.md).
+bool split_cost() {
+    const char *e = getenv("SMILESS_SPLITCOST");
+    return e && atoi(e) != 0;
+}
+
 // static cost-bound terms of every (row, window) staged in shared memory when small
 bool bound_lb_table(const smiless_ctx *ctx, int W) { return (size_t)ctx->sumM * (size_t)W <= 8192; }
 
@@ -632,6 +644,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     // busy mask (measured best once the x stream is prefetched, profiles/r01k_sweep_variants.md)
     const char *sel_env = getenv("SMILESS_SELMASK");
     s << "#define SM_SELMASK " << (sel_env ? atoi(sel_env) : 0) << "\n";
+    s << "#define SM_SPLITCOST " << (split_cost() ? 1 : 0) << "\n";
     const char *vun_env = getenv("SMILESS_VUNROLL");
     s << "#define SM_VUNROLL " << (vun_env ? atoi(vun_env) : 4) << "\n";
     const char *alusul_env = getenv("SMILESS_ALUSUL"), *alug_env = getenv("SMILESS_ALUG");
@@ -860,6 +873,10 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
             if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(upstream)");
             r = driver().moduleGetFunction(&jk.fn_var, jk.mod, "smiless_variants_kernel");
             if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(variants)");
+            if (split_cost()) {
+                r = driver().moduleGetFunction(&jk.fn_varc, jk.mod, "smiless_variants_cost_kernel");
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(variants cost)");
+            }
         }
         if (families & FAM_MEMO) {
             const size_t padI = (size_t)((ctx->sumM + 3) & ~3), padU = (size_t)((ctx->sumM + 1) & ~1);
@@ -874,6 +891,11 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
                 r = driver().funcSetAttribute(jk.fn_var, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
                                               (int)jk.smem_var);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(variants smem)");
+                if (jk.fn_varc) {
+                    r = driver().funcSetAttribute(jk.fn_varc, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
+                                                  (int)jk.smem_var);
+                    if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(variants cost smem)");
+                }
                 r = driver().occupancy(&jk.blocks_up, jk.fn_up, kThreads, jk.smem_up);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(upstream)");
                 r = driver().occupancy(&jk.blocks_var, jk.fn_var, vthreads_per_cta(), jk.smem_var);
@@ -994,6 +1016,7 @@ void smiless_destroy(smiless_ctx *ctx) {
         ctx->dCost.release(); ctx->dLat.release(); ctx->dFeas.release(); ctx->dRes.release(); ctx->dDump.release();
         ctx->dList.release(); ctx->dListCnt.release(); ctx->dW.release();
         ctx->dListA.release(); ctx->dListCntA.release(); ctx->dChunkCnt.release();
+        ctx->dCostList.release(); ctx->dCostN.release();
         ctx->dX.release(); ctx->dRecNx.release(); ctx->dRecNlu.release(); ctx->dRecPre.release();
         if (ctx->hRes) cudaFreeHost(ctx->hRes);
         for (auto &ev : ctx->ev)
@@ -1323,6 +1346,10 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             CK(ctx->dRecNx.ensure((size_t)batch_p), "cudaMalloc");
             CK(ctx->dRecNlu.ensure((size_t)batch_p), "cudaMalloc");
             CK(ctx->dRecPre.ensure((size_t)batch_p), "cudaMalloc");
+            if (jk->fn_varc) {
+                CK(ctx->dCostList.ensure((size_t)(batch_p * upp)), "cudaMalloc cost list");
+                CK(ctx->dCostN.ensure(1), "cudaMalloc");
+            }
             MemoParamsHost mp;
             memset(&mp, 0, sizeof mp);
             mp.tabNI = ctx->dNI.p;
@@ -1338,6 +1365,8 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             mp.rec_nx = ctx->dRecNx.p;
             mp.rec_pre = ctx->dRecPre.p;
             mp.rec_nlu = ctx->dRecNlu.p;
+            mp.cost_list = ctx->dCostList.p;
+            mp.cost_n = ctx->dCostN.p;
             mp.dump = pp.dump;
             mp.cand_begin = cb;
             mp.cand_end = ce;
@@ -1371,10 +1400,18 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "upstream launch");
                 ++launches;
                 CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                if (jk->fn_varc) CK(cudaMemsetAsync(ctx->dCostN.p, 0, sizeof(unsigned), st), "memset cost list");
                 r = driver().launchKernel(jk->fn_var, (unsigned)grid_var, 1, 1, vthreads_per_cta(), 1, 1,
                                           (unsigned)jk->smem_var, (CUstream)st, args, nullptr);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "variants launch");
                 ++launches;
+                if (jk->fn_varc) {                 // split cost: re-walk the units with a feasible candidate
+                    CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                    r = driver().launchKernel(jk->fn_varc, (unsigned)grid_var, 1, 1, vthreads_per_cta(), 1, 1,
+                                              (unsigned)jk->smem_var, (CUstream)st, args, nullptr);
+                    if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "variants cost launch");
+                    ++launches;
+                }
             }
             grid_used = std::max(grid, grid_var);
         } else if (bnb_path && D > 0 && jk->blocks_bound > 0) {

@@ -257,6 +257,21 @@ def test_large_gaps_exercise_clamp_and_int64_path_agree():
 # The bench launch configuration at full size (C2, J = 10^4, 2^28-candidate slice)
 # ---------------------------------------------------------------------------------------
 
+def test_bench_configuration_split_cost_same_result(monkeypatch):
+    """The bench slice at full size with the split-cost throughput path (every unit walked
+    without the sum-of-u accumulators, units with a feasible candidate re-walked for their
+    costs) returns the single-pass winner bit for bit and walks every candidate."""
+    import bench
+    p, kw = bench.workload("C2")
+    pl = S.planner_for(p)
+    one = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=S.FLAG_NO_PRUNE, **kw)
+    monkeypatch.setenv("SMILESS_SPLITCOST", "1")
+    two = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=S.FLAG_NO_PRUNE, **kw)
+    assert (two.index, two.cost, two.max_latency_us) == (one.index, one.cost, one.max_latency_us)
+    assert two.n_full_evals == two.n_decided == one.n_decided
+    assert two.launches > one.launches                  # the cost pass ran
+
+
 def test_bench_configuration_full_size_properties():
     """bench.py's step: C2 at J = 10^4, functions 0/1 pinned, 2^28 candidates, no pruning.
     The oracle cannot walk 2^28 x 10^4 x 6 steps, so we check (a) the winner on the
@@ -665,13 +680,16 @@ def test_throughput_mode_with_and_without_prefix_memoisation(memo, monkeypatch):
     assert n_checked > 20
 
 
-@pytest.mark.parametrize("g,selmask,alu", [("1", "0", "0 0"), ("1", "2", "255 255"), ("2", "255", "42 0"),
-                                            ("4", "6", "0 170")])
-def test_memo_variants_shapes_are_exact(g, selmask, alu, monkeypatch):
+@pytest.mark.parametrize("g,selmask,alu,split", [("1", "0", "0 0", "1"), ("1", "2", "255 255", "0"),
+                                                  ("2", "255", "42 0", "1"), ("4", "6", "0 170", "0"),
+                                                  ("2", "0", "0 0", "1")])
+def test_memo_variants_shapes_are_exact(g, selmask, alu, split, monkeypatch):
     """The variants kernel's tuning knobs (configs per lane G, select vs IMAD.HI busy mask
-    per window variant, adds pinned to the ALU pipe) change only the instruction mix:
-    per-candidate parity with the oracle for each."""
+    per window variant, adds pinned to the ALU pipe, split cost: every unit walked without
+    the sum-of-u accumulators and the units with a feasible candidate re-walked for their
+    costs) change only the instruction mix: per-candidate parity with the oracle for each."""
     monkeypatch.setenv("SMILESS_MEMO", "1")
+    monkeypatch.setenv("SMILESS_SPLITCOST", split)
     monkeypatch.setenv("SMILESS_G", g)
     monkeypatch.setenv("SMILESS_SELMASK", selmask)
     monkeypatch.setenv("SMILESS_ALUG", alu.split()[0])
