@@ -159,19 +159,35 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
     pinned = name == "C5"
     digits = list(range(int(p.n_configs[0]) * Wn)) if pinned else [None]
     warm = dict(n_fixed=1, fixed_digits=[0]) if pinned else {}
+    seed = os.environ.get("SMILESS_SEED_CAP", "0") == "1"
+    seed_w = p.windows_us[:1]                                            # window 0 only: configs-only sub-space
     pl.plan(arr, p.sla_us, p.windows_us, end=1 << 20, **warm)            # NVRTC compile outside the timing
+    if seed:
+        pl.plan(arr, p.sla_us, seed_w, end=1 << 16)
     barrier()
     a = torch.cuda.Event(enable_timing=True)
     b = torch.cuda.Event(enable_timing=True)
     t0 = time.perf_counter()
     a.record(stream)
+    cap0, seed_ms = None, None
+    if seed:
+        # Incumbent from the window-0 sub-space (every window fixed to grid value 0; a subset of the
+        # full space, so its best feasible cost is >= OPT and a valid cost cap: the full plan stays exact)
+        ts = time.perf_counter()
+        rs = pl.plan(arr, p.sla_us, seed_w, shard=rank, n_shards=world)
+        cb = torch.tensor([cost_bits(rs.cost) if rs.feasible else INF_BITS], dtype=torch.int64, device=xdev)
+        if world > 1:
+            dist.all_reduce(cb, op=dist.ReduceOp.MIN)
+        cap0 = bits_cost(int(cb.item())) if int(cb.item()) != INF_BITS else None
+        seed_ms = (time.perf_counter() - ts) * 1e3
     if pinned:
         best, decided, full_evals, _ = plan_pinned_rounds(
             lambda d0, cap: pl.plan(arr, p.sla_us, p.windows_us, n_fixed=1, fixed_digits=[d0],
                                     **({"cost_cap": cap} if cap is not None else {})),
-            digits, rank, world, xdev)
+            digits, rank, world, xdev, initial_cap=cap0)
     else:
-        r = pl.plan(arr, p.sla_us, p.windows_us, shard=rank, n_shards=world)
+        r = pl.plan(arr, p.sla_us, p.windows_us, shard=rank, n_shards=world,
+                    **({"cost_cap": cap0} if cap0 is not None else {}))
         decided, full_evals = r.n_decided, r.n_full_evals
         best = (r.cost, 0, r.index, r.max_latency_us) if r.feasible else None
     keys = [cost_bits(best[0]) if best else INF_BITS, best[1] if best else 0, best[2] if best else 0]
@@ -194,7 +210,8 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
     sec = float(tt.item()) / 1e3
     cost = bits_cost(keys[0])
     out = {"candidates": decided, "time_to_optimal_s": sec, "wall_s": wall, "decided_per_s": decided / sec,
-           "full_evals_local": full_evals, "cost": cost, "max_latency_us": lat if cost is not None else -1}
+           "full_evals_local": full_evals, "cost": cost, "max_latency_us": lat if cost is not None else -1,
+           "seed_cap": {"enabled": seed, "cap": cap0, "wall_ms": seed_ms}}
     if cost is not None:
         kw = dict(n_fixed=1, fixed_digits=[keys[1]]) if pinned else {}
         c, w = pl.decode(keys[2], Wn, **kw)

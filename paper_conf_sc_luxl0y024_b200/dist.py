@@ -93,7 +93,7 @@ def reduce_lex(keys, payload, device, group=None):
     return out, [int(x) for x in s.tolist()]
 
 
-def plan_pinned_rounds(plan_digit, digits, rank, world, device, group=None):
+def plan_pinned_rounds(plan_digit, digits, rank, world, device, group=None, initial_cap=None):
     """Plan sub-spaces (one per value of a pinned leading digit) round-robin over the ranks:
     round r gives digit r*world + rank to this rank.  After every round the ranks MIN-all-
     reduce their cheapest feasible cost (8 bytes) and the next sub-plan gets it as its cost
@@ -104,9 +104,11 @@ def plan_pinned_rounds(plan_digit, digits, rank, world, device, group=None):
 
     plan_digit(d, cap) -> result with .feasible, .cost, .index, .max_latency_us, .n_decided,
     .n_full_evals (cap None = no cap).  Returns (best, decided, full_evals, caps) where best
-    = (cost, digit, index, max_latency) of this rank or None and caps = the caps it passed."""
+    = (cost, digit, index, max_latency) of this rank or None and caps = the caps it passed.
+    initial_cap: the cost of a feasible candidate known beforehand (the same on every rank),
+    or None; it caps the first round too."""
     best, decided, full_evals, caps = None, 0, 0, []
-    cap_bits = INF_BITS
+    cap_bits = cost_bits(initial_cap) if initial_cap is not None else INF_BITS
     n_rounds = (len(digits) + world - 1) // world
     for rnd in range(n_rounds):
         i = rnd * world + rank

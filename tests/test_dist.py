@@ -141,7 +141,7 @@ class _Res:
         self.n_decided, self.n_full_evals = n, n
 
 
-def _pinned_worker(rank, world, port, zero_prices, out_q):
+def _pinned_worker(rank, world, port, zero_prices, out_q, seed=None):
     """C1 as 16 sub-spaces of function 0's digit (256 candidates each), planned round-robin
     with the global incumbent as cost cap; a sub-plan is emulated with the library's
     semantics (lowest (cost, index) among feasible candidates costing <= cap) on the oracle's
@@ -166,7 +166,12 @@ def _pinned_worker(rank, world, port, zero_prices, out_q):
         k = s[ok][np.lexsort((s[ok], c[g][ok]))[0]]
         return _Res(True, float(c[d * 256 + k]), int(k), int(l[d * 256 + k]), 256)
 
-    best, dec, _, caps = plan_pinned_rounds(plan_digit, list(range(16)), rank, world, "cpu")
+    init = None
+    if seed == "opt":                     # a cap equal to OPT: candidates costing exactly the cap stay eligible
+        init = float(c[f].min())
+    elif seed == "max":                   # the loosest real cap: the most expensive feasible candidate
+        init = float(c[f].max())
+    best, dec, _, caps = plan_pinned_rounds(plan_digit, list(range(16)), rank, world, "cpu", initial_cap=init)
     keys = [cost_bits(best[0]) if best else INF_BITS, best[1] if best else 0, best[2] if best else 0]
     keys, pay = reduce_lex(keys, [best[3] if best else -1], "cpu")
     out_q.put((rank, (keys, pay, dec, caps)))
@@ -174,8 +179,9 @@ def _pinned_worker(rank, world, port, zero_prices, out_q):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,zero_prices", [(2, False), (3, False), (2, True)])
-def test_pinned_rounds_with_global_cost_cap(world, zero_prices):
+@pytest.mark.parametrize("world,zero_prices,seed", [(2, False, None), (3, False, None), (2, True, None),
+                                                     (2, False, "opt"), (3, False, "max"), (2, True, "opt")])
+def test_pinned_rounds_with_global_cost_cap(world, zero_prices, seed):
     """bench.py's C5 driver (dist.plan_pinned_rounds): the caps exchanged between rounds are
     real feasible costs (>= OPT), so the reduced (cost, digit, index) equals the oracle's
     global OPT, ties included (zero prices: every candidate costs 0, lowest index wins)."""
@@ -188,7 +194,7 @@ def test_pinned_rounds_with_global_cost_cap(world, zero_prices):
     port = _free_port()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_pinned_worker, args=(r, world, port, zero_prices, q)) for r in range(world)]
+    procs = [ctx.Process(target=_pinned_worker, args=(r, world, port, zero_prices, q, seed)) for r in range(world)]
     for pr in procs:
         pr.start()
     out = dict(q.get(timeout=180) for _ in range(world))
