@@ -824,3 +824,23 @@ def test_exact_evaluator_wide_dags():
         b = int(rng.integers(0, space - 4096))
         g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, begin=b, end=b + 4096)
         assert_same_plan(g, o.plan(begin=b, end=b + 4096), o)
+
+
+@pytest.mark.parametrize("name", ["C2", "C3"])
+def test_bench_full_space_seed_cap_same_opt(monkeypatch, name):
+    """bench.full_space_opt with the window-0 seed cap (SMILESS_SEED_CAP=1: the best cost of
+    the window-0 sub-space caps the whole-space plan) returns the uncapped run's OPT, and the
+    winner re-checks on the oracle bit for bit (DESIGN.md §11 item 3)."""
+    import torch
+    import bench
+    dev = torch.device("cuda:0")
+    stream = torch.cuda.current_stream(dev)
+    outs = {}
+    for seed in ("0", "1"):
+        monkeypatch.setenv("SMILESS_SEED_CAP", seed)
+        outs[seed] = bench.full_space_opt(name, S, 0, 1, dev, dev, stream, 0, lambda: None)
+    a, b = outs["0"], outs["1"]
+    assert b["seed_cap"]["enabled"] and not a["seed_cap"]["enabled"]
+    assert b["seed_cap"]["cap"] is not None and b["seed_cap"]["cap"] >= a["cost"]
+    assert (b["cost"], b["index"], b["max_latency_us"]) == (a["cost"], a["index"], a["max_latency_us"])
+    assert b["oracle_check"] == {"feasible": True, "cost_bits_equal": True, "latency_equal": True}
