@@ -151,7 +151,9 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
     reduced lexicographically on (cost bits, digit, index) across ranks."""
     import torch
     import torch.distributed as dist
-    from paper_conf_sc_luxl0y024_b200.dist import cost_bits, bits_cost, reduce_lex, plan_pinned_rounds, INF_BITS
+    from paper_conf_sc_luxl0y024_b200.dist import (cost_bits, bits_cost, reduce_lex, plan_pinned_rounds,
+                                                   plan_range_rounds, INF_BITS)
+    rounds = int(os.environ.get("SMILESS_BENCH_ROUNDS", "1" if world == 1 else "2"))
     p = W.make_config(name)
     Wn = len(p.windows_us)
     pl = S.planner_for(p, device=local, stream=stream.cuda_stream)
@@ -186,10 +188,15 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
                                     **({"cost_cap": cap} if cap is not None else {})),
             digits, rank, world, xdev, initial_cap=cap0)
     else:
-        r = pl.plan(arr, p.sla_us, p.windows_us, shard=rank, n_shards=world,
-                    **({"cost_cap": cap0} if cap0 is not None else {}))
-        decided, full_evals = r.n_decided, r.n_full_evals
-        best = (r.cost, 0, r.index, r.max_latency_us) if r.feasible else None
+        # one exact plan, every rank on its interleaved share of every B&B survivor's subtree;
+        # with N > 1 the index range runs in `rounds` pieces and the ranks exchange the
+        # incumbent cost between them (dist.plan_range_rounds; exact for any cap >= OPT)
+        rb, decided, full_evals, _ = plan_range_rounds(
+            lambda b0, b1, cap: pl.plan(arr, p.sla_us, p.windows_us, begin=b0, end=b1, shard=rank, n_shards=world,
+                                        **({"cost_cap": cap} if cap is not None else {})),
+            p.space_size(), rounds, rank, world, xdev, initial_cap=cap0)
+        best = (rb[0], 0, rb[1], rb[2]) if rb is not None else None
+    local_decided = decided
     keys = [cost_bits(best[0]) if best else INF_BITS, best[1] if best else 0, best[2] if best else 0]
     payload = [best[3] if best else -1]
     if world > 1:
@@ -199,8 +206,16 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
         dist.all_reduce(hi_lo)
         decided = (int(hi_lo[0].item()) << 32) + int(hi_lo[1].item())
         lat = pay[0]
+        # every rank's share (balanced under pruning), as hi/lo int64 halves
+        mine = torch.tensor([local_decided >> 32, local_decided & 0xffffffff, full_evals], dtype=torch.int64,
+                            device=xdev)
+        allv = [torch.zeros_like(mine) for _ in range(world)]
+        dist.all_gather(allv, mine)
+        per_rank = [(int(v[0].item()) << 32) + int(v[1].item()) for v in allv]
+        per_rank_full = [int(v[2].item()) for v in allv]
     else:
         lat = payload[0]
+        per_rank, per_rank_full = [local_decided], [full_evals]
     b.record(stream)
     torch.cuda.synchronize(dev)
     wall = time.perf_counter() - t0
@@ -210,7 +225,9 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
     sec = float(tt.item()) / 1e3
     cost = bits_cost(keys[0])
     out = {"candidates": decided, "time_to_optimal_s": sec, "wall_s": wall, "decided_per_s": decided / sec,
-           "full_evals_local": full_evals, "cost": cost, "max_latency_us": lat if cost is not None else -1,
+           "full_evals_local": full_evals, "decided_per_rank": per_rank, "full_evals_per_rank": per_rank_full,
+           "rounds": 1 if pinned else rounds,
+           "cost": cost, "max_latency_us": lat if cost is not None else -1,
            "seed_cap": {"enabled": seed, "cap": cap0, "wall_ms": seed_ms}}
     if cost is not None:
         kw = dict(n_fixed=1, fixed_digits=[keys[1]]) if pinned else {}

@@ -27,6 +27,7 @@
 #include <vector>
 
 #include "kernels.h"
+#include <nvtx3/nvToolsExt.h>
 
 extern "C" const char smiless_evaluator_src[];  // generated from evaluator.cuh at build time
 
@@ -167,6 +168,7 @@ struct PlanParamsHost {
     u64 cap;                       // cost cap bits (~0: none)
     int cost_prune;
     int pad0;
+    u64 list_in_cap;               // list mode: entries list_in holds (clamps *list_n)
     int fixed[SMILESS_MAX_FUNCS];  // evaluator uses SM_NFIXED_ALLOC <= SMILESS_MAX_FUNCS; extra tail is ignored
 };
 
@@ -226,6 +228,11 @@ struct BoundParamsHost {
     u64 *inc;                      // incumbent cost bits shared with the evaluator
     int cost_prune;
     int pad0;
+    u64 list_stride, list_r0;      // list mode: prefix = list_in[c / upp] * stride + r0 + c % upp
+    u64 list_cap;                  // capacity of list_out
+    unsigned *overflow;            // set to 1 if a launch would exceed list_cap (never, by sizing)
+    int shard, n_shards;           // ordinals c = c' * n_shards + shard of the launch
+    int attr_shard, attr_n;        // replicated level: decided counted for c % attr_n == attr_shard
     int fixed[SMILESS_MAX_FUNCS];
 };
 
@@ -423,14 +430,20 @@ int upload_tables(smiless_ctx *ctx) {
     CK(ctx->dU.ensure(padU), "cudaMalloc");
     CK(ctx->dPtr.ensure(ctx->pred_ptr.size()), "cudaMalloc");
     CK(ctx->dIdx.ensure(std::max<size_t>(ctx->pred_idx.size(), 1)), "cudaMalloc");
-    CK(cudaMemcpy(ctx->dI.p, I.data(), padI * sizeof(int), cudaMemcpyHostToDevice), "H2D tables");
-    CK(cudaMemcpy(ctx->dNI.p, NI.data(), padI * sizeof(int), cudaMemcpyHostToDevice), "H2D tables");
-    CK(cudaMemcpy(ctx->dT.p, T.data(), padI * sizeof(int), cudaMemcpyHostToDevice), "H2D tables");
-    CK(cudaMemcpy(ctx->dU.p, U.data(), padU * sizeof(double), cudaMemcpyHostToDevice), "H2D tables");
-    CK(cudaMemcpy(ctx->dPtr.p, ctx->pred_ptr.data(), ctx->pred_ptr.size() * sizeof(int), cudaMemcpyHostToDevice),
+    // stream-ordered uploads: the kernels that read them run on ctx->stream, which may be a
+    // non-blocking stream (not ordered after the legacy default stream).  The pageable
+    // sources are staged before cudaMemcpyAsync returns, so the local vectors may go.
+    cudaStream_t st = ctx->stream;
+    CK(cudaMemcpyAsync(ctx->dI.p, I.data(), padI * sizeof(int), cudaMemcpyHostToDevice, st), "H2D tables");
+    CK(cudaMemcpyAsync(ctx->dNI.p, NI.data(), padI * sizeof(int), cudaMemcpyHostToDevice, st), "H2D tables");
+    CK(cudaMemcpyAsync(ctx->dT.p, T.data(), padI * sizeof(int), cudaMemcpyHostToDevice, st), "H2D tables");
+    CK(cudaMemcpyAsync(ctx->dU.p, U.data(), padU * sizeof(double), cudaMemcpyHostToDevice, st), "H2D tables");
+    CK(cudaMemcpyAsync(ctx->dPtr.p, ctx->pred_ptr.data(), ctx->pred_ptr.size() * sizeof(int), cudaMemcpyHostToDevice,
+                       st),
        "H2D dag");
     if (!ctx->pred_idx.empty())
-        CK(cudaMemcpy(ctx->dIdx.p, ctx->pred_idx.data(), ctx->pred_idx.size() * sizeof(int), cudaMemcpyHostToDevice),
+        CK(cudaMemcpyAsync(ctx->dIdx.p, ctx->pred_idx.data(), ctx->pred_idx.size() * sizeof(int),
+                           cudaMemcpyHostToDevice, st),
            "H2D dag");
     ctx->tables_dirty = false;
     return SMILESS_OK;
@@ -951,7 +964,7 @@ int stage_row_windows(smiless_ctx *ctx, const smiless_plan_args *a) {
     if (a->row_windows_us) std::copy(a->row_windows_us, a->row_windows_us + ctx->sumM, w.begin());
     if (ctx->dW.p && ctx->dW.n >= padI && w == ctx->hW && !ctx->tables_dirty) return SMILESS_OK;  // unchanged
     CK(ctx->dW.ensure(padI), "cudaMalloc row windows");
-    CK(cudaMemcpy(ctx->dW.p, w.data(), padI * sizeof(int), cudaMemcpyHostToDevice), "H2D windows");
+    CK(cudaMemcpyAsync(ctx->dW.p, w.data(), padI * sizeof(int), cudaMemcpyHostToDevice, ctx->stream), "H2D windows");
     ctx->hW.swap(w);
     return SMILESS_OK;
 }
@@ -1084,8 +1097,10 @@ int smiless_load_profiles(smiless_ctx *ctx, const int32_t *n_configs, const int3
     for (int r = 0; r < sum; ++r) {
         if (exec_us[r] < 0 || exec_us[r] >= (1 << 29)) return fail(ctx, SMILESS_EINVAL, "exec_us[%d] out of [0, 2^29)", r);
         if (init_us[r] < 0 || init_us[r] >= (1 << 29)) return fail(ctx, SMILESS_EINVAL, "init_us[%d] out of [0, 2^29)", r);
-        if (!std::isfinite(price_per_us[r]) || price_per_us[r] < 0)
-            return fail(ctx, SMILESS_EINVAL, "price_per_us[%d] must be finite and >= 0", r);
+        // -0.0 is rejected too: the kernels take the first cost term as is, so its sign bit
+        // would make the cost bits order wrongly against the oracle's 0.0 + term
+        if (!std::isfinite(price_per_us[r]) || price_per_us[r] < 0 || std::signbit(price_per_us[r]))
+            return fail(ctx, SMILESS_EINVAL, "price_per_us[%d] must be finite and >= +0.0", r);
         tmax = std::max<i64>(tmax, init_us[r]);
         imax = std::max<i64>(imax, exec_us[r]);
     }
@@ -1182,6 +1197,15 @@ int smiless_evaluate(smiless_ctx *ctx, const smiless_plan_args *a, const uint64_
 
 namespace {
 
+// NVTX range for the profilers (nsys / ncu --nvtx): the stages of a plan call (header-only
+// nvtx3; a no-op unless a tool injects itself)
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange &) = delete;
+    NvtxRange &operator=(const NvtxRange &) = delete;
+};
+
 // SMILESS_PROFILE_HOST=1: host-side stage timestamps of every plan call on stderr (tuning aid)
 struct HostProf {
     bool on;
@@ -1212,6 +1236,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
               int32_t *config_out, int32_t *window_out) {
     if (!a_in) return fail(ctx, SMILESS_EINVAL, "args is NULL");
     HostProf hp;
+    NvtxRange nv_plan("smiless_plan");
     smiless_plan_args a_copy = *a_in;
     i64 sla_max = slas[0];
     for (int s_ = 1; s_ < n_sla; ++s_) sla_max = std::max<i64>(sla_max, slas[s_]);
@@ -1271,7 +1296,10 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         const int families = memo_path ? (FAM_MEMO | FAM_PLAN) : (bnb_path ? (FAM_PLAN | FAM_BOUND) : FAM_PLAN);
         hp.mark("setup");
         JitKernel *jk = nullptr;
-        if ((rc = get_kernel(ctx, a, rp, n_off, families, &jk))) return rc;
+        {
+            NvtxRange nv("nvrtc specialisation (cached)");
+            if ((rc = get_kernel(ctx, a, rp, n_off, families, &jk))) return rc;
+        }
         hp.mark("get_kernel");
         const u64 V = (u64)a->n_windows * (u64)configs_per_lane(ctx, a);   // candidates per unit
         const u64 ub = cb / V, ue = (ce + V - 1) / V;
@@ -1385,6 +1413,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 mp.blk_best = ctx->dBlk.p;
             }
             CK(cudaEventRecord(ctx->ev[1], st), "event");
+            NvtxRange nv("memo: upstream + variants batches");
             u64 bi = 0;
             for (u64 b0 = pl0; b0 < ph0; b0 += batch_p, ++bi) {
                 if (bi % (u64)n_shards != (u64)shard) continue;
@@ -1416,12 +1445,24 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             grid_used = std::max(grid, grid_var);
         } else if (bnb_path && D > 0 && jk->blocks_bound > 0) {
             // ---- exact branch-and-bound: prefixes of functions n_fixed..D-1, then list mode ----
+            // Sharding (multi-GPU): the deep level's prefixes (one level) or the deep children of
+            // every shallow survivor (two levels) are interleaved over the shards, ordinal
+            // c = c' * n_shards + shard, so every rank decides an equal share of every survivor's
+            // subtree; the shallow level (<= 2^22 prefixes) is replicated on every rank.
             const u64 S = cands_per_prefix(ctx, a, D);
             const u64 upp = S / V;                            // evaluator units per prefix
             const u64 p_lo = cb / S, p_hi = (ce + S - 1) / S;
-            const u64 batch = (u64)1 << 22;                   // prefixes per bound launch
-            CK(ctx->dList.ensure((size_t)batch), "cudaMalloc list");
+            const u64 batch = (u64)1 << 22;                   // prefixes per range-mode bound launch
+            const int DA = bb_depth_a(ctx, a, D);
+            const u64 R = DA > 0 ? cands_per_prefix(ctx, a, DA) / S : 1;   // deep children per shallow prefix
+            // deep survivor list: no launch enumerates more than list_cap ordinals, so it cannot
+            // overflow (the kernel still checks, and a violation fails the call)
+            u64 list_cap = R > ((u64)1 << 24) ? ((u64)1 << 26) : ((u64)1 << 24);
+            if (const char *lc_env = getenv("SMILESS_BB_LISTCAP"))   // testing: force the split paths
+                list_cap = std::max<u64>(1, std::min<u64>(list_cap, (u64)atoll(lc_env)));
+            CK(ctx->dList.ensure((size_t)list_cap), "cudaMalloc list");
             CK(ctx->dListCnt.ensure(1), "cudaMalloc");
+            pp.list_in_cap = list_cap;
             BoundParamsHost bp;
             memset(&bp, 0, sizeof bp);
             bp.tabNI = ctx->dNI.p;
@@ -1436,6 +1477,8 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             bp.stats = ctx->dStats.p;
             bp.list_out = ctx->dList.p;
             bp.list_cnt = ctx->dListCnt.p;
+            bp.list_cap = list_cap;
+            bp.overflow = (unsigned *)ctx->dErr.p;            // bit 2 (value 4): list overflow
             bp.cands_per_prefix = S;
             bp.cand_begin = cb;
             bp.cand_end = ce;
@@ -1444,6 +1487,10 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             bp.sumM = ctx->sumM;
             bp.sla = (int)a->sla_us;
             bp.zero = 0;
+            bp.shard = shard;
+            bp.n_shards = n_shards;
+            bp.attr_shard = 0;
+            bp.attr_n = 1;
             for (int k = 0; k < ctx->N; ++k) {
                 int m = ctx->I[ctx->row0[k]];
                 for (int c = 1; c < ctx->M[k]; ++c) m = std::min(m, ctx->I[ctx->row0[k] + c]);
@@ -1479,63 +1526,82 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 ++launches;
                 return SMILESS_OK;
             };
-            const int DA = bb_depth_a(ctx, a, D);
             if (DA > 0) {
                 // ---- two levels: depth DA over every prefix, depth D over the DA survivors' children --
                 const u64 SA = cands_per_prefix(ctx, a, DA);
-                const u64 R = SA / S;                             // depth-D children per depth-DA prefix
                 const u64 a_lo = cb / SA, a_hi = (ce + SA - 1) / SA;
                 CK(ctx->dListA.ensure((size_t)batch), "cudaMalloc list");
                 CK(ctx->dListCntA.ensure(1), "cudaMalloc");
-                const u64 per_chunk = std::max<u64>(1, batch / R);   // shallow survivors per deep launch
-                u64 bi = 0;
-                for (u64 b0 = a_lo; b0 < a_hi; b0 += batch, ++bi) {
-                    if (bi % (u64)n_shards != (u64)shard) continue;
+                for (u64 b0 = a_lo; b0 < a_hi; b0 += batch) {
                     const u64 b1 = std::min(a_hi, b0 + batch);
                     CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
                     CK(cudaMemsetAsync(ctx->dListCntA.p, 0, sizeof(unsigned), st), "memset list");
                     bp.list_in = nullptr;
                     bp.list_n = nullptr;
                     bp.list_upp = 1;
+                    bp.list_stride = 1;
+                    bp.list_r0 = 0;
                     bp.prefix_begin = b0;
                     bp.prefix_end = b1;
                     bp.cands_per_prefix = SA;
                     bp.list_out = ctx->dListA.p;
                     bp.list_cnt = ctx->dListCntA.p;
-                    if ((rc = run_bound(jk->fn_bound_a))) return rc;
+                    bp.list_cap = batch;
+                    bp.shard = 0;                                 // replicated on every shard ...
+                    bp.n_shards = 1;
+                    bp.attr_shard = shard;                        // ... its pruned prefixes counted once
+                    bp.attr_n = n_shards;
+                    {
+                        NvtxRange nv("bnb shallow level");
+                        if ((rc = run_bound(jk->fn_bound_a))) return rc;
+                    }
                     unsigned n_a = 0;
                     hp.mark("launch_a");
                     CK(cudaMemcpyAsync(&n_a, ctx->dListCntA.p, sizeof n_a, cudaMemcpyDeviceToHost, st), "D2H count");
                     CK(cudaStreamSynchronize(st), "count");
                     hp.mark("sync_a");
-                    // per-chunk entry counts, uploaded once (no host sync inside the loop).  With the
-                    // cost bound on, the first chunk is small: its evaluation sets the incumbent the
-                    // static prefix bound of every later chunk prunes against.
-                    const char *first_env = getenv("SMILESS_BB_FIRST");
-                    const u64 first = std::max<u64>(1, std::min<u64>(per_chunk, pp.cost_prune ? (first_env ? (u64)atoll(first_env) : 64)
-                                                                                             : per_chunk));
-                    std::vector<unsigned> cnts;
-                    std::vector<u64> starts;
-                    for (u64 c0 = 0; c0 < n_a;) {
-                        const u64 len = std::min<u64>(c0 == 0 ? first : per_chunk, n_a - c0);
-                        starts.push_back(c0);
-                        cnts.push_back((unsigned)len);
-                        c0 += len;
+                    // deep launches (first survivor entry, entries, first child, children per entry):
+                    // at most list_cap ordinals each.  With the cost bound on, the first launch is small:
+                    // its evaluation sets the incumbent the static prefix bound of every later launch
+                    // prunes against.
+                    struct DeepLaunch { u64 e0; unsigned ne; u64 r0, span; };
+                    std::vector<DeepLaunch> L;
+                    if (R <= list_cap) {
+                        const u64 per_chunk = list_cap / R;
+                        const char *first_env = getenv("SMILESS_BB_FIRST");
+                        const u64 first = std::max<u64>(
+                            1, std::min<u64>(per_chunk, pp.cost_prune ? (first_env ? (u64)atoll(first_env) : 64) : per_chunk));
+                        for (u64 c0 = 0; c0 < n_a;) {
+                            const u64 len = std::min<u64>(c0 == 0 ? first : per_chunk, n_a - c0);
+                            L.push_back({c0, (unsigned)len, 0, R});
+                            c0 += len;
+                        }
+                    } else {                                      // a survivor's children over several launches
+                        for (u64 e = 0; e < n_a; ++e)
+                            for (u64 r0 = 0; r0 < R; r0 += list_cap) L.push_back({e, 1u, r0, std::min(list_cap, R - r0)});
                     }
-                    const u64 n_chunks_a = cnts.size();
-                    if (cnts.empty()) cnts.push_back(0);
+                    std::vector<unsigned> cnts(std::max<size_t>(L.size(), 1), 0u);
+                    for (size_t i = 0; i < L.size(); ++i) cnts[i] = L[i].ne;
                     CK(ctx->dChunkCnt.ensure(cnts.size()), "cudaMalloc counts");
-                    CK(cudaMemcpy(ctx->dChunkCnt.p, cnts.data(), cnts.size() * sizeof(unsigned), cudaMemcpyHostToDevice),
+                    CK(cudaMemcpyAsync(ctx->dChunkCnt.p, cnts.data(), cnts.size() * sizeof(unsigned),
+                                       cudaMemcpyHostToDevice, st),
                        "H2D counts");
-                    for (u64 i = 0; i < n_chunks_a; ++i) {
-                        const u64 c0 = starts[i];
+                    bp.list_cap = list_cap;
+                    bp.shard = shard;
+                    bp.n_shards = n_shards;
+                    bp.attr_shard = 0;
+                    bp.attr_n = 1;
+                    NvtxRange nv("bnb deep level + evaluate");
+                    for (size_t i = 0; i < L.size(); ++i) {
                         CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
                         CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
-                        bp.list_in = ctx->dListA.p + c0;
+                        bp.list_in = ctx->dListA.p + L[i].e0;
                         bp.list_n = ctx->dChunkCnt.p + i;
-                        bp.list_upp = R;
+                        bp.list_upp = L[i].span;
+                        bp.list_stride = R;
+                        bp.list_r0 = L[i].r0;
                         bp.prefix_begin = 0;
-                        bp.prefix_end = ~0ull;
+                        bp.prefix_end = 0;
                         bp.cands_per_prefix = S;
                         bp.list_out = ctx->dList.p;
                         bp.list_cnt = ctx->dListCnt.p;
@@ -1543,16 +1609,20 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                         if ((rc = run_eval())) return rc;
                     }
                     hp.mark("chunks_launched");
-                    CK(cudaStreamSynchronize(st), "chunks");      // cnts must outlive its uploads
+                    CK(cudaStreamSynchronize(st), "chunks");      // the next batch reuses dListA
                     hp.mark("sync_chunks");
                 }
             } else {
-                u64 bi = 0;
-                for (u64 b0 = p_lo; b0 < p_hi; b0 += batch, ++bi) {
-                    if (bi % (u64)n_shards != (u64)shard) continue;
+                NvtxRange nv("bnb level + evaluate");
+                for (u64 b0 = p_lo; b0 < p_hi; b0 += batch) {
                     const u64 b1 = std::min(p_hi, b0 + batch);
                     CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
                     CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
+                    bp.list_in = nullptr;
+                    bp.list_n = nullptr;
+                    bp.list_upp = 1;
+                    bp.list_stride = 1;
+                    bp.list_r0 = 0;
                     bp.prefix_begin = b0;
                     bp.prefix_end = b1;
                     if ((rc = run_bound(jk->fn_bound))) return rc;
@@ -1573,6 +1643,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 CK(ctx->dListCnt.ensure(1), "cudaMalloc");
             }
             CK(cudaEventRecord(ctx->ev[1], st), "event");
+            NvtxRange nv("evaluate");
             for (u64 q0 = 0; q0 < claims_total; q0 += claims_per_launch) {
                 const u64 q1 = std::min(claims_total, q0 + claims_per_launch);
                 CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
@@ -1588,6 +1659,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                     pp.list_out = ctx->dList.p;
                     pp.list_cnt = ctx->dListCnt.p;
                     pp.list_base = ub + (q0 / kChunkUnits * (u64)n_shards + (u64)shard) * kChunkUnits;
+                    pp.list_in_cap = claims_per_launch;
                     pp.horizon = horizon;
                 }
                 void *args[] = {&pp};
@@ -1612,6 +1684,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             }
         }
         CK(cudaEventRecord(ctx->ev[2], st), "event");
+        NvtxRange nv("argmin reduce");
         for (int s_ = 0; s_ < n_sla; ++s_) {
             e = smiless_dev_reduce_best(ctx->dBlk.p + 2 * s_, grid_used, n_sla, ctx->dRes.p + s_, st);
             if (e) return cuda_fail(ctx, (cudaError_t)e, "reduce launch");
@@ -1632,6 +1705,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     }
     // a10: exact int64 re-evaluation of each winner (also decodes its digits), one thread per SLA
     {
+        NvtxRange nv("exact winner re-check");
         ExactParams ep;
         fill_exact_params(ctx, a, d_arr, ep);
         for (int s_ = 0; s_ < n_sla; ++s_) ep.slas[s_] = slas[s_];
@@ -1656,6 +1730,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     const ResBlock &h0 = *ctx->hRes;
     if (h0.err & 1) return fail(ctx, SMILESS_EINVAL, "arrivals must be non-decreasing");
     if (h0.err & 2) return fail(ctx, SMILESS_EINVAL, "arrival times out of range (|r| >= 2^62)");
+    if (h0.err & 4) return fail(ctx, SMILESS_ECUDA, "internal: branch-and-bound survivor list overflow");
     if (!single && ce > cb) {
         n_decided = h0.stats[0];
         n_full = h0.stats[1];

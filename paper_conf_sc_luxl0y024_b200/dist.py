@@ -128,3 +128,37 @@ def plan_pinned_rounds(plan_digit, digits, rank, world, device, group=None, init
             dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
             cap_bits = int(t.item())
     return best, decided, full_evals, caps
+
+
+def plan_range_rounds(plan_range, space, rounds, rank, world, device, group=None, initial_cap=None):
+    """One exact plan of [0, space) split into `rounds` contiguous index ranges, each planned
+    by every rank on its interleaved shard (plan_range(begin, end, cap) calls smiless_plan with
+    shard=rank, n_shards=world).  After every round the ranks MIN-all-reduce their cheapest
+    feasible cost bits and the next round gets it as its cost cap, so each GPU's cost bound
+    prunes against the global incumbent inside the plan (SURVEY 8(e) collective (1)).  A cap
+    is always a real feasible candidate's cost, i.e. >= OPT, so every round still returns its
+    best candidate among those costing <= the cap, and the lexicographic (cost, index) minimum
+    over rounds and ranks is OPT with the lowest-index tie-break.
+
+    Returns (best, decided, full_evals, caps): best = (cost, index, max_latency) of this rank
+    or None; caps = the caps this rank passed (None = no cap)."""
+    best, decided, full_evals, caps = None, 0, 0, []
+    cap_bits = cost_bits(initial_cap) if initial_cap is not None else INF_BITS
+    rounds = max(1, min(int(rounds), int(space)))
+    for rnd in range(rounds):
+        b0 = space * rnd // rounds
+        b1 = space * (rnd + 1) // rounds
+        cap = bits_cost(cap_bits) if cap_bits != INF_BITS else None
+        caps.append(cap)
+        r = plan_range(b0, b1, cap)
+        decided += r.n_decided
+        full_evals += r.n_full_evals
+        if r.feasible and (best is None or (r.cost, r.index) < best[:2]):
+            best = (r.cost, r.index, r.max_latency_us)
+        if best is not None:
+            cap_bits = min(cap_bits, cost_bits(best[0]))
+        if world > 1 and rnd + 1 < rounds:
+            t = torch.tensor([cap_bits], dtype=torch.int64, device=device)
+            dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+            cap_bits = int(t.item())
+    return best, decided, full_evals, caps

@@ -208,3 +208,69 @@ def test_pinned_rounds_with_global_cost_cap(world, zero_prices, seed):
         assert all(cp is None or cp >= ref_cost for cp in caps)
         n_caps += sum(cp is not None for cp in caps)
     assert n_caps > 0                     # later rounds did run under a cap
+
+
+def _range_rounds_worker(rank, world, port, rounds, zero_prices, out_q):
+    """One exact plan of C1's 4096 candidates split into `rounds` index ranges; in each round
+    every rank plans its interleaved shard (emulated with the library's semantics on the
+    oracle's per-candidate costs: lowest (cost, index) among the shard's feasible candidates
+    costing <= cap) and the ranks exchange the incumbent before the next round."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import workloads as W
+    from oracle import OracleProblem
+    from paper_conf_sc_luxl0y024_b200.dist import plan_range_rounds, reduce_lex
+    p = W.make_config("C1", n_arrivals=40)
+    if zero_prices:
+        p = p.replace(price_per_us=np.zeros_like(p.price_per_us))
+    c, l, f = OracleProblem(p).evaluate(np.arange(4096, dtype=np.uint64))
+
+    def plan_range(b0, b1, cap):
+        g = np.arange(b0, b1)
+        g = g[g % world == rank]                       # this rank's interleaved share
+        ok = f[g] & (c[g] <= (np.inf if cap is None else cap))
+        if not ok.any():
+            return _Res(False, float("inf"), None, -1, len(g))
+        k = g[ok][np.lexsort((g[ok], c[g][ok]))[0]]
+        return _Res(True, float(c[k]), int(k), int(l[k]), len(g))
+
+    best, dec, _, caps = plan_range_rounds(plan_range, 4096, rounds, rank, world, "cpu")
+    keys = [cost_bits(best[0]) if best else INF_BITS, best[1] if best else 0]
+    keys, pay = reduce_lex(keys, [best[2] if best else -1, dec], "cpu")
+    out_q.put((rank, (keys, pay, dec, caps)))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,rounds,zero_prices", [(2, 4, False), (3, 3, False), (2, 5, True), (3, 1, False)])
+def test_range_rounds_with_in_plan_incumbent_exchange(world, rounds, zero_prices):
+    """dist.plan_range_rounds (the exact full-space plans of C2/C3 on N GPUs): every rank
+    decides its share of every round, the caps passed are real feasible costs (>= OPT), and
+    the reduced (cost, index) is the oracle's OPT with the lowest-index tie-break."""
+    import workloads as W
+    from oracle import OracleProblem
+    p = W.make_config("C1", n_arrivals=40)
+    if zero_prices:
+        p = p.replace(price_per_us=np.zeros_like(p.price_per_us))
+    ref_idx, ref_cost, ref_lat = OracleProblem(p).plan()
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_range_rounds_worker, args=(r, world, port, rounds, zero_prices, q))
+             for r in range(world)]
+    for pr in procs:
+        pr.start()
+    out = dict(q.get(timeout=180) for _ in range(world))
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    total = sum(out[r][2] for r in range(world))
+    assert total == 4096
+    for r in range(world):
+        keys, pay, dec, caps = out[r]
+        assert dec >= 4096 // (2 * world)
+        assert bits_cost(keys[0]) == ref_cost and keys[1] == ref_idx and pay[0] == ref_lat
+        assert len(caps) == rounds and all(cp is None or cp >= ref_cost for cp in caps)
+        if rounds > 1:
+            assert caps[-1] is not None       # the global incumbent reached every rank's last round

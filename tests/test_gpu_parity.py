@@ -844,3 +844,102 @@ def test_bench_full_space_seed_cap_same_opt(monkeypatch, name):
     assert b["seed_cap"]["cap"] is not None and b["seed_cap"]["cap"] >= a["cost"]
     assert (b["cost"], b["index"], b["max_latency_us"]) == (a["cost"], a["index"], a["max_latency_us"])
     assert b["oracle_check"] == {"feasible": True, "cost_bits_equal": True, "latency_equal": True}
+
+
+# ---------------------------------------------------------------------------------------
+# Multi-GPU sharding of the exact pruned plans: interleaved deep B&B work
+# ---------------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("listcap", ["0", "1", "5"])
+def test_branch_and_bound_shards_and_list_splits_are_exact(listcap, monkeypatch):
+    """Every (D, DA) pair, 2 and 3 shards, and a forced small survivor-list capacity (a
+    shallow survivor's children then span several deep launches): the shards' merged
+    per-candidate costs equal the oracle's, each candidate is decided by exactly one shard,
+    and the best shard winner is the oracle's OPT."""
+    if listcap != "0":
+        monkeypatch.setenv("SMILESS_BB_LISTCAP", listcap)
+    rng = np.random.default_rng(61 + int(listcap))
+    n_checked = 0
+    for t in range(40):
+        if n_checked == 6:
+            break
+        n = int(rng.integers(4, 7))
+        p = W.random_problem(rng, n, 3, int(rng.integers(2, 4)), int(rng.integers(20, 120)),
+                             sla_us=int(rng.integers(15_000, 60_000)))
+        space = p.space_size()
+        if space > 30000:
+            continue
+        o = OracleProblem(p)
+        oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
+        ref = o.plan()
+        for d in range(2, n):
+            for da in [0] + list(range(1, d)):
+                monkeypatch.setenv("SMILESS_BB_DEPTH", str(d))
+                monkeypatch.setenv("SMILESS_BB_DEPTH_A", str(da))
+                pl = S.planner_for(p)
+                for world in (2, 3):
+                    merged = np.full(space, np.nan)
+                    parts = []
+                    for s_ in range(world):
+                        out = np.empty(space)
+                        parts.append(pl.plan(p.arrivals_us, p.sla_us, p.windows_us, shard=s_, n_shards=world,
+                                             cost_out=out))
+                        hit = ~np.isnan(out)
+                        assert np.isnan(merged[hit]).all()          # no candidate evaluated twice
+                        merged[hit] = out[hit]
+                    assert_dump_matches(merged, oc, of)
+                    assert sum(r.n_decided for r in parts) == space
+                    win = [(r.cost, r.index) for r in parts if r.feasible]
+                    if ref is None:
+                        assert not win
+                    else:
+                        assert min(win) == (ref[1], ref[0])
+                    # with the cost bound (no dump): same OPT
+                    parts = [pl.plan(p.arrivals_us, p.sla_us, p.windows_us, shard=s_, n_shards=world)
+                             for s_ in range(world)]
+                    assert sum(r.n_decided for r in parts) == space
+                    win = [(r.cost, r.index) for r in parts if r.feasible]
+                    assert (min(win) if win else None) == (None if ref is None else (ref[1], ref[0]))
+        n_checked += 1
+    assert n_checked >= 4
+
+
+@pytest.mark.parametrize("name,world", [("C2", 2), ("C3", 2), ("C2", 4), ("C3", 3)])
+def test_full_space_plan_shards_split_the_work(name, world):
+    """The exact full-space plans of C2 (2^42) and C3 (7.2e15) sharded over `world` ranks
+    (run one after the other on this GPU): every rank decides at least space / (2 world)
+    candidates and walks some to J, the shares sum to the space, and the best rank winner
+    is the single-rank OPT (which the oracle re-checks)."""
+    import torch
+    p = W.make_config(name)
+    pl = S.planner_for(p)
+    arr = torch.as_tensor(p.arrivals_us).cuda()
+    one = pl.plan(arr, p.sla_us, p.windows_us)
+    assert one.feasible
+    oc, ol, of = OracleProblem(p).evaluate([one.index])
+    assert of[0] and oc[0] == one.cost and ol[0] == one.max_latency_us
+    space = p.space_size()
+    parts = [pl.plan(arr, p.sla_us, p.windows_us, shard=s_, n_shards=world) for s_ in range(world)]
+    assert sum(r.n_decided for r in parts) == space
+    for r in parts:
+        assert r.n_decided >= space // (2 * world), [q.n_decided for q in parts]
+        assert r.n_full_evals > 0
+    assert min((r.cost, r.index) for r in parts if r.feasible) == (one.cost, one.index)
+
+
+def test_c5_heavy_subplan_children_split_over_launches():
+    """C5's sub-plan of function 0's digit 112 (2^63 candidates): its shallow survivors have
+    2^28 deep children each, more than one survivor list holds, so their children run over
+    several deep launches.  Single rank and 2 shards agree; the oracle re-checks the winner."""
+    import torch
+    p = W.make_config("C5")
+    pl = S.planner_for(p)
+    arr = torch.as_tensor(p.arrivals_us).cuda()
+    kw = dict(n_fixed=1, fixed_digits=[112])
+    one = pl.plan(arr, p.sla_us, p.windows_us, **kw)
+    assert one.feasible
+    oc, ol, of = OracleProblem(p, **kw).evaluate([one.index])
+    assert of[0] and oc[0] == one.cost and ol[0] == one.max_latency_us
+    parts = [pl.plan(arr, p.sla_us, p.windows_us, shard=s_, n_shards=2, **kw) for s_ in range(2)]
+    assert sum(r.n_decided for r in parts) == 1 << 63
+    assert min((r.cost, r.index) for r in parts if r.feasible) == (one.cost, one.index)
