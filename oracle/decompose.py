@@ -17,7 +17,10 @@ from __future__ import annotations
 import numpy as np
 
 
-def decompose_search(prob, it_us: int, row_windows, oracle_cls):
+def decompose_search(prob, it_us: int, row_windows, oracle_cls, trace=None):
+    """Returns (configs, cost, max latency, feasible, number of paths).  If `trace` is a
+    dict it receives the steps: "paths", "path_choices" (each path's Top-1 result, configs
+    in path order), "path_latency" (closed form before combining), "combined"."""
     n = prob.n_funcs
     M = [int(m) for m in prob.n_configs]
     off = np.concatenate([[0], np.cumsum(prob.n_configs)]).astype(int)
@@ -82,6 +85,9 @@ def decompose_search(prob, it_us: int, row_windows, oracle_cls):
                 if others + I(k, rank[k][r]) <= pl:
                     cfg[k] = rank[k][r]
                     break
+    if trace is not None:
+        trace.update(paths=[list(P) for P in paths], path_choices=[list(c) for c in choice],
+                     path_latency=list(path_lat), combined=list(cfg))
     o = oracle_cls(prob, row_windows=row_windows)
     idx = 0
     for k in range(n):

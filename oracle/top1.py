@@ -17,7 +17,11 @@ from __future__ import annotations
 import numpy as np
 
 
-def top1_search(prob, it_us: int, row_windows, oracle_cls):
+def top1_search(prob, it_us: int, row_windows, oracle_cls, trace=None):
+    """Returns (leaf configs, cost, max latency, feasible, nodes evaluated).  If `trace` is a
+    list, the nodes in the order the paper's walk visits them (each layer
+    stops at its first SLA-meeting node) are appended as (layer, configs, meets SLA); layer 0
+    is the root T^0."""
     n = prob.n_funcs
     M = [int(m) for m in prob.n_configs]
     off = np.concatenate([[0], np.cumsum(prob.n_configs)]).astype(int)
@@ -48,6 +52,8 @@ def top1_search(prob, it_us: int, row_windows, oracle_cls):
 
     root = [rank[k][0] for k in range(n)]
     cost, lat, feas = evaluate([root])
+    if trace is not None:
+        trace.append((0, list(root), bool(feas[0])))
     if feas[0]:
         return root, float(cost[0]), int(lat[0]), True, nodes
     chosen = []
@@ -59,6 +65,8 @@ def top1_search(prob, it_us: int, row_windows, oracle_cls):
         if layer:
             c, l, f = evaluate(layer)
             for i in range(len(layer)):
+                if trace is not None:
+                    trace.append((k + 1, list(layer[i]), bool(f[i])))
                 if f[i]:
                     pick = layer[i][k]
                     break

@@ -531,6 +531,17 @@ RangePlan range_plan(const smiless_ctx *ctx, const smiless_plan_args *a) {
     RangePlan rp{true, 64, d_cap};
     if (a->flags & SMILESS_FLAG_FORCE_INT64) return rp;
     const i64 LIM = 0x7fffffffll;
+    // SMILESS_FORCE_K (testing): use this chunk length if the int32 range rule holds for it
+    // (else the int64 path), so the shorter-chunk variants are exercised on ordinary inputs
+    if (const char *fk = getenv("SMILESS_FORCE_K")) {
+        const int K = atoi(fk);
+        if (K == 64 || K == 32 || K == 16 || K == 8 || K == 4) {
+            const i64 bound = (i64)K * d_cap + sla + (i64)ctx->N * (ctx->Tmax + ctx->Imax) + wmax + ctx->Tmax +
+                              (i64)K * ctx->Imax;
+            if (bound < LIM && (i64)K * wmax < LIM) return RangePlan{false, K, d_cap};
+            return rp;
+        }
+    }
     for (int K : {64, 32, 16, 8, 4}) {
         const i64 bound = (i64)K * d_cap + sla + (i64)ctx->N * (ctx->Tmax + ctx->Imax) + wmax + ctx->Tmax +
                           (i64)K * ctx->Imax;

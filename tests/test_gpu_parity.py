@@ -943,3 +943,69 @@ def test_c5_heavy_subplan_children_split_over_launches():
     parts = [pl.plan(arr, p.sla_us, p.windows_us, shard=s_, n_shards=2, **kw) for s_ in range(2)]
     assert sum(r.n_decided for r in parts) == 1 << 63
     assert min((r.cost, r.index) for r in parts if r.feasible) == (one.cost, one.index)
+
+
+# ---------------------------------------------------------------------------------------
+# Full-size parity (J = 10^4) of the fast evaluators around each config's OPT, and every
+# int32 chunk length K
+# ---------------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("name,nf,fixed", [("C2", 0, []), ("C3", 0, []), ("C5", 1, [112])])
+def test_full_size_per_candidate_costs_around_opt(name, nf, fixed):
+    """P:305 (OPT by exhaustive search): 4,096 consecutive candidates around the exact plan's
+    winner at the full J = 10^4, evaluated by the memoised throughput kernels (no pruning)
+    and by the prune-mode plan kernel, cost bits and feasibility per candidate against the
+    oracle.  C5 pins function 0's digit (its space is 2^70)."""
+    import torch
+    p = W.make_config(name)
+    kw = dict(n_fixed=nf, fixed_digits=fixed)
+    pl = S.planner_for(p)
+    arr = torch.as_tensor(p.arrivals_us).cuda()
+    opt = pl.plan(arr, p.sla_us, p.windows_us, **kw)
+    assert opt.feasible
+    lo = opt.index // 4096 * 4096
+    oc, ol, of = OracleProblem(p, **kw).evaluate(np.arange(lo, lo + 4096, dtype=np.uint64))
+    assert of.any() and of[opt.index - lo] and oc[opt.index - lo] == opt.cost
+    for flags in (S.FLAG_NO_PRUNE, 0):
+        out = np.empty(4096)
+        r = pl.plan(arr, p.sla_us, p.windows_us, begin=lo, end=lo + 4096, flags=flags, cost_out=out, **kw)
+        assert_dump_matches(out, oc, of)
+        assert r.index == opt.index and r.cost == opt.cost
+
+
+@pytest.mark.parametrize("K", ["32", "16", "8", "4"])
+def test_every_int32_chunk_length_is_exact(K, monkeypatch):
+    """The int32 path rebases times every K steps; K in {32, 16, 8, 4} is chosen only for
+    large windows/SLAs, so force it (SMILESS_FORCE_K) on random DAGs and on a full-size C3
+    slice: per-candidate costs in throughput (memo) and prune mode equal the oracle's."""
+    monkeypatch.setenv("SMILESS_FORCE_K", K)
+    rng = np.random.default_rng(300 + int(K))
+    n_checked = 0
+    for t in range(60):
+        n = int(rng.integers(2, 7))
+        p = W.random_problem(rng, n, 4, int(rng.integers(1, 6)), int(rng.integers(2, 140)))
+        space = p.space_size()
+        if space > 20000:
+            continue
+        oc, ol, of = OracleProblem(p).evaluate(np.arange(space, dtype=np.uint64))
+        pl = S.planner_for(p)
+        for flags in (0, S.FLAG_NO_PRUNE):
+            out = np.empty(space)
+            r = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=flags, cost_out=out)
+            assert_dump_matches(out, oc, of)
+            assert not r.int64_path
+        n_checked += 1
+        if n_checked == 12:
+            break
+    assert n_checked >= 8
+    p = W.make_config("C3")
+    pl = S.planner_for(p)
+    opt = pl.plan(p.arrivals_us, p.sla_us, p.windows_us)          # exact full-space plan with this K
+    assert opt.feasible and not opt.int64_path
+    lo = opt.index // 2048 * 2048
+    oc, ol, of = OracleProblem(p).evaluate(np.arange(lo, lo + 2048, dtype=np.uint64))
+    assert of[opt.index - lo] and oc[opt.index - lo] == opt.cost
+    out = np.empty(2048)
+    r = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, begin=lo, end=lo + 2048, flags=S.FLAG_NO_PRUNE, cost_out=out)
+    assert not r.int64_path
+    assert_dump_matches(out, oc, of)

@@ -440,3 +440,109 @@ def test_derived_windows_reproduce_eq5_on_periodic_arrivals():
                     assert billed[k] == J * int(T[r] + I[r])
                 else:
                     assert billed[k] == int(T[r] + I[r]) + (J - 1) * IT
+
+
+# ---------------------------------------------------------------------------
+# Hand-derived paper examples for the NEXT oracles and the cost rounding
+# (tests/golden/P*.json, each with its citation and derivation)
+# ---------------------------------------------------------------------------
+
+def _golden(name):
+    return json.load(open(os.path.join(GOLDEN, name)))
+
+
+def _problem_from(g, windows=(0,)):
+    return mk(g["preds"], g["exec_us"], g["init_us"], g["arrivals_us"], list(windows), sla=g.get("sla_us", 10**9),
+              prices=g.get("price_per_us") or [float.fromhex(h) for h in g["price_per_us_hex"]],
+              n_configs=g.get("n_configs"))
+
+
+@pytest.mark.parametrize("name", ["P1_top1_walk_chain.json", "P1b_top1_ranking_case_I_II.json"])
+def test_top1_walk_follows_fig6_narrative(name):
+    """the Top-1 walk visits T^0 -> T^1_1 -> T^1_2 -> T^2_2 -> T^1_3 -> T^2_3 ->
+    T^3_3 on the hand-built chain (golden P1), ranks configurations by the Case I / Case II
+    per-invocation cost (golden P1b), and stops at the hand-derived leaf."""
+    from oracle.top1 import top1_search
+    g = _golden(name)
+    p = _problem_from(g)
+    trace = []
+    cfg, cost, lat, ok, nodes = top1_search(p, g["it_us"], g["row_windows_us"], OracleProblem, trace=trace)
+    assert [[l, c, f] for l, c, f in trace] == g["expected_walk"]
+    assert cfg == g["expected_leaf"] and ok
+    assert lat == g["expected_latency_us"] and cost == g["expected_cost"]
+
+
+def test_decompose_combine_on_diamond():
+    """paths of the diamond, each path's Top-1 choice, F_s/F_e take the fastest
+    of their paths' choices, branch functions keep their path latency (golden P2)."""
+    from oracle.decompose import decompose_search
+    g = _golden("P2_decompose_diamond.json")
+    p = _problem_from(g)
+    tr = {}
+    cfg, cost, lat, ok, n_paths = decompose_search(p, g["it_us"], g["row_windows_us"], OracleProblem, trace=tr)
+    assert tr["paths"] == g["expected_paths"] and n_paths == 2
+    assert tr["path_choices"] == g["expected_path_choices"]
+    assert tr["path_latency"] == g["expected_path_latency"]
+    assert cfg == g["expected_combined"] and ok
+    assert lat == g["expected_latency_us"] and cost == g["expected_cost"]
+
+
+def _autoscale_golden():
+    g = _golden("P3_autoscale_eq7.json")
+
+    class _P:
+        n_funcs = len(g["n_configs"])
+        n_configs = g["n_configs"]
+        price_per_us = np.asarray([float.fromhex(h) for h in g["price_per_us_hex"]])
+    exp = [(c, b, i, float(x)) for c, b, i, x in g["expected"]]
+    return g, _P, exp
+
+
+def test_autoscale_eq7_hand_worked_with_tie():
+    """P:226-239 Eq. (7)/(8): the brute-force oracle gives the hand-worked (config, B,
+    instances, cost) per function, including the lower-config tie-break (golden P3)."""
+    from oracle.autoscale import autoscale
+    g, prob, exp = _autoscale_golden()
+    out = autoscale(prob, g["slope_us"], g["intercept_us"], g["invocations"], g["it_us"], g["target_us"])
+    assert [tuple(o) for o in out] == exp
+
+
+def test_autoscale_library_matches_hand_worked_golden():
+    """The library's host-side bisection (smiless_autoscale) on the same golden."""
+    from paper_conf_sc_luxl0y024_b200 import smiless as S
+    g, prob, exp = _autoscale_golden()
+    n = prob.n_funcs
+    pl = S.Planner(device=0)
+    pl.load_dag(*W.csr_from_preds([[]] * n))
+    ncfg = np.asarray(g["n_configs"], np.int32)
+    z = np.zeros(int(ncfg.sum()), np.int32)
+    pl.load_profiles(ncfg, z + 1, z, prob.price_per_us)
+    out = pl.autoscale(g["slope_us"], g["intercept_us"], g["invocations"], g["it_us"], g["target_us"])
+    assert [(int(o[0]), int(o[1]), int(o[2]), float(o[3])) for o in out] == exp
+
+
+def test_cost_is_left_to_right_without_fma_for_paper_prices():
+    """G15 / Eq. (3)-(4) with the paper's non-dyadic prices (golden P4): the oracle's cost
+    bits are the left-to-right correctly rounded sum, which differs from the FMA-contracted
+    one, so an oracle (or kernel) that fuses a product into the sum fails here."""
+    g = _golden("P4_cost_no_fma.json")
+    p = _problem_from(g)
+    c, l, f = OracleProblem(p).evaluate([0])
+    assert c[0].hex() == g["expected_cost_hex"]
+    assert g["expected_cost_hex"] != g["fma_contracted_cost_hex"]
+    assert g["expected_cost_hex"] != g["right_to_left_cost_hex"]
+    # the same numbers by exact rational arithmetic, rounding after every operation
+    E = [t + i for t, i in zip(g["init_us"], g["exec_us"])]
+    U = [Fraction(float.fromhex(h)) for h in g["price_per_us_hex"]]
+    rnd = lambda q: float(q)  # noqa: E731  (correctly rounded)
+    lr = rnd(U[0] * E[0])
+    for k in (1, 2):
+        lr = rnd(Fraction(lr) + Fraction(rnd(U[k] * E[k])))
+    fused = rnd(U[0] * E[0])
+    for k in (1, 2):
+        fused = rnd(Fraction(fused) + U[k] * E[k])
+    assert lr.hex() == g["expected_cost_hex"] and fused.hex() == g["fma_contracted_cost_hex"]
+    rl = rnd(U[2] * E[2])
+    for k in (1, 0):
+        rl = rnd(Fraction(rl) + Fraction(rnd(U[k] * E[k])))
+    assert rl.hex() == g["right_to_left_cost_hex"]
