@@ -80,6 +80,7 @@ enum {
 #define SMILESS_MAX_WINDOWS 32
 #define SMILESS_MAX_CONFIGS 256
 #define SMILESS_MAX_SLAS 8
+#define SMILESS_MAX_INSTANCES 16
 
 /* Create a context bound to CUDA device `cuda_device` and stream `cuda_stream`
  * (a cudaStream_t; NULL = the legacy default stream; borrowed, not owned).
@@ -146,6 +147,17 @@ typedef struct {
                                      re-plan's) lets the evaluator's cost bound prune from the first
                                      launch (DESIGN.md section 5 item 11).  cost_cap >= 0, not NaN;
                                      EINVAL with SMILESS_FLAG_NO_PRUNE or in smiless_plan_sla_sweep */
+    const int32_t *instances;     /* optional [n_funcs] host array (NULL = one instance each): NEXT-4
+                                     scale-out (reading G26): function k runs
+                                     instances[k] identical instances (same configuration and window);
+                                     request j is dispatched to instance j mod instances[k] (round
+                                     robin), each instance serves its requests in request order, and
+                                     the first request of each instance finds it pre-warmed (G5).
+                                     Each instance is billed for its own loaded time.
+                                     1 <= instances[k] <= SMILESS_MAX_INSTANCES.  With any value > 1
+                                     the throughput-mode prefix memoisation is not used (the plan runs
+                                     on smiless_plan_kernel); results are exact as always.  The
+                                     instance counts typically come from smiless_autoscale_rows.    */
 } smiless_plan_args;
 
 typedef struct {

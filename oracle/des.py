@@ -110,7 +110,31 @@ def simulate_instance(x: Sequence[int], exec_us: int, init_us: int, window_us: i
     return done, billed
 
 
-def simulate(prob, config: Sequence[int], window: Sequence[int]) -> Tuple[List[int], List[int]]:
+def simulate_function(x: Sequence[int], exec_us: int, init_us: int, window_us: int,
+                      instances: int = 1) -> Tuple[List[int], int]:
+    """Scale-out (reading G26): `instances` identical instances, request j
+    dispatched to instance j mod n (round robin), each instance serving its requests in
+    request order (an input ready before the previous request of the same instance is
+    admitted when that one is: effective arrival = running max over the instance's
+    requests).  Returns (completion per request, billed loaded time summed over instances)."""
+    J = len(x)
+    done = [0] * J
+    billed = 0
+    for i in range(min(instances, J)):
+        idx = list(range(i, J, instances))
+        xs, m = [], None
+        for j in idx:
+            m = int(x[j]) if m is None else max(m, int(x[j]))
+            xs.append(m)
+        d, b = simulate_instance(xs, exec_us, init_us, window_us)
+        for j, t in zip(idx, d):
+            done[j] = t
+        billed += b
+    return done, billed
+
+
+def simulate(prob, config: Sequence[int], window: Sequence[int],
+             instances: Sequence[int] = None) -> Tuple[List[int], List[int]]:
     """(billed per function, E2E latency per request) for one candidate.
 
     Input-ready time of function k for request j: r_j for a source, else the
@@ -131,8 +155,9 @@ def simulate(prob, config: Sequence[int], window: Sequence[int]) -> Tuple[List[i
         else:
             x = [max(dones[p][j] for p in preds) for j in range(len(r))]
         row = off[k] + int(config[k])
-        d, b = simulate_instance(x, int(prob.exec_us[row]), int(prob.init_us[row]),
-                                 int(prob.windows_us[int(window[k])]))
+        d, b = simulate_function(x, int(prob.exec_us[row]), int(prob.init_us[row]),
+                                 int(prob.windows_us[int(window[k])]),
+                                 1 if instances is None else int(instances[k]))
         dones.append(d)
         billed.append(b)
     sinks = [k for k in range(n) if k not in listed]

@@ -50,6 +50,7 @@ class _Problem(ctypes.Structure):
         ("n_fixed", ctypes.c_int32),
         ("fixed_digits", ctypes.c_void_p),
         ("row_windows", ctypes.c_void_p),
+        ("instances", ctypes.c_void_p),
     ]
 
 
@@ -82,10 +83,12 @@ class OracleProblem:
     """Holds contiguous copies of a workloads.Problem for the C oracle."""
 
     def __init__(self, prob, sla_us: Optional[int] = None, n_fixed: int = 0,
-                 fixed_digits: Sequence[int] = (), row_windows: Optional[Sequence[int]] = None):
+                 fixed_digits: Sequence[int] = (), row_windows: Optional[Sequence[int]] = None,
+                 instances: Optional[Sequence[int]] = None):
         """row_windows (optional, [sum M]): the window of each (function, config) row, used
         instead of the grid (windows_us must then hold a single entry) -- the paper's
-        derived pre-warm windows (NEXT-1)."""
+        derived pre-warm windows (NEXT-1).  instances (optional, [N]): n_k round-robin
+        instances per function (NEXT-4 scale-out, reading G26); None = one each."""
         self.keep = dict(
             pred_ptr=np.ascontiguousarray(prob.pred_ptr, dtype=np.int32),
             pred_idx=np.ascontiguousarray(prob.pred_idx, dtype=np.int32) if len(prob.pred_idx) else np.zeros(1, np.int32),
@@ -97,7 +100,10 @@ class OracleProblem:
             windows=np.ascontiguousarray(prob.windows_us, dtype=np.int32),
             fixed=np.ascontiguousarray(np.asarray(list(fixed_digits) or [0], dtype=np.int32)),
             roww=None if row_windows is None else np.ascontiguousarray(np.asarray(row_windows, dtype=np.int32)),
+            inst=None if instances is None else np.ascontiguousarray(np.asarray(instances, dtype=np.int32)),
         )
+        if instances is not None:
+            assert len(self.keep["inst"]) == int(prob.pred_ptr.shape[0] - 1)
         if row_windows is not None:
             assert len(prob.windows_us) == 1 and len(self.keep["roww"]) == int(np.sum(prob.n_configs))
         k = self.keep
@@ -112,7 +118,8 @@ class OracleProblem:
             sla_us=int(prob.sla_us if sla_us is None else sla_us),
             windows_us=k["windows"].ctypes.data, n_windows=int(k["windows"].shape[0]),
             n_fixed=int(n_fixed), fixed_digits=k["fixed"].ctypes.data,
-            row_windows=None if k["roww"] is None else k["roww"].ctypes.data)
+            row_windows=None if k["roww"] is None else k["roww"].ctypes.data,
+            instances=None if k["inst"] is None else k["inst"].ctypes.data)
 
     # -- API ---------------------------------------------------------------
     def space_size(self) -> int:

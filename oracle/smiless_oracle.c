@@ -50,6 +50,8 @@ typedef struct {
     const int32_t *fixed_digits; /* [n_fixed] digit = config * W + window         */
     const int32_t *row_windows;  /* optional [sum M]: the window of (k, c) itself  */
                                  /* (NEXT-1 derived windows; then W must be 1)    */
+    const int32_t *instances;    /* optional [N]: n_k >= 1 instances of function k */
+                                 /* (NEXT-4 scale-out, reading G26); NULL = all 1  */
 } oracle_problem;
 
 /* Row offset of function k in the function-major profile arrays. */
@@ -100,8 +102,13 @@ static void find_sinks(const oracle_problem *P, uint8_t *is_sink) {
  *   x   = r_j                          for a source function
  *       = max_{p in pred(k)} D[p][j]   otherwise   (AND-join; "max over
  *                                        parallel branches")
- *   j == 0:  start = x, bill = T   (first invocation pre-warmed, reading G5)
- *   j >= 1, f = D[k][j-1] (previous completion on this instance), g = x - f:
+ *   Scale-out (NEXT-4, "launching multiple instances of the same function";
+ *   reading G26): function k runs n_k identical instances (same configuration and
+ *   window); request j is served by instance j mod n_k (round-robin dispatch), each
+ *   instance in request order.  n_k = 1 is the single instance of P:169-200.
+ *
+ *   j <  n_k:  start = x, bill = T   (first invocation on its instance pre-warmed, G5)
+ *   j >= n_k, f = D[k][j-n_k] (previous completion on this instance), g = x - f:
  *     g <= 0       : start = f,   bill = 0      busy -> FIFO wait, stays warm
  *                                               (Case III, Fig. 5(c); G6)
  *     window == 0  : start = x,   bill = g      keep-alive, idle time billed
@@ -121,8 +128,9 @@ static void simulate_into(const oracle_problem *P, const int32_t *config, const 
     const int N = P->n_funcs;
     const int64_t J = P->n_arrivals;
     const int64_t *r = P->arrivals_us;
-    int64_t I[64], T[64], w[64];
+    int64_t I[64], T[64], w[64], n_inst[64];
     for (int k = 0; k < N; ++k) {
+        n_inst[k] = P->instances ? P->instances[k] : 1;
         int64_t row = row0(P, k) + config[k];
         I[k] = P->exec_us[row];
         T[k] = P->init_us[row];
@@ -142,11 +150,11 @@ static void simulate_into(const oracle_problem *P, const int32_t *config, const 
                 }
             }
             int64_t start, bill;
-            if (j == 0) {
+            if (j < n_inst[k]) {
                 start = x;
                 bill = T[k];
             } else {
-                int64_t f = D[(int64_t)k * J + (j - 1)];
+                int64_t f = D[(int64_t)k * J + (j - n_inst[k])];
                 int64_t g = x - f;
                 if (g <= 0) {
                     start = f;
@@ -193,9 +201,18 @@ static double cost_of(const oracle_problem *P, const int32_t *config, const int6
 }
 
 /* Public: simulate one explicit candidate.  Returns 0, or -1 on bad args. */
+/* instances, when given, must be >= 1 */
+static int bad_problem(const oracle_problem *P) {
+    if (P->n_funcs < 1 || P->n_funcs > 64 || P->n_arrivals < 1) return 1;
+    if (P->instances)
+        for (int k = 0; k < P->n_funcs; ++k)
+            if (P->instances[k] < 1) return 1;
+    return 0;
+}
+
 int oracle_simulate(const oracle_problem *P, const int32_t *config, const int32_t *window,
                     int64_t *billed, int64_t *latency) {
-    if (P->n_funcs < 1 || P->n_funcs > 64 || P->n_arrivals < 1) return -1;
+    if (bad_problem(P)) return -1;
     uint8_t is_sink[64];
     find_sinks(P, is_sink);
     int64_t *D = (int64_t *)malloc(sizeof(int64_t) * (size_t)P->n_funcs * (size_t)P->n_arrivals);
@@ -242,7 +259,7 @@ static void eval_one(worker_scratch *s, uint64_t index, double *cost, int64_t *m
 
 int oracle_evaluate(const oracle_problem *P, const uint64_t *idx, int64_t n,
                     double *cost, int64_t *max_lat, uint8_t *feasible) {
-    if (P->n_funcs < 1 || P->n_funcs > 64 || P->n_arrivals < 1) return -1;
+    if (bad_problem(P)) return -1;
     uint8_t is_sink[64];
     find_sinks(P, is_sink);
     worker_scratch s;
@@ -289,7 +306,7 @@ static void *plan_worker(void *arg) {
  */
 int oracle_plan(const oracle_problem *P, uint64_t begin, uint64_t end, int n_threads,
                 uint64_t *best_idx, double *best_cost, int64_t *best_lat) {
-    if (P->n_funcs < 1 || P->n_funcs > 64 || P->n_arrivals < 1) return -1;
+    if (bad_problem(P)) return -1;
     uint64_t space = oracle_space_size(P);
     if (space == 0) return -1;
     if (end == 0 || end > space) end = space;

@@ -405,7 +405,7 @@ int ensure_device(smiless_ctx *ctx) {
     for (auto &ev : ctx->ev) CK(cudaEventCreate(&ev), "cudaEventCreate");
     CK(cudaMallocHost((void **)&ctx->hRes, sizeof(ResBlock) * SMILESS_MAX_SLAS), "cudaMallocHost");
     CK(ctx->dRes.ensure(SMILESS_MAX_SLAS), "cudaMalloc");
-    CK(ctx->dScal.ensure(2), "cudaMalloc");
+    CK(ctx->dScal.ensure(34), "cudaMalloc");          // [0] R, [1] o_last, [2..34) scale-out tail sums
     CK(ctx->dErr.ensure(1), "cudaMalloc");
     CK(ctx->dCounter.ensure(1), "cudaMalloc");
     CK(ctx->dStats.ensure(2), "cudaMalloc");
@@ -416,8 +416,10 @@ int ensure_device(smiless_ctx *ctx) {
 
 int upload_tables(smiless_ctx *ctx) {
     if (!ctx->tables_dirty) return SMILESS_OK;
-    const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
-    const size_t padU = (size_t)((ctx->sumM + 1) & ~1);
+    // one spare all-zero row after the last (I = T = 0, U = 0): the virtual sink of
+    // scale-out plans (see dag_spec_source), staged with sumM + 1 rows
+    const size_t padI = (size_t)((ctx->sumM + 1 + 3) & ~3);
+    const size_t padU = (size_t)((ctx->sumM + 1 + 1) & ~1);
     std::vector<int> I(padI, 0), NI(padI, 0), T(padI, 0);
     std::vector<double> U(padU, 0.0);
     std::copy(ctx->I.begin(), ctx->I.end(), I.begin());
@@ -503,6 +505,10 @@ int validate_args(smiless_ctx *ctx, const smiless_plan_args *a, bool need_arriva
         return fail(ctx, SMILESS_ERANGE, "candidate space exceeds 2^63-1; pin leading digits with n_fixed");
     if (a->n_shards < 0 || (a->n_shards > 0 && (a->shard < 0 || a->shard >= a->n_shards)))
         return fail(ctx, SMILESS_EINVAL, "bad shard/n_shards");
+    if (a->instances)
+        for (int k = 0; k < ctx->N; ++k)
+            if (a->instances[k] < 1 || a->instances[k] > SMILESS_MAX_INSTANCES)
+                return fail(ctx, SMILESS_EINVAL, "instances[%d] out of [1, %d]", k, SMILESS_MAX_INSTANCES);
     if (a->flags & SMILESS_FLAG_COST_CAP) {
         if (!(a->cost_cap >= 0.0)) return fail(ctx, SMILESS_EINVAL, "cost_cap must be >= 0 (not NaN)");
         if (a->flags & SMILESS_FLAG_NO_PRUNE) return fail(ctx, SMILESS_EINVAL, "FLAG_COST_CAP requires prune mode");
@@ -520,6 +526,9 @@ struct RangePlan {
     i64 d_cap;
 };
 
+int inst_prologue(const smiless_ctx *ctx, const smiless_plan_args *a);
+int inst_max(const smiless_ctx *ctx, const smiless_plan_args *a);
+
 RangePlan range_plan(const smiless_ctx *ctx, const smiless_plan_args *a) {
     i64 wmax = a->windows_us[a->n_windows - 1];
     if (a->row_windows_us) {
@@ -531,21 +540,25 @@ RangePlan range_plan(const smiless_ctx *ctx, const smiless_plan_args *a) {
     RangePlan rp{true, 64, d_cap};
     if (a->flags & SMILESS_FLAG_FORCE_INT64) return rp;
     const i64 LIM = 0x7fffffffll;
+    // scale-out: the rings reach n_max - 1 requests back inside a frame, and the prologue
+    // (j = 1 .. P) must lie in chunk 0 (K >= P)
+    const i64 ring_span = (i64)(inst_max(ctx, a) - 1) * d_cap;
+    const int P = inst_prologue(ctx, a);
     // SMILESS_FORCE_K (testing): use this chunk length if the int32 range rule holds for it
     // (else the int64 path), so the shorter-chunk variants are exercised on ordinary inputs
     if (const char *fk = getenv("SMILESS_FORCE_K")) {
         const int K = atoi(fk);
         if (K == 64 || K == 32 || K == 16 || K == 8 || K == 4) {
             const i64 bound = (i64)K * d_cap + sla + (i64)ctx->N * (ctx->Tmax + ctx->Imax) + wmax + ctx->Tmax +
-                              (i64)K * ctx->Imax;
-            if (bound < LIM && (i64)K * wmax < LIM) return RangePlan{false, K, d_cap};
+                              (i64)K * ctx->Imax + ring_span;
+            if (K >= P && bound < LIM && (i64)K * wmax < LIM) return RangePlan{false, K, d_cap};
             return rp;
         }
     }
     for (int K : {64, 32, 16, 8, 4}) {
         const i64 bound = (i64)K * d_cap + sla + (i64)ctx->N * (ctx->Tmax + ctx->Imax) + wmax + ctx->Tmax +
-                          (i64)K * ctx->Imax;
-        if (bound < LIM && (i64)K * wmax < LIM) return RangePlan{false, K, d_cap};
+                          (i64)K * ctx->Imax + ring_span;
+        if (K >= P && bound < LIM && (i64)K * wmax < LIM) return RangePlan{false, K, d_cap};
     }
     return rp;
 }
@@ -555,7 +568,23 @@ RangePlan range_plan(const smiless_ctx *ctx, const smiless_plan_args *a) {
 // ------------------------------------------------------------------------------------
 // Configs of the last function carried per lane (a unit = G x W candidates): as many as keep
 // G * W <= 16 variants (registers) and divide M_{N-1}.  SMILESS_G overrides (tuning).
+// Scale-out plans (NEXT-4, reading G26): a->instances[k] round-robin instances of function k.
+int inst_of(const smiless_plan_args *a, int k) { return a->instances ? a->instances[k] : 1; }
+int inst_max(const smiless_ctx *ctx, const smiless_plan_args *a) {
+    int m = 1;
+    for (int k = 0; k < ctx->N; ++k) m = std::max(m, inst_of(a, k));
+    return m;
+}
+bool inst_mode(const smiless_ctx *ctx, const smiless_plan_args *a) { return inst_max(ctx, a) > 1; }
+// prologue steps j = 1 .. P of a scale-out plan (the first request of instances 2 .. n_k), a
+// multiple of 4 so that the main loop keeps its 16-byte aligned offset loads
+int inst_prologue(const smiless_ctx *ctx, const smiless_plan_args *a) {
+    const int m = inst_max(ctx, a);
+    return m > 1 ? ((m - 1 + 3) & ~3) : 0;
+}
+
 int configs_per_lane(const smiless_ctx *ctx, const smiless_plan_args *a) {
+    if (inst_mode(ctx, a)) return 1;                 // last kernel function = the virtual sink (M = 1)
     const int M = ctx->M[ctx->N - 1], W = a->n_windows;
     int G = 1;
     const char *env = getenv("SMILESS_G");
@@ -564,6 +593,65 @@ int configs_per_lane(const smiless_ctx *ctx, const smiless_plan_args *a) {
     for (int g = 1; g <= want; ++g)
         if (M % g == 0 && g * W <= 32) G = g;
     return G;
+}
+
+// candidates per evaluator unit (lane): G configs x W windows of the last function; 1 for a
+// scale-out plan, whose last kernel function is the virtual sink (one variant)
+u64 unit_cands(const smiless_ctx *ctx, const smiless_plan_args *a) {
+    return inst_mode(ctx, a) ? 1 : (u64)a->n_windows * (u64)configs_per_lane(ctx, a);
+}
+// window variants of the last kernel function
+int variant_windows(const smiless_ctx *ctx, const smiless_plan_args *a) {
+    return inst_mode(ctx, a) ? 1 : a->n_windows;
+}
+
+// The DAG the evaluator kernels are specialised for.  Normally the application DAG.  For a
+// scale-out plan one virtual function V is appended: it joins every real sink, has one
+// configuration (I = T = 0, U = 0: the spare zero table row), keep-alive, one instance, and its
+// digit has radix 1 (the candidate index is unchanged).  Every real function is then an
+// "upstream" function of the kernel and can carry an instance ring; V is the kernel's last
+// function (sink sharing with one variant).  Cost: + U_V * E_V = + 0.0 (bit-exact).  Latency:
+// D_V,j = max_{i <= j} x_i (running max, I = 0), so max_j (D_V,j - r_j) = max_j L_j exactly
+// (r non-decreasing), which is all the SLA verdict and the pruning use.
+struct KDag {
+    int N = 0;
+    bool virt = false;
+    std::vector<std::vector<int>> preds;
+    std::vector<int> M, row0, inst;
+    u64 sink = 0;
+    std::vector<char> taint;     // scale-out function or downstream of one (bound kernel: lower bounds)
+};
+
+KDag kernel_dag(const smiless_ctx *ctx, const smiless_plan_args *a) {
+    KDag d;
+    d.virt = inst_mode(ctx, a);
+    d.N = ctx->N + (d.virt ? 1 : 0);
+    d.preds.resize(d.N);
+    d.M.resize(d.N);
+    d.row0.resize(d.N);
+    d.inst.resize(d.N, 1);
+    d.taint.resize(d.N, 0);
+    for (int k = 0; k < ctx->N; ++k) {
+        for (int e = ctx->pred_ptr[k]; e < ctx->pred_ptr[k + 1]; ++e) d.preds[k].push_back(ctx->pred_idx[e]);
+        d.M[k] = ctx->M[k];
+        d.row0[k] = ctx->row0[k];
+        d.inst[k] = inst_of(a, k);
+    }
+    if (d.virt) {
+        const int v = ctx->N;
+        for (int k = 0; k < ctx->N; ++k)
+            if ((ctx->sinkmask >> k) & 1ull) d.preds[v].push_back(k);
+        d.M[v] = 1;
+        d.row0[v] = ctx->sumM;
+        d.sink = 1ull << v;
+    } else {
+        d.sink = ctx->sinkmask;
+    }
+    for (int k = 0; k < d.N; ++k) {
+        d.taint[k] = d.inst[k] > 1;
+        for (int q : d.preds[k]) d.taint[k] |= d.taint[q];
+    }
+    return d;
 }
 
 // Branch-and-bound depth D (functions 0..D-1 assigned per prefix, D..N-1 relaxed), or 0 for
@@ -633,10 +721,20 @@ bool bound_lb_table(const smiless_ctx *ctx, int W) { return (size_t)ctx->sumM * 
 
 std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, bool off_smem,
                             int minb, int families) {
-    const int N = ctx->N, W = a->n_windows, NU = N - 1, nf = a->n_fixed;
+    const KDag kd = kernel_dag(ctx, a);
+    const int N = kd.N, W = a->n_windows, NU = N - 1, nf = a->n_fixed;
     const int G = configs_per_lane(ctx, a);
+    const int VW = variant_windows(ctx, a);
+    const int P = inst_prologue(ctx, a);
     const char *un_env = getenv("SMILESS_UNROLL");
     const int unroll = (un_env && atoi(un_env) == 2) ? 2 : 4;
+    // instance rings: function k keeps its n_k - 1 older completions in RG[rg0[k] ..]
+    std::vector<int> rg0(N, 0);
+    int n_rg = 0;
+    for (int k = 0; k < N; ++k) {
+        rg0[k] = n_rg;
+        n_rg += kd.inst[k] - 1;
+    }
     std::ostringstream s;
     s << "// generated by host.cpp:dag_spec_source -- DAG-specialised prefix of evaluator.cuh\n";
     s << "#define SM_N " << N << "\n#define SM_NU " << NU << "\n#define SM_NU_ALLOC " << std::max(NU, 1) << "\n";
@@ -645,9 +743,11 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_K " << rp.K << "\n#define SM_TIME64 " << (rp.time64 ? 1 : 0) << "\n";
     s << "#define SM_OFF_SMEM " << (off_smem ? 1 : 0) << "\n#define SM_THREADS " << kThreads
       << "\n#define SM_MINB " << minb << "\n";
-    s << "#define SM_W0_ZERO " << (!a->row_windows_us && a->windows_us[0] == 0 ? 1 : 0) << "\n";
+    // window variants of the last kernel function: the grid, or the virtual sink's keep-alive
+    s << "#define SM_VW " << VW << "\n";
+    s << "#define SM_W0_ZERO " << (kd.virt || (!a->row_windows_us && a->windows_us[0] == 0) ? 1 : 0) << "\n";
     s << "#define SM_G " << G << "\n#define SM_UNROLL " << unroll << "\n";
-    s << "#define SM_UPP " << (ctx->M[N - 1] / G) << "\n";   // units (config groups) per upstream prefix
+    s << "#define SM_UPP " << (kd.M[N - 1] / G) << "\n";   // units (config groups) per upstream prefix
     s << "#define SM_VTHREADS " << vthreads_per_cta() << "\n#define SM_VMINB " << vmin_blocks() << "\n";
     s << "#define SM_BUILD_PLAN " << ((families & FAM_PLAN) ? 1 : 0) << "\n#define SM_BUILD_BOUND "
       << ((families & FAM_BOUND) ? 1 : 0) << "\n#define SM_BUILD_MEMO " << ((families & FAM_MEMO) ? 1 : 0) << "\n";
@@ -674,18 +774,29 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     const char *alusul_env = getenv("SMILESS_ALUSUL"), *alug_env = getenv("SMILESS_ALUG");
     s << "#define SM_ALUSUL " << (alusul_env ? atoi(alusul_env) : 0) << "\n#define SM_ALUG "
       << (alug_env ? atoi(alug_env) : 0) << "\n";
+    // scale-out (NEXT-4): any instance count > 1, the prologue length, the ring size
+    s << "#define SM_INST " << (kd.virt ? 1 : 0) << "\n#define SM_PRO " << P << "\n#define SM_RG_ALLOC "
+      << std::max(n_rg, 1) << "\n";
+    s << "#define SM_NINST(k) (";
+    for (int k = 0; k < N; ++k) s << "(k)==" << k << "?" << kd.inst[k] << ":";
+    s << "1)\n";
+    s << "#define SM_ROWINST(r) (";                      // instances of the function owning table row r
+    for (int k = 0; k < N; ++k) s << "(r)<" << kd.row0[k] + kd.M[k] << "?" << kd.inst[k] << ":";
+    s << "1)\n";
     // compile-time window grid (immediates) and a constant-bank copy for runtime indices
     s << "#define SM_WIN(v) (";
     for (int v = 0; v < W; ++v) s << "(v)==" << v << "?" << a->windows_us[v] << ":";
     s << "0)\n";
+    // windows of the last kernel function's variants (the virtual sink: keep-alive)
+    s << "#define SM_VWIN(v) " << (kd.virt ? "0" : "SM_WIN(v)") << "\n";
     s << "__constant__ int c_win[" << W << "] = {";
     for (int v = 0; v < W; ++v) s << (v ? "," : "") << a->windows_us[v];
     s << "};\n#define SM_WINV(i) c_win[(i)]\n";
     s << "#define SM_ROW0(k) (";
-    for (int k = 0; k < N; ++k) s << "(k)==" << k << "?" << ctx->row0[k] << ":";
+    for (int k = 0; k < N; ++k) s << "(k)==" << k << "?" << kd.row0[k] << ":";
     s << "0)\n";
     s << "#define SM_MK(k) (";
-    for (int k = 0; k < N; ++k) s << "(k)==" << k << "?" << ctx->M[k] << ":";
+    for (int k = 0; k < N; ++k) s << "(k)==" << k << "?" << kd.M[k] << ":";
     s << "0)\n";
     s << R"(
 typedef long long i64;
@@ -703,13 +814,13 @@ static __device__ __forceinline__ tm_t opaque_sub(tm_t a, tm_t b);
 static __device__ __forceinline__ tm_t vaddmax(tm_t a, tm_t b, tm_t c);
 static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
 )";
-    // ---- decode: unit u -> digits (function N-1: config only) -------------------------
+    // ---- decode: unit u -> digits (last kernel function: config group only) ---------------
     s << "static __device__ __forceinline__ void dag_decode(u64 u, int (&dig)[SM_N], const int *fixed) {\n";
     if (nf <= N - 1) {
-        const int groups = ctx->M[N - 1] / G;   // config groups of the last function
+        const int groups = kd.M[N - 1] / G;   // config groups of the last function
         s << "  dig[" << N - 1 << "] = (int)(u % " << groups << "ull); u /= " << groups << "ull;\n";
         for (int k = N - 2; k >= nf; --k) {
-            const u64 radix = (u64)ctx->M[k] * (u64)W;
+            const u64 radix = (u64)kd.M[k] * (u64)W;
             s << "  dig[" << k << "] = (int)(u % " << radix << "ull); u /= " << radix << "ull;\n";
         }
     }
@@ -720,39 +831,78 @@ static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
     // min over predecessors of NF (= -(max over predecessors of F): the AND-join).
     // vminz blocks VIMNMX3 formation (ptxas erratum); nothing below negates a min/max input.
     auto nf_min = [&](int k) {
-        const int e0 = ctx->pred_ptr[k], e1 = ctx->pred_ptr[k + 1];
-        std::string e = "NF[" + std::to_string(ctx->pred_idx[e0]) + "]";
-        for (int e_ = e0 + 1; e_ < e1; ++e_) e = "vminz(" + e + ", NF[" + std::to_string(ctx->pred_idx[e_]) + "], z)";
+        const auto &pr = kd.preds[k];
+        std::string e = "NF[" + std::to_string(pr[0]) + "]";
+        for (size_t i = 1; i < pr.size(); ++i) e = "vminz(" + e + ", NF[" + std::to_string(pr[i]) + "], z)";
         return e;
     };
-    auto is_src = [&](int k) { return ctx->pred_ptr[k] == ctx->pred_ptr[k + 1]; };
-    // ---- j = 0: start = x; nx = -x is stored (st0) ---------------------------------------
+    auto is_src = [&](int k) { return kd.preds[k].empty(); };
+    auto ks = [](int k) { return std::to_string(k); };
+    // ---- j = 0: start = x; nx = -x is stored (st0); scale-out functions start EF = D_0 - r_0 --
     s << "template <int A> static __device__ __forceinline__ void dag_first(tm_t (&NF)[A], const tm_t (&NI)[A], "
-         "tm_t *st0, int tid, tm_t &nxl, tm_t &nlu, const tm_t z) {\n";
+         "tm_t *st0, int tid, tm_t &nxl, tm_t &nlu, const tm_t z, i64 (&EF)[A]) {\n";
     for (int k = 0; k < N - 1; ++k) {
         s << "  { const tm_t nx = " << (is_src(k) ? std::string("(tm_t)0") : nf_min(k)) << "; st0[" << k
           << " * SM_THREADS + tid] = nx; NF[" << k << "] = NI[" << k << "] + nx; }\n";
+        if (kd.inst[k] > 1) s << "  EF[" << k << "] = -(i64)NF[" << k << "];\n";
     }
     s << "  nxl = " << (is_src(N - 1) ? std::string("(tm_t)0") : nf_min(N - 1)) << ";\n";
     for (int k = 0; k < N - 1; ++k)
-        if ((ctx->sinkmask >> k) & 1ull) s << "  nlu = vminz(nlu, NF[" << k << "], z);\n";
-    s << "  (void)NF; (void)NI; (void)st0; (void)tid; (void)nlu; (void)z;\n}\n";
+        if ((kd.sink >> k) & 1ull) s << "  nlu = vminz(nlu, NF[" << k << "], z);\n";
+    s << "  (void)NF; (void)NI; (void)st0; (void)tid; (void)nlu; (void)z; (void)EF;\n}\n";
     // ---- j >= 1: g = x - f = x + NF; returns x of the last function ----------------------
-    s << "template <int A> static __device__ __forceinline__ tm_t dag_step(tm_t (&NF)[A], tm_t (&SU)[A], const tm_t "
-         "(&NI)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], const tm_t o, const tm_t z) {\n";
+    // JJ = 0: steady state; JJ >= 1: prologue step j = JJ of a scale-out plan, where a function
+    // with JJ < n_k serves the first request of instance JJ (pre-warmed, G5: start = x, no u).
+    // Instance rings: f = RG[rg0] (completion n_k requests back), shifted each step; NF[k] is
+    // always the newest completion (what the joins and sinks read).
+    s << "template <int JJ, int A, int R> static __device__ __forceinline__ tm_t dag_step(tm_t (&NF)[A], tm_t (&RG)[R], "
+         "tm_t (&SU)[A], const tm_t (&NI)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], const tm_t o, const tm_t z, "
+         "i64 (&EF)[A]) {\n";
     for (int k = 0; k < N - 1; ++k) {
-        const std::string g = is_src(k) ? "o + NF[" + std::to_string(k) + "]"
-                                        : "NF[" + std::to_string(k) + "] - " + nf_min(k);
-        s << "  fstep(NF[" << k << "], SU[" << k << "], " << g << ", NI[" << k << "], Te[" << k << "], Wn[" << k
-          << "]);\n";
+        const int n = kd.inst[k];
+        if (n == 1) {
+            const std::string g = is_src(k) ? "o + NF[" + ks(k) + "]" : "NF[" + ks(k) + "] - " + nf_min(k);
+            s << "  fstep(NF[" << k << "], SU[" << k << "], " << g << ", NI[" << k << "], Te[" << k << "], Wn[" << k
+              << "]);\n";
+            continue;
+        }
+        const std::string nx = is_src(k) ? std::string("opaque_sub(z, o)") : nf_min(k);   // -x
+        s << "  {\n";
+        s << "    tm_t nf = RG[" << rg0[k] << "];\n";
+        for (int r = 0; r + 1 < n - 1; ++r) s << "    RG[" << rg0[k] + r << "] = RG[" << rg0[k] + r + 1 << "];\n";
+        s << "    RG[" << rg0[k] + n - 2 << "] = NF[" << k << "];\n";
+        s << "    if (JJ != 0 && JJ < " << n << ") {\n";
+        s << "      NF[" << k << "] = NI[" << k << "] + " << nx << ";\n";
+        s << "      EF[" << k << "] += -(i64)NF[" << k << "] - (i64)o;\n";
+        s << "    } else {\n";
+        const std::string g = is_src(k) ? std::string("o + nf") : "nf - " + nf_min(k);
+        s << "      fstep(nf, SU[" << k << "], " << g << ", NI[" << k << "], Te[" << k << "], Wn[" << k << "]);\n";
+        s << "      NF[" << k << "] = nf;\n";
+        s << "    }\n  }\n";
     }
-    s << "  (void)NF; (void)SU; (void)NI; (void)Te; (void)Wn; (void)o; (void)z;\n";
+    s << "  (void)NF; (void)RG; (void)SU; (void)NI; (void)Te; (void)Wn; (void)o; (void)z; (void)EF;\n";
     s << "  return " << (is_src(N - 1) ? std::string("o") : "opaque_sub(z, " + nf_min(N - 1) + ")") << ";\n}\n";
+    // ---- scale-out billing: sum_{i < n_eff} (D_{J-1-i} - r_{J-1-i}) from the final ring -------
+    s << "template <int A, int R> static __device__ __forceinline__ i64 dag_elast(const int k, const tm_t (&NF)[A], "
+         "const tm_t (&RG)[R], const i64 *otail, const i64 J) {\n  i64 e = 0;\n";
+    for (int k = 0; k < N - 1; ++k) {
+        const int n = kd.inst[k];
+        if (n == 1) continue;
+        s << "  if (k == " << k << ") {\n    e = -(i64)NF[" << k << "] - otail[0];\n";
+        for (int i = 1; i < n; ++i)
+            s << "    if (J > " << i << ") e += -(i64)RG[" << rg0[k] + n - 1 - i << "] - otail[" << i << "];\n";
+        s << "  }\n";
+    }
+    s << "  (void)NF; (void)RG; (void)otail; (void)J; (void)k;\n  return e;\n}\n";
+    // ---- rebase of the instance rings (F -= sh  <=>  NF += sh) ---------------------------
+    s << "template <int R> static __device__ __forceinline__ void dag_ring_rebase(tm_t (&RG)[R], const tm_t sh) {\n";
+    for (int r = 0; r < n_rg; ++r) s << "  RG[" << r << "] += sh;\n";
+    s << "  (void)RG; (void)sh;\n}\n";
     // ---- upstream sinks' latency: nlu = min_j (NF_k + o_j) = -max_j L_j -------------------
     s << "template <int A> static __device__ __forceinline__ void dag_sinks(const tm_t (&NF)[A], const tm_t o, tm_t "
          "&nlu) {\n";
     for (int k = 0; k < N - 1; ++k)
-        if ((ctx->sinkmask >> k) & 1ull) s << "  nlu = vaddmin(NF[" << k << "], o, nlu);\n";
+        if ((kd.sink >> k) & 1ull) s << "  nlu = vaddmin(NF[" << k << "], o, nlu);\n";
     s << "  (void)NF; (void)o; (void)nlu;\n}\n";
     // ---- B&B pre-pass (smiless_bound_kernel): prefix decode, relaxed first/step ---------------
     {
@@ -760,7 +910,7 @@ static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
              "const int *fixed) {\n";
         for (int k = 0; k < N; ++k) s << "  dig[" << k << "] = 0;\n";
         for (int k = N - 1; k >= nf; --k) {
-            const u64 radix = (u64)ctx->M[k] * (u64)W;
+            const u64 radix = (u64)kd.M[k] * (u64)W;
             s << "  if (" << k << " < DD) { dig[" << k << "] = (int)(u % " << radix << "ull); u /= " << radix
               << "ull; }\n";
         }
@@ -771,21 +921,34 @@ static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
         for (int k = 0; k < N; ++k)
             s << "  NF[" << k << "] = NI[" << k << "] + " << (is_src(k) ? std::string("(tm_t)0") : nf_min(k)) << ";\n";
         for (int k = 0; k < N; ++k)
-            if ((ctx->sinkmask >> k) & 1ull) s << "  nl = vminz(nl, NF[" << k << "], z);\n";
+            if ((kd.sink >> k) & 1ull) s << "  nl = vminz(nl, NF[" << k << "], z);\n";
         s << "  (void)z;\n}\n";
+        // Lower bounds of every done time: an assigned function (k < DD) is exact under model M
+        // only if no scale-out function is it or upstream of it (a scale-out function is
+        // bounded, and model M's start is not monotone in f); otherwise every branch of model M
+        // has start >= max(x, f) (one instance) or start >= x (several), so keep-alive with
+        // max(x, f) + I (one instance) or x + I (several) is a lower bound, monotone in its
+        // lower-bounded inputs.  Relaxed functions (k >= DD) take their smallest exec time.
         s << "template <int DD, int A> static __device__ __forceinline__ void dag_bstep(tm_t (&NF)[A], const tm_t "
              "(&NI)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], const tm_t o, tm_t &nl, const tm_t z) {\n"
              "  tm_t su = 0;\n";
         for (int k = 0; k < N; ++k) {
-            const std::string g = is_src(k) ? "o + NF[" + std::to_string(k) + "]"
-                                            : "NF[" + std::to_string(k) + "] - " + nf_min(k);
-            // assigned (k < DD): model M; relaxed: keep-alive (start - f = max(g, 0)), smallest exec
-            s << "  if (" << k << " < DD) fstep(NF[" << k << "], su, " << g << ", NI[" << k << "], Te[" << k
-              << "], Wn[" << k << "]);\n  else { const tm_t g = " << g << "; NF[" << k << "] = NF[" << k
-              << "] + NI[" << k << "] - vmax(g, (tm_t)0); }\n";
+            const std::string g = is_src(k) ? "o + NF[" + ks(k) + "]" : "NF[" + ks(k) + "] - " + nf_min(k);
+            const std::string nx = is_src(k) ? std::string("opaque_sub(z, o)") : nf_min(k);
+            if (kd.inst[k] > 1) {
+                s << "  NF[" << k << "] = NI[" << k << "] + " << nx << ";\n";
+            } else if (kd.taint[k]) {
+                s << "  { const tm_t g = " << g << "; NF[" << k << "] = NF[" << k << "] + NI[" << k
+                  << "] - vmax(g, (tm_t)0); }\n";
+            } else {
+                // assigned (k < DD): model M; relaxed: keep-alive (start - f = max(g, 0)), smallest exec
+                s << "  if (" << k << " < DD) fstep(NF[" << k << "], su, " << g << ", NI[" << k << "], Te[" << k
+                  << "], Wn[" << k << "]);\n  else { const tm_t g = " << g << "; NF[" << k << "] = NF[" << k
+                  << "] + NI[" << k << "] - vmax(g, (tm_t)0); }\n";
+            }
         }
         for (int k = 0; k < N; ++k)
-            if ((ctx->sinkmask >> k) & 1ull) s << "  nl = vaddmin(NF[" << k << "], o, nl);\n";
+            if ((kd.sink >> k) & 1ull) s << "  nl = vaddmin(NF[" << k << "], o, nl);\n";
         s << "  (void)su; (void)Te; (void)Wn; (void)z;\n}\n";
     }
     return s.str();
@@ -804,10 +967,15 @@ size_t smem_memo_up(const smiless_ctx *ctx, const RangePlan &rp, i64 n_off) {
            ((tsz * (size_t)ctx->N * kThreads + 15) & ~(size_t)15);
 }
 size_t smem_memo_var(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off);
+// table rows the plan / bound kernels stage: a scale-out plan adds the virtual sink's zero row
+int kernel_rows(const smiless_ctx *ctx, const smiless_plan_args *a) { return ctx->sumM + (inst_mode(ctx, a) ? 1 : 0); }
+int kernel_funcs(const smiless_ctx *ctx, const smiless_plan_args *a) { return ctx->N + (inst_mode(ctx, a) ? 1 : 0); }
+
 size_t smem_bound_bytes(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off) {
-    const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
-    const size_t lbt = bound_lb_table(ctx, a->n_windows) ? 8 * (size_t)((ctx->sumM * a->n_windows + 1) & ~1) : 0;
-    return 3 * padI * 4 + 8 * (size_t)((ctx->sumM + 1) & ~1) + lbt + (rp.time64 ? 8 : 4) * (size_t)n_off;
+    const int rows = kernel_rows(ctx, a);
+    const size_t padI = (size_t)((rows + 3) & ~3);
+    const size_t lbt = bound_lb_table(ctx, a->n_windows) ? 8 * (size_t)((rows * a->n_windows + 1) & ~1) : 0;
+    return 3 * padI * 4 + 8 * (size_t)((rows + 1) & ~1) + lbt + (rp.time64 ? 8 : 4) * (size_t)n_off;
 }
 
 int nvrtc_compile(smiless_ctx *ctx, const std::string &src, std::vector<char> &cubin, std::string &log) {
@@ -836,12 +1004,13 @@ int nvrtc_compile(smiless_ctx *ctx, const std::string &src, std::vector<char> &c
 }
 
 size_t smem_bytes(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off, bool off_smem) {
-    const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
-    const size_t padU = (size_t)((ctx->sumM + 1) & ~1);
+    const int rows = kernel_rows(ctx, a), kn = kernel_funcs(ctx, a);
+    const size_t padI = (size_t)((rows + 3) & ~3);
+    const size_t padU = (size_t)((rows + 1) & ~1);
     const size_t tsz = rp.time64 ? 8 : 4;
     size_t b = 3 * padI * 4 + padU * 8;
-    b += 8ull * (size_t)(ctx->N - 1 + a->n_windows * configs_per_lane(ctx, a)) * kThreads;
-    b += (tsz * (size_t)ctx->N * kThreads + 15) & ~(size_t)15;
+    b += 8ull * (size_t)(kn - 1 + (int)unit_cands(ctx, a)) * kThreads;
+    b += (tsz * (size_t)kn * kThreads + 15) & ~(size_t)15;
     if (off_smem) b += tsz * (size_t)n_off;
     return b;
 }
@@ -965,12 +1134,13 @@ void fill_exact_params(const smiless_ctx *ctx, const smiless_plan_args *a, const
     }
     for (int v = 0; v < a->n_windows; ++v) ep.win[v] = a->windows_us[v];
     ep.rowwin = a->row_windows_us ? ctx->dW.p : nullptr;
+    for (int k = 0; k < ctx->N; ++k) ep.inst[k] = inst_of(a, k);
     for (int k = 0; k < a->n_fixed; ++k) ep.fixed[k] = a->fixed_digits[k];
 }
 
 // Per-row windows of this call (row_windows_us) or zeros: the kernels always stage the table.
 int stage_row_windows(smiless_ctx *ctx, const smiless_plan_args *a) {
-    const size_t padI = (size_t)((ctx->sumM + 3) & ~3);
+    const size_t padI = (size_t)((ctx->sumM + 1 + 3) & ~3);
     std::vector<int> w(padI, 0);
     if (a->row_windows_us) std::copy(a->row_windows_us, a->row_windows_us + ctx->sumM, w.begin());
     if (ctx->dW.p && ctx->dW.n >= padI && w == ctx->hW && !ctx->tables_dirty) return SMILESS_OK;  // unchanged
@@ -1292,6 +1462,10 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                                      ctx->dScal.p, ctx->dErr.p, ctx->dRrem.p, st);
     if (e) return cuda_fail(ctx, (cudaError_t)e, "prep_offsets launch");
     ++launches;
+    if (inst_mode(ctx, a)) {
+        e = smiless_dev_prep_tail(d_arr, a->n_arrivals, rp.d_cap, rp.K, ctx->dScal.p, st);
+        if (e) return cuda_fail(ctx, (cudaError_t)e, "prep_tail launch");
+    }
 
     const bool single = a->n_fixed == ctx->N;    // nothing left to search: one candidate
     double eval_ms = 0.0;
@@ -1301,6 +1475,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         const bool prune_mode = !(a->flags & SMILESS_FLAG_NO_PRUNE);
         const char *memo_env0 = getenv("SMILESS_MEMO");
         const bool memo_path = !prune_mode && a->n_fixed < ctx->N && (!memo_env0 || atoi(memo_env0) != 0) &&
+                               !inst_mode(ctx, a) &&
                                smem_memo_up(ctx, rp, n_off) <= 227 * 1024 &&
                                smem_memo_var(ctx, a, rp, n_off) <= 227 * 1024;
         const bool bnb_path = !memo_path && bb_depth(ctx, a) > 0 && smem_bound_bytes(ctx, a, rp, n_off) <= 227 * 1024;
@@ -1312,7 +1487,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             if ((rc = get_kernel(ctx, a, rp, n_off, families, &jk))) return rc;
         }
         hp.mark("get_kernel");
-        const u64 V = (u64)a->n_windows * (u64)configs_per_lane(ctx, a);   // candidates per unit
+        const u64 V = unit_cands(ctx, a);   // candidates per unit
         const u64 ub = cb / V, ue = (ce + V - 1) / V;
         const u64 U = ue - ub;
         const u64 n_chunks = (U + kChunkUnits - 1) / kChunkUnits;
@@ -1342,7 +1517,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         pp.cand_end = ce;
         pp.n_steps = n_steps;
         pp.n_off = n_off;
-        pp.sumM = ctx->sumM;
+        pp.sumM = kernel_rows(ctx, a);
         pp.sla = (int)a->sla_us;
         for (int s_ = 0; s_ < n_sla; ++s_) pp.slas[s_] = (int)slas[s_];
         pp.prune = (a->flags & SMILESS_FLAG_NO_PRUNE) ? 0 : 1;
@@ -1495,7 +1670,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             bp.cand_end = ce;
             bp.n_steps = n_steps;
             bp.n_off = n_off;
-            bp.sumM = ctx->sumM;
+            bp.sumM = kernel_rows(ctx, a);
             bp.sla = (int)a->sla_us;
             bp.zero = 0;
             bp.shard = shard;

@@ -52,6 +52,32 @@ __global__ void prep_offsets_kernel(const i64 *__restrict__ arr, i64 J, i64 d_ca
     }
 }
 
+// Scale-out plans (NEXT-4): scal[2 + (n-1)] = sum_{i < min(n, J)} (r_{J-1-i} - r_i) for
+// n = 1..16 (real time), scal[18 + i] = clamped offset of arrival J-1-i in the evaluator's final
+// frame (the base of the last chunk it runs: arrival K * q_last), i = 0..15.  One thread.
+__global__ void prep_tail_kernel(const i64 *__restrict__ arr, i64 J, i64 d_cap, int K, i64 *__restrict__ scal) {
+    if (blockIdx.x != 0 || threadIdx.x != 0) return;
+    const i64 n_steps = J - 1, nfc = n_steps / K;
+    const i64 q_last = nfc == 0 ? 0 : (nfc * K < n_steps ? nfc : nfc - 1);
+    const i64 jb = (i64)K * q_last;
+    i64 acc = 0;
+    for (int n = 1; n <= 16; ++n) {
+        const i64 i = n - 1;
+        if (i < J) acc += arr[J - 1 - i] - arr[i];
+        scal[2 + i] = acc;
+    }
+    for (int i = 0; i < 16; ++i) {
+        const i64 j = J - 1 - i;
+        i64 o = 0;
+        if (j >= jb) {
+            for (i64 m = jb; m < j; ++m) { const i64 g = arr[m + 1] - arr[m]; o += g < d_cap ? g : d_cap; }
+        } else if (j >= 0) {
+            for (i64 m = j; m < jb; ++m) { const i64 g = arr[m + 1] - arr[m]; o -= g < d_cap ? g : d_cap; }
+        }
+        scal[18 + i] = o;
+    }
+}
+
 __device__ __forceinline__ bool key_less(u64 ca, u64 ia, u64 cb, u64 ib) {
     return ca < cb || (ca == cb && ia < ib);
 }
@@ -80,7 +106,8 @@ __global__ void reduce_best_kernel(const u64 *__restrict__ slots, int n, int str
 }
 
 // Exact evaluation, absolute int64 times, generic DAG (runtime CSR in device memory), the
-// plain case split of model M with per-step billing -- independent of the
+// plain case split of model M (with scale-out instances, reading G26: request j
+// on instance j mod n_k, previous completion D[k][j - n_k]) with per-step billing -- independent of the
 // NVRTC evaluator's reformulations.  One WARP per candidate, lane k = function k, run as a
 // wavefront: a function's level is 1 + the highest level of its predecessors, and at
 // iteration t lane k handles invocation j = t - level_k.  Its predecessors (lower levels)
@@ -121,6 +148,7 @@ __global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParam
     const int row = p.row0[k] + cfg;
     const i64 I = act ? p.tabI[row] : 0, T = act ? p.tabT[row] : 0;
     const i64 w = act ? (p.rowwin ? p.rowwin[row] : p.win[win]) : 0;
+    const int nin = act ? p.inst[k] : 1;                // instances (request j on instance j mod nin)
     const int e0 = act ? p.pred_ptr[k] : 0, deg = act ? p.pred_ptr[k + 1] - e0 : 0;
     const bool sink = act && ((p.sinkmask >> k) & 1u);
     int pc[4];                                            // first predecessors, in registers
@@ -166,14 +194,16 @@ __global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParam
             for (int e = 4; e < deg; ++e) x = max(x, rg[p.pred_idx[e0 + e]][sl]);
             // the case split of model M as selects (lanes of one warp take different cases;
             // straight-line code keeps them converged)
-            const i64 f = D, g = x - f, s = f + w;
+            // previous completion on this request's instance: D[k][j - nin] (own ring slot,
+            // nin <= 16 < 32 so it is still there), or the register copy for one instance
+            const i64 f = nin == 1 ? D : rg[k][(j - nin) & 31], g = x - f, s = f + w;
             const bool busy = g <= 0;                     // busy: FIFO, stays warm (G6)
             const bool keep = w == 0;                     // keep-alive (Case II)
             const bool cold = x < s;                      // pre-warm not begun: cold (G3)
             const bool part = x < s + T;                  // init partly covered (G4); else covered (Case I)
             i64 start = busy ? f : keep ? x : cold ? x + T : part ? s + T : x;
             i64 bill = busy ? 0 : keep ? g : (cold || part) ? T : x - s;
-            if (j == 0) {                                 // first invocation pre-warmed (G5)
+            if (j < nin) {                                // first invocation of an instance pre-warmed (G5)
                 start = x;
                 bill = T;
             }
@@ -220,6 +250,11 @@ int smiless_dev_prep_offsets(const long long *arr, long long J, long long d_cap,
                                                                          rrem);
     else
         smiless_dev::prep_offsets_kernel<int><<<grid, bs, 0, st>>>(arr, J, d_cap, K, (int *)off, n_off, scal, err, rrem);
+    return (int)cudaGetLastError();
+}
+
+int smiless_dev_prep_tail(const long long *arr, long long J, long long d_cap, int K, long long *scal, cudaStream_t st) {
+    smiless_dev::prep_tail_kernel<<<1, 32, 0, st>>>(arr, J, d_cap, K, scal);
     return (int)cudaGetLastError();
 }
 

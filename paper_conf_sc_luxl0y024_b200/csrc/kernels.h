@@ -44,11 +44,13 @@ struct ExactParams {
     int win[SMILESS_DEV_MAX_WINDOWS];
     int fixed[SMILESS_DEV_MAX_FUNCS];
     const int *rowwin;           // per-row windows (NULL: the grid)
+    int inst[SMILESS_DEV_MAX_FUNCS];   // scale-out instances per function (>= 1, <= 16)
 };
 
 extern "C" {
 int smiless_dev_prep_offsets(const long long *arr, long long J, long long d_cap, int K, int time64, void *off,
                              long long n_off, long long *scal, int *err, long long *rrem, cudaStream_t st);
+int smiless_dev_prep_tail(const long long *arr, long long J, long long d_cap, int K, long long *scal, cudaStream_t st);
 int smiless_dev_reduce_best(const unsigned long long *slots, int n, int stride, ResBlock *res, cudaStream_t st);
 int smiless_dev_eval_exact(const ExactParams *p, cudaStream_t st);
 }

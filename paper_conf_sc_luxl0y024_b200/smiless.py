@@ -55,6 +55,7 @@ class PlanArgs(ctypes.Structure):
         ("cost_out", ctypes.c_void_p),
         ("row_windows_us", ctypes.c_void_p),
         ("cost_cap", ctypes.c_double),
+        ("instances", ctypes.c_void_p),
     ]
 
 
@@ -194,7 +195,7 @@ class Planner:
 
     # ---- args ----------------------------------------------------------------------------
     def _args(self, arrivals, sla_us, windows_us, n_fixed=0, fixed_digits=(), begin=0, end=0, flags=0,
-              shard=0, n_shards=0, cost_out=None, row_windows=None, cost_cap=None):
+              shard=0, n_shards=0, cost_out=None, row_windows=None, cost_cap=None, instances=None):
         keep = []
         if _is_device_tensor(arrivals):
             import torch
@@ -222,6 +223,10 @@ class Planner:
             rw = _i32(row_windows)
             keep.append(rw)
             a.row_windows_us = rw.ctypes.data
+        if instances is not None:
+            ins = _i32(instances)
+            keep.append(ins)
+            a.instances = ins.ctypes.data
         if cost_out is not None:
             assert cost_out.dtype == np.float64 and cost_out.flags.c_contiguous
             keep.append(cost_out)

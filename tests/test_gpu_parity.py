@@ -1009,3 +1009,117 @@ def test_every_int32_chunk_length_is_exact(K, monkeypatch):
     r = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, begin=lo, end=lo + 2048, flags=S.FLAG_NO_PRUNE, cost_out=out)
     assert not r.int64_path
     assert_dump_matches(out, oc, of)
+
+
+# ---------------------------------------------------------------------------------------
+# NEXT-4 inside model M: scale-out instances (reading G26) on every kernel path
+# ---------------------------------------------------------------------------------------
+
+def test_scale_out_golden_on_the_gpu():
+    """Golden S_E7 (hand-worked) through smiless_evaluate and smiless_plan."""
+    import json, os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "S_E7_scale_out.json")))
+    for case in g["cases"]:
+        ptr, idx = W.csr_from_preds([[]])
+        p = W.Problem("t", ptr, idx, np.ones(1, np.int32), np.asarray(case["exec_us"], np.int32),
+                      np.asarray(case["init_us"], np.int32), np.ones(1), np.asarray(case["arrivals_us"], np.int64),
+                      10**6, np.asarray(case["windows_us"], np.int32))
+        pl = S.planner_for(p)
+        c, l, f = pl.evaluate([0], p.arrivals_us, p.sla_us, p.windows_us, instances=case["instances"])
+        assert c[0] == float(sum(case["billed"])) and l[0] == max(case["latency"])
+        for flags in (0, S.FLAG_NO_PRUNE, S.FLAG_FORCE_INT64):
+            r = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, instances=case["instances"], flags=flags)
+            assert r.index == 0 and r.cost == c[0] and r.max_latency_us == l[0]
+
+
+@pytest.mark.parametrize("flags", [0, S.FLAG_NO_PRUNE, S.FLAG_FORCE_INT64, S.FLAG_NO_PRUNE | S.FLAG_FORCE_INT64])
+def test_scale_out_random_dags_per_candidate_costs(flags):
+    """Random DAGs with 1-4 round-robin instances per function (rings, prologue, virtual
+    sink, scale-out billing): every candidate's cost bits and feasibility equal the oracle's,
+    the winner is the oracle's OPT, and smiless_evaluate (the independent exact kernel)
+    agrees too."""
+    rng = np.random.default_rng(400 + flags)
+    n_checked = 0
+    for t in range(80):
+        n = int(rng.integers(1, 7))
+        p = W.random_problem(rng, n, 4, int(rng.integers(1, 5)), int(rng.integers(1, 140)))
+        space = p.space_size()
+        if space > 20000:
+            continue
+        inst = [int(rng.integers(1, 5)) for _ in range(n)]
+        o = OracleProblem(p, instances=inst)
+        idx = np.arange(space, dtype=np.uint64)
+        oc, ol, of = o.evaluate(idx)
+        pl = S.planner_for(p)
+        out = np.empty(space)
+        g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=flags, cost_out=out, instances=inst)
+        assert_dump_matches(out, oc, of)
+        assert_same_plan(g, o.plan(), o)
+        gc, gl, gf = pl.evaluate(idx[:512], p.arrivals_us, p.sla_us, p.windows_us, instances=inst)
+        assert_same_eval(gc, gl, gf, oc[:512], ol[:512], of[:512])
+        n_checked += 1
+        if n_checked == 25:
+            break
+    assert n_checked >= 15
+
+
+def test_scale_out_branch_and_bound_and_shards(monkeypatch):
+    """B&B depths with scale-out functions (lower-bound relaxation downstream of them),
+    2 shards, and the cost bound: per-candidate parity and the oracle's OPT."""
+    rng = np.random.default_rng(77)
+    n_checked = 0
+    for t in range(40):
+        n = int(rng.integers(4, 7))
+        p = W.random_problem(rng, n, 3, int(rng.integers(2, 4)), int(rng.integers(20, 120)),
+                             sla_us=int(rng.integers(15_000, 60_000)))
+        space = p.space_size()
+        if space > 30000:
+            continue
+        inst = [int(rng.integers(1, 4)) for _ in range(n)]
+        o = OracleProblem(p, instances=inst)
+        oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
+        ref = o.plan()
+        for d in range(2, n):
+            for da in (0, 1):
+                if da >= d:
+                    continue
+                monkeypatch.setenv("SMILESS_BB_DEPTH", str(d))
+                monkeypatch.setenv("SMILESS_BB_DEPTH_A", str(da))
+                pl = S.planner_for(p)
+                out = np.empty(space)
+                g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, cost_out=out, instances=inst)
+                assert_dump_matches(out, oc, of)
+                assert_same_plan(g, ref, o)
+                g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, instances=inst)      # cost bound on
+                assert_same_plan(g, ref, o)
+                parts = [pl.plan(p.arrivals_us, p.sla_us, p.windows_us, shard=s_, n_shards=2, instances=inst)
+                         for s_ in range(2)]
+                assert sum(r.n_decided for r in parts) == space
+                win = [(r.cost, r.index) for r in parts if r.feasible]
+                assert (min(win) if win else None) == (None if ref is None else (ref[1], ref[0]))
+        n_checked += 1
+        if n_checked == 8:
+            break
+    assert n_checked >= 5
+
+
+@pytest.mark.parametrize("K", ["64", "16", "8"])
+def test_scale_out_chunk_lengths(K, monkeypatch):
+    """The prologue must sit inside chunk 0 (K >= prologue) and the rings span chunk
+    rebases: forced K with up to 8 instances (prologue 8) against the oracle."""
+    monkeypatch.setenv("SMILESS_FORCE_K", K)
+    rng = np.random.default_rng(500 + int(K))
+    for t in range(30):
+        n = int(rng.integers(1, 5))
+        p = W.random_problem(rng, n, 3, int(rng.integers(1, 4)), int(rng.integers(2, 100)))
+        space = p.space_size()
+        if space > 8000:
+            continue
+        inst = [int(rng.integers(1, 9)) for _ in range(n)]
+        o = OracleProblem(p, instances=inst)
+        oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
+        pl = S.planner_for(p)
+        for flags in (0, S.FLAG_NO_PRUNE):
+            out = np.empty(space)
+            pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=flags, cost_out=out, instances=inst)
+            assert_dump_matches(out, oc, of)

@@ -546,3 +546,96 @@ def test_cost_is_left_to_right_without_fma_for_paper_prices():
     for k in (1, 0):
         rl = rnd(Fraction(rl) + Fraction(rnd(U[k] * E[k])))
     assert rl.hex() == g["right_to_left_cost_hex"]
+
+
+# ---------------------------------------------------------------------------
+# NEXT-4 scale-out inside model M (reading G26: n_k round-robin instances)
+# ---------------------------------------------------------------------------
+
+def test_scale_out_worked_example():
+    """Golden S_E7: one function on 1, 2, 3 instances under a Case III burst,
+    and 2 instances with pre-warm windows (covered and partly covered)."""
+    g = _golden("S_E7_scale_out.json")
+    for case in g["cases"]:
+        p = mk([[]], case["exec_us"], case["init_us"], case["arrivals_us"], case["windows_us"])
+        billed, lat = OracleProblem(p, instances=case["instances"]).simulate([0], case["window_idx"])
+        assert billed.tolist() == case["billed"], case
+        assert lat.tolist() == case["latency"], case
+        b2, l2 = des.simulate(p, [0], case["window_idx"], instances=case["instances"])
+        assert b2 == case["billed"] and l2 == case["latency"]
+
+
+def test_scale_out_oracle_matches_event_driven_simulator():
+    """Random DAGs with 1-4 instances per function: the oracle's case split on
+    D[k][j - n_k] equals the DES running n_k explicit instance state machines."""
+    rng = np.random.default_rng(23)
+    for _ in range(1500):
+        n = int(rng.integers(1, 7))
+        p = W.random_problem(rng, n, 3, int(rng.integers(1, 5)), int(rng.integers(1, 16)))
+        inst = [int(rng.integers(1, 5)) for _ in range(n)]
+        o = OracleProblem(p, instances=inst)
+        c = [int(rng.integers(0, p.n_configs[k])) for k in range(n)]
+        w = [int(rng.integers(0, len(p.windows_us))) for k in range(n)]
+        billed, lat = o.simulate(c, w)
+        b2, l2 = des.simulate(p, c, w, instances=inst)
+        assert billed.tolist() == b2
+        assert lat.tolist() == l2
+
+
+def test_scale_out_keepalive_is_fcfs_multiserver_queue():
+    """Textbook G/D/c: with keep-alive, deterministic service I and sorted arrivals, n
+    round-robin instances serve each request exactly when the FCFS c-server queue does
+    (the request starts at max(arrival, earliest server release); a heap of release
+    times), so the completion times (latency) agree."""
+    import heapq
+    rng = np.random.default_rng(29)
+    for _ in range(400):
+        c = int(rng.integers(1, 6))
+        J = int(rng.integers(1, 60))
+        I = int(rng.integers(1, 500))
+        arr = np.cumsum(rng.integers(0, 300, size=J)).astype(np.int64)
+        p = mk([[]], [I], [int(rng.integers(0, 200))], arr, [0])
+        billed, lat = OracleProblem(p, instances=[c]).simulate([0], [0])
+        free = [int(arr[0])] * c                        # every server ready at the first arrival (G5)
+        heapq.heapify(free)
+        want = []
+        for a in arr:
+            s = max(int(a), heapq.heappop(free))
+            heapq.heappush(free, s + I)
+            want.append(s + I - int(a))
+        assert lat.tolist() == want
+
+
+def test_scale_out_periodic_closed_forms():
+    """Periodic arrivals (period IT) with keep-alive on n instances, I <= n IT (no
+    queueing: L = sum of I): every request's latency is the chain's sum of I, and
+    each instance bills T + I + (its last - its first request) IT; with n >= J every
+    request is an instance's first: billed = J (T + I)."""
+    rng = np.random.default_rng(31)
+    for _ in range(200):
+        K = int(rng.integers(1, 4))
+        J = int(rng.integers(1, 40))
+        n = int(rng.integers(1, 6))
+        IT = int(rng.integers(100, 1000))
+        I = [int(rng.integers(1, n * IT // K + 1)) for _ in range(K)]
+        T = [int(rng.integers(0, 500)) for _ in range(K)]
+        p = mk([[]] + [[k] for k in range(K - 1)], I, T, [j * IT for j in range(J)], [0])
+        billed, lat = OracleProblem(p, instances=[n] * K).simulate([0] * K, [0] * K)
+        assert lat.tolist() == [sum(I)] * J
+        for k in range(K):
+            want = sum(T[k] + I[k] + ((J - 1 - i) // n * n) * IT for i in range(min(n, J)))
+            assert billed[k] == want
+        big = OracleProblem(p, instances=[J] * K).simulate([0] * K, [0] * K)[0]
+        assert big.tolist() == [J * (T[k] + I[k]) for k in range(K)]
+
+
+def test_scale_out_one_instance_is_model_m():
+    """instances = [1] * N is exactly the single-instance model (every existing pin)."""
+    rng = np.random.default_rng(37)
+    for _ in range(300):
+        n = int(rng.integers(1, 6))
+        p = W.random_problem(rng, n, 3, int(rng.integers(1, 4)), int(rng.integers(1, 30)))
+        o1, o2 = OracleProblem(p), OracleProblem(p, instances=[1] * n)
+        idx = np.arange(min(p.space_size(), 64), dtype=np.uint64)
+        a, b = o1.evaluate(idx), o2.evaluate(idx)
+        assert all(np.array_equal(x.view(np.uint8), y.view(np.uint8)) for x, y in zip(a, b))
