@@ -67,13 +67,16 @@ def configs_per_lane(p) -> int:
     return G
 
 
-def algorithmic_ops_per_candidate(p, memo: bool = True) -> float:
+def algorithmic_ops_per_candidate(p, memo: bool = True, split: bool = True) -> float:
     """Integer ops per candidate over the whole horizon for the algorithm as implemented
     (DESIGN.md "Roofline").  Per invocation j >= 1:
       upstream, once per prefix (memo) or per lane-unit: 7 per function-step (g, u, delta,
         busy mask, masked update, +I, sum u), +1 per extra join input, +1 per upstream sink;
       per last-function config 3 shared ops (x + CN, CN += -I, o + CN);
       per window variant 7 (g, u, delta, mask, update, sum u, latency), 4 for keep-alive;
+      with the split cost (default, memo path): 6 per window variant -- the sum of u is not
+      carried through the walk; the few units holding a feasible candidate are re-walked
+      with it, which this count leaves out (it only lowers `achieved`);
     divided by the candidates sharing each part (prefix: M_{N-1} x W, unit: G x W)."""
     n = p.n_funcs
     Wn = len(p.windows_us)
@@ -83,7 +86,7 @@ def algorithmic_ops_per_candidate(p, memo: bool = True) -> float:
     up_sinks = sum(1 for k in range(n - 1) if k not in listed)
     w0 = 1 if int(p.windows_us[0]) == 0 else 0
     upstream = 7 * (n - 1) + joins + up_sinks
-    per_unit = G * (3 + 4 * w0 + 7 * (Wn - w0))
+    per_unit = G * (3 + 4 * w0 + (6 if (memo and split) else 7) * (Wn - w0))
     up_share = int(p.n_configs[-1]) * Wn if memo else G * Wn
     per_cand_step = upstream / up_share + per_unit / (G * Wn)
     return per_cand_step * (len(p.arrivals_us) - 1)
@@ -509,7 +512,8 @@ def main():
     sm_mhz = clocks["sm_mhz"] or peaks.get("sm_max_mhz", 1965.0)
     peak_ops = props.multi_processor_count * ISSUE_LANES_PER_CLK_PER_SM * float(clocks["sm_max_mhz"] or 1965.0) * 1e6
     memo = os.environ.get("SMILESS_MEMO", "1") != "0"
-    ops_per_cand = algorithmic_ops_per_candidate(p, memo=memo)
+    split = os.environ.get("SMILESS_SPLITCOST", "1") != "0"
+    ops_per_cand = algorithmic_ops_per_candidate(p, memo=memo, split=split)
     ops = ops_per_cand * res.n_decided
     kernel_ms_per_step = kernel_ms / args.steps
     achieved = ops / (kernel_ms_per_step / 1e3)

@@ -171,6 +171,10 @@ typedef struct {
     double total_device_ms;   /* device time of the whole call (first upload .. last kernel)      */
     int32_t int64_path;       /* 1 if the int64 evaluator ran (int32 range check failed / forced)  */
     int32_t launches;         /* kernels this call launched                                        */
+    uint64_t h2d_bytes;       /* host -> device bytes this call copied (inputs: arrivals unless on
+                                 the device, windows / tables when changed, counts, caps)          */
+    uint64_t d2h_bytes;       /* device -> host bytes this call copied (result block, counts,
+                                 cost_out)                                                         */
 } smiless_plan_result;
 
 /* Size of the suffix candidate space prod_{k >= n_fixed} M_k * W.
@@ -230,6 +234,18 @@ typedef struct {
 SMILESS_API int smiless_autoscale(const smiless_ctx *ctx, const double *slope_us, const double *intercept_us,
                                   const int64_t *invocations, int64_t it_us, const int64_t *target_us,
                                   smiless_autoscale_result *out);
+
+/* NEXT-4, per configuration: the Eq. (7)/(8) constraint of the auto-scaler solved for every
+ * (function, configuration) row: batch_out[row] = the largest B in [1, G_k] with
+ * slope_us[row] * B + intercept_us[row] <= target_us[k] (bisection; IEEE, no FMA), and
+ * instances_out[row] = ceil(G_k / B); both 0 when even B = 1 misses the target or G_k <= 0.
+ * The instance count of a function's fastest configuration is the smallest scale-out with
+ * which it can keep up with a predicted peak of G_k invocations per window; it is what the
+ * scale-out plans of smiless_plan_args.instances use (reading G26).  Host-only.
+ * Returns OK, ESTATE or EINVAL. */
+SMILESS_API int smiless_autoscale_rows(const smiless_ctx *ctx, const double *slope_us, const double *intercept_us,
+                                       const int64_t *invocations, const int64_t *target_us, int64_t *batch_out,
+                                       int64_t *instances_out);
 
 /* NEXT-3: SMIless's handling of complex DAGs: decompose the DAG into its
  * source-to-sink paths (subgraphs with only sequential dependencies), optimise each path

@@ -31,3 +31,24 @@ def autoscale(prob, slope, intercept, invocations, it_us, target_us):
                     break
         out.append(best)
     return out
+
+
+def autoscale_rows(prob, slope, intercept, invocations, target_us):
+    """Eq. (7)/(8) constraint per (function, configuration) row by brute force: the largest
+    B in [1, G] with slope * B + intercept <= I_s, and ceil(G / B) instances; (0, 0) when
+    even B = 1 misses I_s or G <= 0."""
+    off = [0]
+    for m in prob.n_configs:
+        off.append(off[-1] + int(m))
+    batch, inst = [], []
+    for k in range(prob.n_funcs):
+        G = int(invocations[k])
+        for c in range(int(prob.n_configs[k])):
+            r = off[k] + c
+            best = 0
+            for B in range(1, G + 1):
+                if float(slope[r]) * float(B) + float(intercept[r]) <= float(target_us[k]):
+                    best = B
+            batch.append(best)
+            inst.append(-(-G // best) if best else 0)
+    return batch, inst

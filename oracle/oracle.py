@@ -85,6 +85,8 @@ class OracleProblem:
     def __init__(self, prob, sla_us: Optional[int] = None, n_fixed: int = 0,
                  fixed_digits: Sequence[int] = (), row_windows: Optional[Sequence[int]] = None,
                  instances: Optional[Sequence[int]] = None):
+        if instances is None:
+            instances = getattr(prob, "instances", None)   # the workload's scale-out counts
         """row_windows (optional, [sum M]): the window of each (function, config) row, used
         instead of the grid (windows_us must then hold a single entry) -- the paper's
         derived pre-warm windows (NEXT-1).  instances (optional, [N]): n_k round-robin

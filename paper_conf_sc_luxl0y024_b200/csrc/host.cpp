@@ -355,6 +355,7 @@ struct smiless_ctx {
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
 
     std::map<std::string, JitKernel> jit_cache;
+    u64 h2d = 0, d2h = 0;        // host<->device bytes copied by the current plan call
 };
 
 namespace {
@@ -436,6 +437,8 @@ int upload_tables(smiless_ctx *ctx) {
     // non-blocking stream (not ordered after the legacy default stream).  The pageable
     // sources are staged before cudaMemcpyAsync returns, so the local vectors may go.
     cudaStream_t st = ctx->stream;
+    ctx->h2d += 3 * padI * sizeof(int) + padU * sizeof(double) + ctx->pred_ptr.size() * sizeof(int) +
+                ctx->pred_idx.size() * sizeof(int);
     CK(cudaMemcpyAsync(ctx->dI.p, I.data(), padI * sizeof(int), cudaMemcpyHostToDevice, st), "H2D tables");
     CK(cudaMemcpyAsync(ctx->dNI.p, NI.data(), padI * sizeof(int), cudaMemcpyHostToDevice, st), "H2D tables");
     CK(cudaMemcpyAsync(ctx->dT.p, T.data(), padI * sizeof(int), cudaMemcpyHostToDevice, st), "H2D tables");
@@ -707,13 +710,13 @@ u64 cands_per_prefix(const smiless_ctx *ctx, const smiless_plan_args *a, int d) 
 
 enum { FAM_PLAN = 1, FAM_BOUND = 2, FAM_MEMO = 4, FAM_ALL = 7 };   // kernel families of a module
 
-// Throughput mode with prefix memoisation, SMILESS_SPLITCOST=1: walk every unit without the
-// sum-of-u accumulators and re-walk only the units holding a feasible candidate to finish
-// their costs (DESIGN.md section 5 item 12).  Off by default (measured +3 % candidates/s on
-// the C2 slice, profiles/r01k_sweep_variants.md).
+// Throughput mode with prefix memoisation: walk every unit without the sum-of-u accumulators
+// and re-walk only the units holding a feasible candidate to finish their costs (DESIGN.md
+// section 5 item 12; +3 % candidates/s on the C2 slice).  On by default; SMILESS_SPLITCOST=0
+// walks every unit with the accumulators in one pass.
 bool split_cost() {
     const char *e = getenv("SMILESS_SPLITCOST");
-    return e && atoi(e) != 0;
+    return !e || atoi(e) != 0;
 }
 
 // static cost-bound terms of every (row, window) staged in shared memory when small
@@ -1146,6 +1149,7 @@ int stage_row_windows(smiless_ctx *ctx, const smiless_plan_args *a) {
     if (ctx->dW.p && ctx->dW.n >= padI && w == ctx->hW && !ctx->tables_dirty) return SMILESS_OK;  // unchanged
     CK(ctx->dW.ensure(padI), "cudaMalloc row windows");
     CK(cudaMemcpyAsync(ctx->dW.p, w.data(), padI * sizeof(int), cudaMemcpyHostToDevice, ctx->stream), "H2D windows");
+    ctx->h2d += padI * sizeof(int);
     ctx->hW.swap(w);
     return SMILESS_OK;
 }
@@ -1157,6 +1161,7 @@ int stage_arrivals(smiless_ctx *ctx, const smiless_plan_args *a, const i64 **d_a
         return SMILESS_OK;
     }
     CK(ctx->dArr.ensure((size_t)a->n_arrivals), "cudaMalloc arrivals");
+    ctx->h2d += (size_t)a->n_arrivals * sizeof(i64);
     CK(cudaMemcpyAsync(ctx->dArr.p, a->arrivals_us, (size_t)a->n_arrivals * sizeof(i64), cudaMemcpyHostToDevice,
                        ctx->stream),
        "H2D arrivals");
@@ -1418,6 +1423,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     if (!a_in) return fail(ctx, SMILESS_EINVAL, "args is NULL");
     HostProf hp;
     NvtxRange nv_plan("smiless_plan");
+    ctx->h2d = ctx->d2h = 0;
     smiless_plan_args a_copy = *a_in;
     i64 sla_max = slas[0];
     for (int s_ = 1; s_ < n_sla; ++s_) sla_max = std::max<i64>(sla_max, slas[s_]);
@@ -1534,6 +1540,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 memcpy(&pp.cap, &c, 8);
             }
             CK(cudaMemcpyAsync(ctx->dInc.p, &pp.cap, 8, cudaMemcpyHostToDevice, st), "H2D incumbent");
+            ctx->h2d += 8;
         }
         pp.shard = shard;
         pp.n_shards = n_shards;
@@ -1744,6 +1751,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                     unsigned n_a = 0;
                     hp.mark("launch_a");
                     CK(cudaMemcpyAsync(&n_a, ctx->dListCntA.p, sizeof n_a, cudaMemcpyDeviceToHost, st), "D2H count");
+                    ctx->d2h += sizeof n_a;
                     CK(cudaStreamSynchronize(st), "count");
                     hp.mark("sync_a");
                     // deep launches (first survivor entry, entries, first child, children per entry):
@@ -1769,6 +1777,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                     std::vector<unsigned> cnts(std::max<size_t>(L.size(), 1), 0u);
                     for (size_t i = 0; i < L.size(); ++i) cnts[i] = L[i].ne;
                     CK(ctx->dChunkCnt.ensure(cnts.size()), "cudaMalloc counts");
+                    ctx->h2d += cnts.size() * sizeof(unsigned);
                     CK(cudaMemcpyAsync(ctx->dChunkCnt.p, cnts.data(), cnts.size() * sizeof(unsigned),
                                        cudaMemcpyHostToDevice, st),
                        "H2D counts");
@@ -1878,6 +1887,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         }
         CK(cudaMemcpyAsync(&ctx->dRes.p->stats[0], ctx->dStats.p, 16, cudaMemcpyDeviceToDevice, st), "D2D stats");
         if (a->cost_out)
+            ctx->d2h += (size_t)(ce - cb) * sizeof(double);
             CK(cudaMemcpyAsync(a->cost_out, ctx->dDump.p, (size_t)(ce - cb) * sizeof(double), cudaMemcpyDeviceToHost, st),
                "D2H dump");
     } else if (single && ce > cb) {
@@ -1904,6 +1914,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     }
     CK(cudaMemcpyAsync(&ctx->dRes.p->err, ctx->dErr.p, sizeof(int), cudaMemcpyDeviceToDevice, st), "D2D err");
     CK(cudaMemcpyAsync(ctx->hRes, ctx->dRes.p, sizeof(ResBlock) * n_sla, cudaMemcpyDeviceToHost, st), "D2H result");
+    ctx->d2h += sizeof(ResBlock) * n_sla;
     CK(cudaEventRecord(ctx->ev[3], st), "event");
     hp.mark("tail_launched");
     CK(cudaStreamSynchronize(st), "plan");
@@ -1946,6 +1957,8 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         r.total_device_ms = tot;
         r.int64_path = rp.time64 ? 1 : 0;
         r.launches = launches;
+        r.h2d_bytes = ctx->h2d;
+        r.d2h_bytes = ctx->d2h;
         int32_t *co = config_out ? config_out + (size_t)s_ * ctx->N : nullptr;
         int32_t *wo = window_out ? window_out + (size_t)s_ * ctx->N : nullptr;
         if (!found) {
@@ -2126,6 +2139,37 @@ int smiless_autoscale(const smiless_ctx *ctx, const double *slope_us, const doub
             if (cost < best.cost) best = smiless_autoscale_result{c, lo, inst, cost};
         }
         out[k] = best;
+    }
+    return SMILESS_OK;
+}
+
+int smiless_autoscale_rows(const smiless_ctx *ctx, const double *slope_us, const double *intercept_us,
+                           const int64_t *invocations, const int64_t *target_us, int64_t *batch_out,
+                           int64_t *instances_out) {
+    if (!ctx || !slope_us || !intercept_us || !invocations || !target_us || !batch_out || !instances_out)
+        return SMILESS_EINVAL;
+    if (!ctx->dag_loaded || !ctx->prof_loaded) return SMILESS_ESTATE;
+    for (int k = 0; k < ctx->N; ++k) {
+        const i64 G = invocations[k];
+        for (int c = 0; c < ctx->M[k]; ++c) {
+            const int row = ctx->row0[k] + c;
+            const double sl = slope_us[row], ic = intercept_us[row], lim = (double)target_us[k];
+            auto ok = [&](i64 B) {
+                volatile double prod = sl * (double)B;   // two rounded operations, never an FMA
+                return prod + ic <= lim;
+            };
+            batch_out[row] = 0;
+            instances_out[row] = 0;
+            if (G <= 0 || !ok(1)) continue;
+            i64 lo = 1, hi = G;                            // bisection: largest feasible B
+            while (lo < hi) {
+                const i64 mid = lo + (hi - lo + 1) / 2;
+                if (ok(mid)) lo = mid;
+                else hi = mid - 1;
+            }
+            batch_out[row] = lo;
+            instances_out[row] = (G + lo - 1) / lo;
+        }
     }
     return SMILESS_OK;
 }

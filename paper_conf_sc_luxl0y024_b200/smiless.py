@@ -26,7 +26,7 @@ _NAMES = {0: "OK", 1: "INFEASIBLE", -1: "EINVAL", -2: "ENOTTOPO", -3: "ERANGE", 
 EXPORTS = ("smiless_create", "smiless_set_stream", "smiless_destroy", "smiless_last_error",
            "smiless_load_dag", "smiless_load_profiles", "smiless_space_size", "smiless_plan",
            "smiless_plan_sla_sweep", "smiless_derive_windows", "smiless_top1_search", "smiless_decompose_search",
-           "smiless_autoscale",
+           "smiless_autoscale", "smiless_autoscale_rows",
            "smiless_evaluate",
            "smiless_decode",
            "smiless_kernel_source", "smiless_jit_compile")
@@ -70,6 +70,8 @@ class PlanResultC(ctypes.Structure):
         ("total_device_ms", ctypes.c_double),
         ("int64_path", ctypes.c_int32),
         ("launches", ctypes.c_int32),
+        ("h2d_bytes", ctypes.c_uint64),
+        ("d2h_bytes", ctypes.c_uint64),
     ]
 
 
@@ -87,6 +89,8 @@ class PlanResult:
     total_device_ms: float
     int64_path: bool
     launches: int
+    h2d_bytes: int = 0          # host -> device bytes the call copied (counted by the library)
+    d2h_bytes: int = 0          # device -> host bytes the call copied
 
     @property
     def feasible(self) -> bool:
@@ -121,6 +125,7 @@ def load_library(build_if_missing: bool = True):
                                            vp, vp]
     lib.smiless_derive_windows.argtypes = [vp, i64, vp]
     lib.smiless_autoscale.argtypes = [vp, vp, vp, vp, i64, vp, vp]
+    lib.smiless_autoscale_rows.argtypes = [vp, vp, vp, vp, vp, vp, vp]
     lib.smiless_decompose_search.argtypes = [vp, ctypes.POINTER(PlanArgs), i64, ctypes.POINTER(PlanResultC), vp,
                                              vp, ctypes.POINTER(ctypes.c_int64)]
     lib.smiless_top1_search.argtypes = [vp, ctypes.POINTER(PlanArgs), i64, ctypes.POINTER(PlanResultC), vp, vp,
@@ -157,6 +162,7 @@ class Planner:
             raise SmilessError(rc, self._lib.smiless_last_error(None).decode())
         self._keep = []
         self.n_funcs = 0
+        self.default_instances = None    # scale-out instances used when a call passes none
 
     def close(self):
         if self._ctx:
@@ -196,6 +202,8 @@ class Planner:
     # ---- args ----------------------------------------------------------------------------
     def _args(self, arrivals, sla_us, windows_us, n_fixed=0, fixed_digits=(), begin=0, end=0, flags=0,
               shard=0, n_shards=0, cost_out=None, row_windows=None, cost_cap=None, instances=None):
+        if instances is None:
+            instances = self.default_instances
         keep = []
         if _is_device_tensor(arrivals):
             import torch
@@ -254,6 +262,19 @@ class Planner:
                                                 int(it_us), tg.ctypes.data, out.ctypes.data))
         return out
 
+    def autoscale_rows(self, slope_us, intercept_us, invocations, target_us):
+        """Eq. (7)/(8) per (function, configuration) row (smiless_autoscale_rows): the largest
+        batch B and the instances ceil(G/B) (0, 0 when infeasible)."""
+        sl = np.ascontiguousarray(np.asarray(slope_us, dtype=np.float64))
+        ic = np.ascontiguousarray(np.asarray(intercept_us, dtype=np.float64))
+        G = np.ascontiguousarray(np.asarray(invocations, dtype=np.int64))
+        tg = np.ascontiguousarray(np.asarray(target_us, dtype=np.int64))
+        b = np.zeros(self._n_rows, np.int64)
+        n = np.zeros(self._n_rows, np.int64)
+        self._check(self._lib.smiless_autoscale_rows(self._ctx, sl.ctypes.data, ic.ctypes.data, G.ctypes.data,
+                                                     tg.ctypes.data, b.ctypes.data, n.ctypes.data))
+        return b, n
+
     def space_size(self, n_windows: int, n_fixed: int = 0) -> int:
         out = ctypes.c_uint64()
         self._check(self._lib.smiless_space_size(self._ctx, int(n_windows), int(n_fixed), ctypes.byref(out)))
@@ -271,7 +292,8 @@ class Planner:
                           max_latency_us=int(r.max_latency_us), config=cfg[:self.n_funcs],
                           window=win[:self.n_funcs], n_decided=int(r.n_decided), n_full_evals=int(r.n_full_evals),
                           eval_kernel_ms=float(r.eval_kernel_ms), total_device_ms=float(r.total_device_ms),
-                          int64_path=bool(r.int64_path), launches=int(r.launches))
+                          int64_path=bool(r.int64_path), launches=int(r.launches),
+                          h2d_bytes=int(r.h2d_bytes), d2h_bytes=int(r.d2h_bytes))
 
     def plan_sla_sweep(self, arrivals, slas_us, windows_us, **kw):
         """One pass over the space, one winner per SLA (smiless_plan_sla_sweep)."""
@@ -373,8 +395,10 @@ class Planner:
 
 
 def planner_for(problem, device: int = 0, stream: Optional[int] = None) -> Planner:
-    """Planner with a workloads.Problem-like object's DAG and profiles loaded."""
+    """Planner with a workloads.Problem-like object's DAG and profiles loaded; the problem's
+    scale-out instance counts (if any) become the default `instances` of every call."""
     p = Planner(device, stream)
+    p.default_instances = getattr(problem, "instances", None)
     p.load_dag(problem.pred_ptr, problem.pred_idx)
     p.load_profiles(problem.n_configs, problem.exec_us, problem.init_us, problem.price_per_us)
     return p

@@ -264,6 +264,7 @@ def test_bench_configuration_split_cost_same_result(monkeypatch):
     import bench
     p, kw = bench.workload("C2")
     pl = S.planner_for(p)
+    monkeypatch.setenv("SMILESS_SPLITCOST", "0")
     one = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=S.FLAG_NO_PRUNE, **kw)
     monkeypatch.setenv("SMILESS_SPLITCOST", "1")
     two = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=S.FLAG_NO_PRUNE, **kw)
@@ -928,11 +929,11 @@ def test_full_space_plan_shards_split_the_work(name, world):
 
 
 def test_c5_heavy_subplan_children_split_over_launches():
-    """C5's sub-plan of function 0's digit 112 (2^63 candidates): its shallow survivors have
+    """C5s's sub-plan of function 0's digit 112 (2^63 candidates): its shallow survivors have
     2^28 deep children each, more than one survivor list holds, so their children run over
     several deep launches.  Single rank and 2 shards agree; the oracle re-checks the winner."""
     import torch
-    p = W.make_config("C5")
+    p = W.make_config("C5s")
     pl = S.planner_for(p)
     arr = torch.as_tensor(p.arrivals_us).cuda()
     kw = dict(n_fixed=1, fixed_digits=[112])
@@ -950,7 +951,14 @@ def test_c5_heavy_subplan_children_split_over_launches():
 # int32 chunk length K
 # ---------------------------------------------------------------------------------------
 
-@pytest.mark.parametrize("name,nf,fixed", [("C2", 0, []), ("C3", 0, []), ("C5", 1, [112])])
+def _fastest_digit0(p):
+    """Digit of function 0 on its fastest configuration, keep-alive (a feasible sub-space of
+    C5 with scale-out)."""
+    return int(np.argmin(p.exec_us[:int(p.n_configs[0])])) * len(p.windows_us)
+
+
+@pytest.mark.parametrize("name,nf,fixed", [("C2", 0, []), ("C3", 0, []), ("C3s", 0, []), ("C5s", 1, [112]),
+                                           ("C5", 1, None)])
 def test_full_size_per_candidate_costs_around_opt(name, nf, fixed):
     """P:305 (OPT by exhaustive search): 4,096 consecutive candidates around the exact plan's
     winner at the full J = 10^4, evaluated by the memoised throughput kernels (no pruning)
@@ -958,6 +966,8 @@ def test_full_size_per_candidate_costs_around_opt(name, nf, fixed):
     oracle.  C5 pins function 0's digit (its space is 2^70)."""
     import torch
     p = W.make_config(name)
+    if fixed is None:
+        fixed = [_fastest_digit0(p)]
     kw = dict(n_fixed=nf, fixed_digits=fixed)
     pl = S.planner_for(p)
     arr = torch.as_tensor(p.arrivals_us).cuda()
@@ -1123,3 +1133,23 @@ def test_scale_out_chunk_lengths(K, monkeypatch):
             out = np.empty(space)
             pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=flags, cost_out=out, instances=inst)
             assert_dump_matches(out, oc, of)
+
+
+def test_c2_window0_subspace_matches_oracle_brute_force():
+    """tests/golden/C2_window0_bruteforce.json: the plain oracle walked every one of the
+    16^6 keep-alive candidates of C2 at J = 10^4 (tools/c2_window0_bruteforce.py, ~46 min on
+    8 cores).  The GPU plan of that sub-space returns the same index and cost bits, and the
+    full 2^42 plan's OPT is that same candidate (C2's optimum keeps every function alive)."""
+    import json, os
+    import torch
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "C2_window0_bruteforce.json")))
+    p = W.make_config("C2")
+    pl = S.planner_for(p)
+    arr = torch.as_tensor(p.arrivals_us).cuda()
+    for flags in (0, S.FLAG_NO_PRUNE):
+        r = pl.plan(arr, p.sla_us, p.windows_us[:1], flags=flags)
+        assert r.index == g["index_subspace"] and r.cost.hex() == g["cost_hex"]
+        assert r.max_latency_us == g["max_latency_us"] and r.n_decided == g["space"]
+    full = pl.plan(arr, p.sla_us, p.windows_us)
+    assert full.index == g["index_full_space"] and full.cost.hex() == g["cost_hex"]
+    assert full.config.tolist() == g["config"] and (full.window == 0).all()

@@ -639,3 +639,23 @@ def test_scale_out_one_instance_is_model_m():
         idx = np.arange(min(p.space_size(), 64), dtype=np.uint64)
         a, b = o1.evaluate(idx), o2.evaluate(idx)
         assert all(np.array_equal(x.view(np.uint8), y.view(np.uint8)) for x, y in zip(a, b))
+
+
+@pytest.mark.parametrize("name", ["C3", "C5"])
+def test_workload_instances_are_the_autoscalers(name):
+    """The scale-out instance counts of C3 / C5 (workloads.SCALE_OUT_INSTANCES, inputs of
+    model M) are the paper's auto-scaler constraint (Eq. (7)/(8)) at each
+    function's fastest configuration for the predicted peak G per 1-s window with
+    IT = I_s = 1 s: the oracle's brute force and the library's bisection both give them."""
+    from oracle.autoscale import autoscale_rows
+    from paper_conf_sc_luxl0y024_b200 import smiless as S
+    p = W.make_config(name)
+    G = W.peak_window_count(p.arrivals_us)
+    n = p.n_funcs
+    b_o, n_o = autoscale_rows(p, p.batch_slope_us, p.batch_intercept_us, [G] * n, [10**6] * n)
+    pl = S.planner_for(p)
+    b_l, n_l = pl.autoscale_rows(p.batch_slope_us, p.batch_intercept_us, [G] * n, [10**6] * n)
+    assert list(b_l) == b_o and list(n_l) == n_o
+    off = np.concatenate([[0], np.cumsum(p.n_configs)])
+    fastest = [off[k] + int(np.argmin(p.exec_us[off[k]:off[k + 1]])) for k in range(n)]
+    assert [n_o[r] for r in fastest] == list(W.SCALE_OUT_INSTANCES[name]) == list(p.instances)

@@ -135,12 +135,10 @@ def poisson_arrivals(rng: np.random.Generator, n: int, rate_per_s: float) -> np.
     return np.cumsum(gaps)
 
 
-def mmpp_arrivals(rng: np.random.Generator, n: int, rates=(0.2, 3.0), dwell_s=(60.0, 5.0)) -> np.ndarray:
-    """Bursty 2-state Markov-modulated Poisson process (15x rate bursts of ~5 s).
-
-    The burst rate is chosen so that the fastest single-instance configuration of C3 still
-    meets the 2 s SLA (model M serves each function with one FIFO instance; scale-out is
-    the autoscaler, NEXT-4): at 10 req/s bursts every candidate is infeasible."""
+def mmpp_arrivals(rng: np.random.Generator, n: int, rates=(0.2, 10.0), dwell_s=(60.0, 5.0)) -> np.ndarray:
+    """Bursty 2-state Markov-modulated Poisson process: 0.2 req/s, mean dwell 60 s, and
+    10 req/s bursts of mean 5 s.  C3 serves the bursts with scale-out
+    instances (NEXT-4); the single-instance variant C3s softens the bursts to 3 req/s."""
     out = np.empty(n, dtype=np.int64)
     t = 0.0
     state = 0
@@ -162,7 +160,7 @@ def mmpp_arrivals(rng: np.random.Generator, n: int, rates=(0.2, 3.0), dwell_s=(6
 
 
 def azure_arrivals(rng: np.random.Generator, n: int, mean_per_window: float = 0.25,
-                   vmr: float = 2.2, period_windows: int = 720) -> np.ndarray:
+                   vmr: float = 3.0, period_windows: int = 720) -> np.ndarray:
     """Azure-Functions-shaped: per-1-s-window counts, negative
     binomial with variance/mean = vmr >= 2 under a sinusoidal
     diurnal envelope compressed 1 min -> 2 s; uniform within
@@ -208,6 +206,8 @@ class Problem:
     # Eq. (1)/(2) batch model per row: inference time of a batch of B = slope * B + intercept
     batch_slope_us: Optional[np.ndarray] = None      # f64 [sum M]
     batch_intercept_us: Optional[np.ndarray] = None  # f64 [sum M]
+    # scale-out: instances of each function (NEXT-4, reading G26); None = one each
+    instances: Optional[np.ndarray] = None           # int32 [N]
 
     @property
     def n_funcs(self) -> int:
@@ -241,7 +241,26 @@ def build_problem(name: str, dag: str, m: int, w: int, arrivals: np.ndarray,
         windows_us=window_grid(w), batch_slope_us=slope, batch_intercept_us=icept)
 
 
-CONFIG_NUMBER = {"C1": 1, "C2": 2, "C3": 3, "C4": 4, "C5": 5}
+CONFIG_NUMBER = {"C1": 1, "C2": 2, "C3": 3, "C4": 4, "C5": 5, "C3s": 3, "C5s": 5}
+
+
+def peak_window_count(arrivals_us, window_us: int = US_PER_S) -> int:
+    """Largest number of predicted invocations in one 1-s window (the predictor
+    forecasts invocations per 1-s window): the G the auto-scaler provisions for."""
+    a = np.asarray(arrivals_us, dtype=np.int64)
+    return int(np.bincount((a - a[0]) // window_us).max())
+
+
+# Scale-out instance counts of C3 / C5 (inputs of model M, reading G26): for every function,
+# the instances the paper's auto-scaler constraint (Eq. (7)/(8), PAPER.md:228-237) needs at the
+# function's fastest configuration to keep up with the predicted peak G = peak_window_count()
+# per window IT = I_s = 1 s: ceil(G / B) with B the largest batch meeting I_s.  Written here as
+# data; tests/test_oracle_pins.py::test_workload_instances_are_the_autoscalers re-derives them
+# with oracle/autoscale.py and the library's smiless_autoscale_rows.
+SCALE_OUT_INSTANCES = {
+    "C3": [2, 1, 4, 2, 3, 3, 2, 1],
+    "C5": [2, 2, 2, 2, 3, 2, 1, 2, 2, 3],
+}
 
 
 def make_config(name: str, n_arrivals: Optional[int] = None) -> Problem:
@@ -262,23 +281,35 @@ def make_config(name: str, n_arrivals: Optional[int] = None) -> Problem:
         arr_seed = rng.integers(1 << 62)
         arr = poisson_arrivals(np.random.default_rng(arr_seed), j, 0.25)
         return build_problem("C2", "ipa6", 16, 8, arr, rng)
-    if name == "C3":
+    if name in ("C3", "C3s"):
+        # C3: 10 req/s bursts served by scale-out instances (NEXT-4);
+        # C3s: the single-instance variant with the bursts softened to 3 req/s (round 1)
         j = n_arrivals or 10_000
         arr_seed = rng.integers(1 << 62)
-        arr = mmpp_arrivals(np.random.default_rng(arr_seed), j)
-        return build_problem("C3", "fan8", 12, 8, arr, rng)
+        rates = (0.2, 10.0) if name == "C3" else (0.2, 3.0)
+        arr = mmpp_arrivals(np.random.default_rng(arr_seed), j, rates=rates)
+        p = build_problem(name, "fan8", 12, 8, arr, rng)
+        if name == "C3":
+            p.instances = np.asarray(SCALE_OUT_INSTANCES["C3"], dtype=np.int32)
+        return p
     if name == "C4":
         # one re-plan window of the SLA x rate sweep (100 arrivals at 0.25 req/s)
         j = n_arrivals or 100
         arr_seed = rng.integers(1 << 62)
         arr = poisson_arrivals(np.random.default_rng(arr_seed), j, 0.25)
         return build_problem("C4", "ipa6", 8, 4, arr, rng)
-    if name == "C5":
+    if name in ("C5", "C5s"):
+        # C5: Azure-shaped 0.25 invocations per 1-s window with VMR 3 served by
+        # scale-out instances (NEXT-4); C5s: the single-instance variant at 0.2 per window,
+        # VMR 2.2 (round 1: the fastest single-instance plan meets 2 s)
         j = n_arrivals or 10_000
         arr_seed = rng.integers(1 << 62)
-        # 0.2 invocations per 1-s window, VMR 2.2: the fastest single-instance plan meets 2 s
-        arr = azure_arrivals(np.random.default_rng(arr_seed), j, mean_per_window=0.2, vmr=2.2)
-        return build_problem("C5", "mixed10", 8, 16, arr, rng)
+        mpw, vmr = (0.25, 3.0) if name == "C5" else (0.2, 2.2)
+        arr = azure_arrivals(np.random.default_rng(arr_seed), j, mean_per_window=mpw, vmr=vmr)
+        p = build_problem(name, "mixed10", 8, 16, arr, rng)
+        if name == "C5":
+            p.instances = np.asarray(SCALE_OUT_INSTANCES["C5"], dtype=np.int32)
+        return p
     raise KeyError(name)
 
 
