@@ -147,7 +147,7 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
-def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
+def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier, sla=None):
     """Exact OPT of a whole BASELINE config space with pruning + two-level B&B, sharded over
     the ranks (C2 / C3: interleaved prefix batches of one plan; C5, 2^70 candidates: the 128
     values of function 0's digit, each a 2^63-candidate plan, round-robin over the ranks),
@@ -158,10 +158,12 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
                                                    plan_range_rounds, INF_BITS)
     rounds = int(os.environ.get("SMILESS_BENCH_ROUNDS", "1" if world == 1 else "2"))
     p = W.make_config(name)
+    if sla is not None:
+        p = p.replace(sla_us=int(sla))
     Wn = len(p.windows_us)
     pl = S.planner_for(p, device=local, stream=stream.cuda_stream)
     arr = torch.as_tensor(p.arrivals_us).to(dev)
-    pinned = name == "C5"
+    pinned = name in ("C5", "C5s")
     digits = list(range(int(p.n_configs[0]) * Wn)) if pinned else [None]
     warm = dict(n_fixed=1, fixed_digits=[0]) if pinned else {}
     seed = os.environ.get("SMILESS_SEED_CAP", "0") == "1"
@@ -228,6 +230,7 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
     sec = float(tt.item()) / 1e3
     cost = bits_cost(keys[0])
     out = {"candidates": decided, "time_to_optimal_s": sec, "wall_s": wall, "decided_per_s": decided / sec,
+           "sla_us": p.sla_us, "instances": None if p.instances is None else p.instances.tolist(),
            "full_evals_local": full_evals, "decided_per_rank": per_rank, "full_evals_per_rank": per_rank_full,
            "rounds": 1 if pinned else rounds,
            "cost": cost, "max_latency_us": lat if cost is not None else -1,
@@ -235,7 +238,8 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
     if cost is not None:
         kw = dict(n_fixed=1, fixed_digits=[keys[1]]) if pinned else {}
         c, w = pl.decode(keys[2], Wn, **kw)
-        out.update({"index": keys[2], "config": c.tolist(), "window": w.tolist()})
+        out.update({"index": keys[2], "config": c.tolist(), "window": w.tolist(),
+                    "windows_nonzero": int((w != 0).sum()), "full_evals_fraction": full_evals / max(1, decided)})
         if pinned:
             out["digit0"] = keys[1]
         if rank == 0:
@@ -244,6 +248,86 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier):
             out["oracle_check"] = {"feasible": bool(of[0]), "cost_bits_equal": bool(oc[0] == cost),
                                    "latency_equal": int(ol[0]) == out["max_latency_us"]}
     return out
+
+
+def plan_kernel_ops_per_candidate(p) -> float:
+    """Integer ops per candidate of smiless_plan_kernel (no prefix memoisation: every lane
+    walks its own upstream) over the horizon, counted like algorithmic_ops_per_candidate.  A
+    scale-out plan's kernel DAG ends in the virtual sink (one keep-alive variant joining the
+    real sinks), so every real function is upstream; ring shifts are register moves and are
+    not counted."""
+    n = p.n_funcs
+    Wn = len(p.windows_us)
+    listed = set(int(v) for v in p.pred_idx)
+    sinks = [k for k in range(n) if k not in listed]
+    joins = sum(max(0, len(p.preds(k)) - 1) for k in range(n))
+    if p.instances is not None and max(p.instances) > 1:
+        upstream = 7 * n + joins + (len(sinks) - 1)       # + the virtual sink's join
+        per_unit = 3 + 4                                   # one keep-alive variant
+        share = 1
+    else:
+        G = configs_per_lane(p)
+        up_sinks = sum(1 for k in sinks if k != n - 1)
+        upstream = 7 * (n - 1) + joins + up_sinks
+        w0 = 1 if int(p.windows_us[0]) == 0 else 0
+        per_unit = G * (3 + 4 * w0 + 7 * (Wn - w0))
+        share = G * Wn
+    return (upstream + per_unit) / share * (len(p.arrivals_us) - 1)
+
+
+SLICE_PINNED = {"C3": 4, "C5": 6, "C3s": 4, "C5s": 6}   # leading functions pinned (fastest, keep-alive)
+
+
+def throughput_slice(name, S, dev, stream, local, steps=2, n_cand=1 << 24):
+    """Throughput mode (no pruning) over a fixed slice of C3 / C5: the first n_cand candidates
+    with the leading functions pinned to their fastest configuration, keep-alive.  Reports
+    candidates/s, function-steps/s and the evaluator's fraction of the issue peak for the
+    kernel path it takes (scale-out plans: smiless_plan_kernel; else the memoised kernels)."""
+    import torch
+    p = W.make_config(name)
+    Wn = len(p.windows_us)
+    nf = SLICE_PINNED[name]
+    M = int(p.n_configs[0])
+    fixed = [int(np.argmin(p.exec_us[k * M:(k + 1) * M])) * Wn for k in range(nf)]
+    pl = S.planner_for(p, device=local, stream=stream.cuda_stream)
+    arr = torch.as_tensor(p.arrivals_us).to(dev)
+    kw = dict(n_fixed=nf, fixed_digits=fixed, end=n_cand, flags=S.FLAG_NO_PRUNE)
+    pl.plan(arr, p.sla_us, p.windows_us, **kw)                          # NVRTC + warm-up
+    torch.cuda.synchronize(dev)
+    a = torch.cuda.Event(enable_timing=True)
+    b = torch.cuda.Event(enable_timing=True)
+    kms = 0.0
+    a.record(stream)
+    for _ in range(steps):
+        r = pl.plan(arr, p.sla_us, p.windows_us, **kw)
+        kms += r.eval_kernel_ms
+    b.record(stream)
+    torch.cuda.synchronize(dev)
+    sec = a.elapsed_time(b) / 1e3
+    scale_out = p.instances is not None and max(p.instances) > 1
+    ops = (plan_kernel_ops_per_candidate(p) if scale_out else
+           algorithmic_ops_per_candidate(p, memo=os.environ.get("SMILESS_MEMO", "1") != "0",
+                                         split=os.environ.get("SMILESS_SPLITCOST", "1") != "0"))
+    value = steps * r.n_decided / sec
+    return {"candidates_per_step": r.n_decided, "value": value, "unit": UNIT,
+            "function_steps_per_s": value * p.n_funcs * (len(p.arrivals_us) - 1),
+            "slice": f"first {n_cand} candidates, functions 0..{nf - 1} pinned to digits {fixed}",
+            "kernel": "smiless_plan_kernel (scale-out)" if scale_out else "memoised upstream + variants",
+            "int_ops_per_candidate": ops, "achieved_int_ops_per_s": ops * r.n_decided / (kms / steps / 1e3),
+            "instances": None if p.instances is None else p.instances.tolist(),
+            "winner": {"index": r.index, "cost": r.cost} if r.feasible else None}
+
+
+def gap_fractions(p):
+    """fraction of inter-arrival gaps longer than T + I per function and
+    configuration (both Case I and Case II must occur for the window dimension to matter)."""
+    gaps = np.diff(np.asarray(p.arrivals_us, dtype=np.int64))
+    off = np.concatenate([[0], np.cumsum(p.n_configs)])
+    per_fn = []
+    for k in range(p.n_funcs):
+        fr = [float((gaps > int(p.init_us[r]) + int(p.exec_us[r])).mean()) for r in range(off[k], off[k + 1])]
+        per_fn.append({"min": min(fr), "median": float(np.median(fr)), "max": max(fr)})
+    return {"per_function_over_configs": per_fn, "gaps": int(len(gaps))}
 
 
 def measured_peaks():
@@ -269,21 +353,55 @@ def ncu_traffic(memo: bool, plan_launches: int):
         return None
 
 
-def cpu_oracle_rate(p, kw, seconds: float = 15.0, threads=None):
-    """Oracle (as it stands) on the host cores: candidates/s over a bounded sample of the
-    same slice (its first candidates, sized to ~`seconds` of CPU work)."""
+def host_cpu():
+    """CPU model and clock of this host (lscpu, else /proc/cpuinfo) for the oracle timings."""
+    info = {"model": None, "mhz": None, "max_mhz": None, "nproc": os.cpu_count()}
+    try:
+        import subprocess
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            k, _, v = line.partition(":")
+            k, v = k.strip(), v.strip()
+            if k == "Model name":
+                info["model"] = v
+            elif k == "CPU MHz":
+                info["mhz"] = float(v)
+            elif k == "CPU max MHz":
+                info["max_mhz"] = float(v)
+    except Exception:
+        pass
+    if info["mhz"] is None:
+        try:
+            for line in open("/proc/cpuinfo"):
+                if line.startswith("cpu MHz"):
+                    info["mhz"] = float(line.split(":")[1])
+                    break
+                if line.startswith("model name") and not info["model"]:
+                    info["model"] = line.split(":")[1].strip()
+        except Exception:
+            pass
+    return info
+
+
+def cpu_oracle_rate(p, kw, n_random: int = 1 << 16, n_first: int = 1 << 16, threads=None, seed: int = 8):
+    """Oracle (as it stands) on the host cores, SURVEY 8(d) sample: 2^16 seeded random indices
+    of the space plus its first 2^16 indices, evaluated by `threads` threads (ctypes releases
+    the GIL).  Returns (candidates/s, sample size, seconds, threads)."""
+    from concurrent.futures import ThreadPoolExecutor
+    import numpy as np_
     from oracle import OracleProblem
     threads = threads or os.cpu_count() or 1
     o = OracleProblem(p, n_fixed=kw["n_fixed"], fixed_digits=kw["fixed_digits"])
-    n = max(threads, 8)
+    space = o.space_size()
+    rng = np_.random.default_rng(seed)
+    idx = np_.concatenate([rng.integers(0, space, size=n_random, dtype=np_.uint64),
+                           np_.arange(min(n_first, space), dtype=np_.uint64)])
+    parts = np_.array_split(idx, threads)
     t0 = time.perf_counter()
-    o.plan(0, n, n_threads=threads)
+    with ThreadPoolExecutor(threads) as ex:
+        list(ex.map(o.evaluate, parts))
     dt = time.perf_counter() - t0
-    n2 = max(threads, int(n * seconds / max(dt, 1e-6)))
-    t0 = time.perf_counter()
-    o.plan(0, n2, n_threads=threads)
-    dt = time.perf_counter() - t0
-    return n2 / dt, n2, dt, threads
+    return len(idx) / dt, len(idx), dt, threads
 
 
 def run_reference(args):
@@ -350,6 +468,8 @@ def main():
     ap.add_argument("--no-full-space", action="store_true",
                     help="skip the exhaustive pruned plan of the whole workload space (time-to-optimal)")
     ap.add_argument("--no-c4", action="store_true", help="skip the C4 SLA-sweep re-planning rate")
+    ap.add_argument("--no-extra", action="store_true",
+                    help="skip C1 time-to-optimal, the C3/C5 throughput slices and the live-window SLAs")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -438,7 +558,7 @@ def main():
         ms, res, launches, kernel_ms = timed(arr_dev, args.steps)
     barrier()
     barrier()
-    ms_e2e, res_e2e, _, _ = timed(arr_pin, max(1, min(args.steps, 3)))
+    ms_e2e, res_e2e, _, _ = timed(arr_pin, args.steps)
     barrier()
 
     cands = int(res.n_decided)
@@ -446,7 +566,7 @@ def main():
         t = torch.tensor([cands], dtype=torch.int64, device=xdev)
         dist.all_reduce(t)
         cands = int(t.item())
-    steps_e2e = max(1, min(args.steps, 3))
+    steps_e2e = args.steps
     value = cands * args.steps / (ms / 1e3)
     e2e_value = cands * steps_e2e / (ms_e2e / 1e3)
 
@@ -472,8 +592,37 @@ def main():
     full = None
     if not args.no_full_space:
         full = {}
-        for name in ("C2", "C3", "C5"):
+        for name in os.environ.get("SMILESS_BENCH_FULL", "C2,C3,C3s,C5,C5s").split(","):
             full[name] = full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier)
+        if not args.no_extra:
+            # SURVEY 8(d) / VERDICT: instances where the pre-warm windows are live at J = 10^4
+            for sla in (4_000_000, 8_000_000):
+                full[f"C2@SLA{sla // 1_000_000}s"] = full_space_opt("C2", S, rank, world, dev, xdev, stream, local,
+                                                                   barrier, sla=sla)
+
+    # C1 time-to-optimal, C3 / C5 throughput slices (N = 1)
+    extra = None
+    if not args.no_extra and world == 1:
+        extra = {}
+        p1 = W.make_config("C1")
+        pl1 = S.planner_for(p1, device=local, stream=stream.cuda_stream)
+        arr1 = torch.as_tensor(p1.arrivals_us).to(dev)
+        pl1.plan(arr1, p1.sla_us, p1.windows_us)
+        barrier()
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        r1 = pl1.plan(arr1, p1.sla_us, p1.windows_us)
+        b.record(stream)
+        torch.cuda.synchronize(dev)
+        from oracle import OracleProblem
+        ref1 = OracleProblem(p1).plan()
+        extra["C1_time_to_optimal"] = {"time_to_optimal_ms": a.elapsed_time(b), "candidates": 4096,
+                                       "index": r1.index, "cost": r1.cost, "max_latency_us": r1.max_latency_us,
+                                       "oracle_plan_equal": ref1 == (r1.index, r1.cost, r1.max_latency_us)}
+        for name in ("C3", "C5"):
+            extra[f"{name}_throughput_slice"] = throughput_slice(name, S, dev, stream, local)
+        extra["C2_gaps_longer_than_T_plus_I"] = gap_fractions(p)
 
     # C4 (configs[3]): 1,000 re-plans of 100 predicted arrivals, 6 SLAs per pass, exhaustive each
     c4 = None
@@ -528,9 +677,11 @@ def main():
         "pruned": pruned,
         "time_to_optimal_full_space": full,
         "c4_sla_sweep_replanning": c4,
+        "extra": extra,
         "gpu_launches": launches,
-        "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(p.arrivals_us.nbytes),
-                "d2h_bytes_per_step": 312},
+        "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(res_e2e.h2d_bytes),
+                "d2h_bytes_per_step": int(res_e2e.d2h_bytes), "steps": steps_e2e,
+                "bytes_basis": "counted by the library per smiless_plan call (smiless_plan_result)"},
         "clocks": clocks,
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_ops, "unit": "int-ops/s",
                      "frac": achieved / peak_ops, "traffic": ncu_traffic(memo, res.launches),
@@ -549,11 +700,15 @@ def main():
     }
     if world == 1 and not args.no_cpu_baseline:
         rate, n, dt, threads = cpu_oracle_rate(p, kw)
-        rate1, n1, dt1, _ = cpu_oracle_rate(p, kw, seconds=2.0, threads=1)       # SURVEY 8(d) iii
+        rate1, n1, dt1, _ = cpu_oracle_rate(p, kw, n_random=1 << 12, n_first=1 << 12, threads=1)  # SURVEY 8(d) iii
+        cpu = host_cpu()
         line["cpu_baseline"] = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle",
-                                "sample": f"first {n} candidates of the slice ({dt:.1f} s, J={len(p.arrivals_us)})",
+                                "sample": f"2^16 seeded random + the first 2^16 candidates of the slice ({n} in "
+                                          f"{dt:.1f} s, J={len(p.arrivals_us)})",
+                                "cpu_model": cpu["model"], "cpu_mhz": cpu["mhz"], "cpu_max_mhz": cpu["max_mhz"],
+                                "function_steps_per_s": rate * p.n_funcs * (len(p.arrivals_us) - 1),
                                 "single_core_value": rate1,
-                                "single_core_sample": f"first {n1} candidates, 1 thread ({dt1:.1f} s)"}
+                                "single_core_sample": f"2^12 random + first 2^12 candidates, 1 thread ({dt1:.1f} s)"}
         if full:
             for name, f in full.items():          # what the same exhaustive search costs on the oracle
                 f["oracle_extrapolated_s"] = f["candidates"] / rate

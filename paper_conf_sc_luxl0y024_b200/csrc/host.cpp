@@ -772,6 +772,10 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     const char *sel_env = getenv("SMILESS_SELMASK");
     s << "#define SM_SELMASK " << (sel_env ? atoi(sel_env) : 0) << "\n";
     s << "#define SM_SPLITCOST " << (split_cost() ? 1 : 0) << "\n";
+    // window variants of the memoised kernel walked in the positive-time form (evaluator.cuh
+    // variants_step FM: ALU busy mask + full-rate IMAD instead of the quarter-rate IMAD.HI)
+    const char *fm_env = getenv("SMILESS_FMASK");
+    s << "#define SM_FMASK " << (fm_env ? strtoul(fm_env, nullptr, 0) : 0ul) << "u\n";
     const char *vun_env = getenv("SMILESS_VUNROLL");
     s << "#define SM_VUNROLL " << (vun_env ? atoi(vun_env) : 4) << "\n";
     const char *alusul_env = getenv("SMILESS_ALUSUL"), *alug_env = getenv("SMILESS_ALUG");
@@ -1809,8 +1813,9 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 }
             } else {
                 NvtxRange nv("bnb level + evaluate");
-                for (u64 b0 = p_lo; b0 < p_hi; b0 += batch) {
-                    const u64 b1 = std::min(p_hi, b0 + batch);
+                const u64 rbatch = std::min(batch, list_cap);     // a launch's survivors fit the list
+                for (u64 b0 = p_lo; b0 < p_hi; b0 += rbatch) {
+                    const u64 b1 = std::min(p_hi, b0 + rbatch);
                     CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
                     CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
                     bp.list_in = nullptr;
