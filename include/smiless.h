@@ -262,6 +262,21 @@ SMILESS_API int smiless_decompose_search(smiless_ctx *ctx, const smiless_plan_ar
                                          smiless_plan_result *res, int32_t *config_out, int32_t *window_out,
                                          int64_t *n_paths);
 
+/* NEXT-3 with model M on the GPU: decompose the DAG into its source-to-sink
+ * paths, plan every path exhaustively (the exact smiless_plan of the path's chain -- its own
+ * functions, configurations, window grid, instances, the same arrivals and SLA -- on the GPU),
+ * then combine as the paper does: a function on several paths takes the (configuration,
+ * window) with the shortest inference time among the paths' choices (F_s / F_e of a parallel
+ * substructure), and every function on one path only moves to its cheapest (configuration,
+ * window) that keeps that path's model-M latency at or below its latency before combining
+ * (paths in DFS order, functions in path order; the alternatives are evaluated on the GPU,
+ * ties to the lowest digit).  The combined plan is evaluated with model M on the whole DAG
+ * (res, config_out, window_out; INFEASIBLE if a path has no feasible plan or the combined plan
+ * misses the SLA); *n_paths the number of paths.  a->n_fixed == 0, no row windows; at most
+ * 4096 paths.  The paths are independent plans (the paper runs them in parallel). */
+SMILESS_API int smiless_decompose_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res,
+                                       int32_t *config_out, int32_t *window_out, int64_t *n_paths);
+
 /* SLA sweep (C4: "impact of SLA settings"): ONE evaluation of the space
  * with one argmin key per SLA in slas[0..n_sla) (1 <= n_sla <= SMILESS_MAX_SLAS); pruning uses
  * their maximum; a->sla_us is ignored and a->cost_out must be NULL.  res[n_sla] and, when not

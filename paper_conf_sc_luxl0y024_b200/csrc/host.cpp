@@ -1891,10 +1891,11 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             ++launches;
         }
         CK(cudaMemcpyAsync(&ctx->dRes.p->stats[0], ctx->dStats.p, 16, cudaMemcpyDeviceToDevice, st), "D2D stats");
-        if (a->cost_out)
+        if (a->cost_out) {
             ctx->d2h += (size_t)(ce - cb) * sizeof(double);
             CK(cudaMemcpyAsync(a->cost_out, ctx->dDump.p, (size_t)(ce - cb) * sizeof(double), cudaMemcpyDeviceToHost, st),
                "D2H dump");
+        }
     } else if (single && ce > cb) {
         // the space is the single candidate of the pinned digits: index 0
         for (int s_ = 0; s_ < n_sla; ++s_) CK(cudaMemsetAsync(&ctx->dRes.p[s_].best_c, 0, 16, st), "memset");
@@ -2290,6 +2291,188 @@ int smiless_decompose_search(smiless_ctx *ctx, const smiless_plan_args *a, int64
     for (int k = 0; k < N; ++k) {
         if (config_out) config_out[k] = ok ? cfg[k] : -1;
         if (window_out) window_out[k] = ok ? 0 : -1;
+    }
+    if (!ok) {
+        res->index = ~0ull;
+        res->cost = HUGE_VAL;
+        res->max_latency_us = -1;
+        return SMILESS_INFEASIBLE;
+    }
+    res->index = idx;
+    res->cost = cost;
+    res->max_latency_us = lat;
+    return SMILESS_OK;
+}
+
+int smiless_decompose_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res,
+                           int32_t *config_out, int32_t *window_out, int64_t *n_paths) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->err.clear();
+    if (!a || !res) return fail(ctx, SMILESS_EINVAL, "args / res is NULL");
+    if (a->n_fixed != 0) return fail(ctx, SMILESS_EINVAL, "decompose plan does not take pinned digits");
+    if (a->row_windows_us) return fail(ctx, SMILESS_EINVAL, "decompose plan searches the window grid (no row windows)");
+    int rc = validate_args(ctx, a, true);
+    if (rc) return rc;
+    const int N = ctx->N, W = a->n_windows;
+    // 1. decompose into source-to-sink paths (subgraphs with only sequential dependencies)
+    std::vector<std::vector<int>> succ(N), paths;
+    for (int k = 0; k < N; ++k)
+        for (int e = ctx->pred_ptr[k]; e < ctx->pred_ptr[k + 1]; ++e) succ[ctx->pred_idx[e]].push_back(k);
+    std::vector<int> cur;
+    bool too_many = false;
+    std::function<void(int)> walk = [&](int k) {
+        if (too_many) return;
+        cur.push_back(k);
+        if (succ[k].empty()) {
+            paths.push_back(cur);
+            if (paths.size() > 4096) too_many = true;
+        }
+        for (int s_ : succ[k]) walk(s_);
+        cur.pop_back();
+    };
+    for (int k = 0; k < N; ++k)
+        if (ctx->pred_ptr[k] == ctx->pred_ptr[k + 1]) walk(k);
+    if (too_many) return fail(ctx, SMILESS_EINVAL, "more than 4096 source-to-sink paths");
+    // one child context per path length (a chain DAG): the NVRTC specialisation is shared by
+    // every path of that length, its profiles are reloaded per path
+    std::map<int, smiless_ctx *> subs;
+    struct SubGuard {
+        std::map<int, smiless_ctx *> &m;
+        ~SubGuard() { for (auto &kv : m) smiless_destroy(kv.second); }
+    } guard{subs};
+    auto sub_for = [&](const std::vector<int> &P, smiless_ctx **out) -> int {
+        const int L = (int)P.size();
+        auto it = subs.find(L);
+        if (it == subs.end()) {
+            smiless_ctx *c = nullptr;
+            int r = smiless_create(&c, ctx->device, ctx->stream);
+            if (r) return fail(ctx, r, "decompose: cannot create a path context");
+            it = subs.emplace(L, c).first;
+        }
+        smiless_ctx *c = it->second;
+        std::vector<int32_t> ptr(L + 1), idx(std::max(L - 1, 1));
+        ptr[0] = 0;
+        for (int q = 0; q < L; ++q) {
+            if (q > 0) idx[q - 1] = q - 1;
+            ptr[q + 1] = q;                               // q has predecessor q - 1 (chain)
+        }
+        int r = smiless_load_dag(c, L, ptr.data(), idx.data());
+        std::vector<int32_t> m, I, T;
+        std::vector<double> U;
+        for (int k : P) {
+            m.push_back(ctx->M[k]);
+            for (int cc = 0; cc < ctx->M[k]; ++cc) {
+                I.push_back(ctx->I[ctx->row0[k] + cc]);
+                T.push_back(ctx->T[ctx->row0[k] + cc]);
+                U.push_back(ctx->U[ctx->row0[k] + cc]);
+            }
+        }
+        if (!r) r = smiless_load_profiles(c, m.data(), I.data(), T.data(), U.data());
+        if (r) return fail(ctx, r, "decompose: path context: %s", smiless_last_error(c));
+        *out = c;
+        return SMILESS_OK;
+    };
+    auto path_args = [&](const std::vector<int> &P, std::vector<int32_t> &inst) {
+        smiless_plan_args pa = *a;
+        pa.begin = pa.end = 0;
+        pa.shard = 0;
+        pa.n_shards = 0;
+        pa.cost_out = nullptr;
+        pa.flags = a->flags & (SMILESS_FLAG_ARRIVALS_ON_DEVICE | SMILESS_FLAG_FORCE_INT64);
+        inst.clear();
+        for (int k : P) inst.push_back(inst_of(a, k));
+        pa.instances = inst.data();
+        return pa;
+    };
+    // 2. each path's exhaustive optimum under model M (exact B&B plan of the chain on the GPU)
+    std::vector<std::vector<int>> pc(paths.size()), pw(paths.size());
+    std::vector<i64> plat(paths.size(), 0);
+    std::vector<int32_t> inst;
+    for (size_t pi = 0; pi < paths.size(); ++pi) {
+        const auto &P = paths[pi];
+        smiless_ctx *c = nullptr;
+        if ((rc = sub_for(P, &c))) return rc;
+        smiless_plan_args pa = path_args(P, inst);
+        smiless_plan_result pr;
+        std::vector<int32_t> co(P.size()), wo(P.size());
+        rc = smiless_plan(c, &pa, &pr, co.data(), wo.data());
+        if (rc < 0) return fail(ctx, rc, "decompose: path plan: %s", smiless_last_error(c));
+        if (rc == SMILESS_INFEASIBLE) {                  // no plan meets the SLA on this path alone
+            memset(res, 0, sizeof *res);
+            res->index = ~0ull;
+            res->cost = HUGE_VAL;
+            res->max_latency_us = -1;
+            for (int k = 0; k < N; ++k) {
+                if (config_out) config_out[k] = -1;
+                if (window_out) window_out[k] = -1;
+            }
+            if (n_paths) *n_paths = (int64_t)paths.size();
+            return SMILESS_INFEASIBLE;
+        }
+        pc[pi].assign(co.begin(), co.end());
+        pw[pi].assign(wo.begin(), wo.end());
+        plat[pi] = pr.max_latency_us;
+    }
+    // 3. combine (reading G25): a function on several paths takes the choice with the
+    // shortest inference time among them (the rule for F_s / F_e of a parallel substructure) ...
+    std::vector<int> cfg(N, -1), win(N, -1), n_on(N, 0);
+    for (size_t pi = 0; pi < paths.size(); ++pi)
+        for (size_t q = 0; q < paths[pi].size(); ++q) {
+            const int k = paths[pi][q], m = pc[pi][q];
+            n_on[k] += 1;
+            if (cfg[k] < 0 || ctx->I[ctx->row0[k] + m] < ctx->I[ctx->row0[k] + cfg[k]]) {
+                cfg[k] = m;
+                win[k] = pw[pi][q];
+            }
+        }
+    // ... and every function on one path only moves to its cheapest (configuration, window) that
+    // keeps that path's model-M latency at or below its latency before combining (evaluated on
+    // the GPU, one batch per function; ties to the lowest digit)
+    for (size_t pi = 0; pi < paths.size(); ++pi) {
+        const auto &P = paths[pi];
+        smiless_ctx *c = nullptr;
+        if ((rc = sub_for(P, &c))) return rc;
+        smiless_plan_args pa = path_args(P, inst);
+        for (size_t q = 0; q < P.size(); ++q) {
+            const int k = P[q];
+            if (n_on[k] != 1) continue;
+            const int R = ctx->M[k] * W;
+            std::vector<uint64_t> idx(R);
+            for (int d = 0; d < R; ++d) {
+                u64 v = 0;
+                for (size_t z = 0; z < P.size(); ++z) {
+                    const u64 dz = (z == q) ? (u64)d : (u64)cfg[P[z]] * (u64)W + (u64)win[P[z]];
+                    v = v * ((u64)ctx->M[P[z]] * (u64)W) + dz;
+                }
+                idx[d] = v;
+            }
+            std::vector<double> cost(R);
+            std::vector<int64_t> lat(R);
+            std::vector<uint8_t> ok(R);
+            rc = smiless_evaluate(c, &pa, idx.data(), R, cost.data(), lat.data(), ok.data());
+            if (rc) return fail(ctx, rc, "decompose: path evaluate: %s", smiless_last_error(c));
+            int best = -1;
+            for (int d = 0; d < R; ++d)
+                if (lat[d] <= plat[pi] && (best < 0 || cost[d] < cost[best])) best = d;
+            if (best >= 0) {
+                cfg[k] = best / W;
+                win[k] = best % W;
+            }
+        }
+    }
+    // 4. the combined plan under model M on the whole DAG
+    u64 idx = 0;
+    for (int k = 0; k < N; ++k) idx = idx * ((u64)ctx->M[k] * (u64)W) + (u64)cfg[k] * (u64)W + (u64)win[k];
+    double cost = 0.0;
+    int64_t lat = 0;
+    uint8_t ok = 0;
+    if ((rc = smiless_evaluate(ctx, a, (const uint64_t *)&idx, 1, &cost, &lat, &ok))) return rc;
+    memset(res, 0, sizeof *res);
+    res->n_decided = res->n_full_evals = 1;
+    if (n_paths) *n_paths = (int64_t)paths.size();
+    for (int k = 0; k < N; ++k) {
+        if (config_out) config_out[k] = ok ? cfg[k] : -1;
+        if (window_out) window_out[k] = ok ? win[k] : -1;
     }
     if (!ok) {
         res->index = ~0ull;

@@ -25,7 +25,7 @@ _NAMES = {0: "OK", 1: "INFEASIBLE", -1: "EINVAL", -2: "ENOTTOPO", -3: "ERANGE", 
 # every symbol include/smiless.h declares (checked by tests/test_abi.py)
 EXPORTS = ("smiless_create", "smiless_set_stream", "smiless_destroy", "smiless_last_error",
            "smiless_load_dag", "smiless_load_profiles", "smiless_space_size", "smiless_plan",
-           "smiless_plan_sla_sweep", "smiless_derive_windows", "smiless_top1_search", "smiless_decompose_search",
+           "smiless_plan_sla_sweep", "smiless_derive_windows", "smiless_top1_search", "smiless_decompose_search", "smiless_decompose_plan",
            "smiless_autoscale", "smiless_autoscale_rows",
            "smiless_evaluate",
            "smiless_decode",
@@ -130,6 +130,8 @@ def load_library(build_if_missing: bool = True):
                                              vp, ctypes.POINTER(ctypes.c_int64)]
     lib.smiless_top1_search.argtypes = [vp, ctypes.POINTER(PlanArgs), i64, ctypes.POINTER(PlanResultC), vp, vp,
                                         ctypes.POINTER(ctypes.c_int64)]
+    lib.smiless_decompose_plan.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.POINTER(PlanResultC), vp, vp,
+                                           ctypes.POINTER(ctypes.c_int64)]
     lib.smiless_evaluate.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i64, vp, vp, vp]
     lib.smiless_decode.argtypes = [vp, i32, u64, ctypes.POINTER(PlanArgs), vp, vp]
     lib.smiless_kernel_source.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.c_char_p, ctypes.c_size_t,
@@ -348,6 +350,23 @@ class Planner:
                           max_latency_us=int(r.max_latency_us), config=cfg[:self.n_funcs],
                           window=win[:self.n_funcs], n_decided=1, n_full_evals=1, eval_kernel_ms=0.0,
                           total_device_ms=0.0, int64_path=False, launches=0), int(n.value)
+
+    def decompose_plan(self, arrivals, sla_us, windows_us, **kw):
+        """NEXT-3 with model M (smiless_decompose_plan): exhaustive GPU plan per source-to-sink
+        path, the paper's combine; returns (PlanResult, number of paths)."""
+        a, keep = self._args(arrivals, sla_us, windows_us, **kw)
+        r = PlanResultC()
+        cfg = np.zeros(max(self.n_funcs, 1), np.int32)
+        win = np.zeros(max(self.n_funcs, 1), np.int32)
+        npaths = ctypes.c_int64()
+        rc = self._check(self._lib.smiless_decompose_plan(self._ctx, ctypes.byref(a), ctypes.byref(r), cfg.ctypes.data,
+                                                          win.ctypes.data, ctypes.byref(npaths)),
+                         allow=(OK, INFEASIBLE))
+        del keep
+        return PlanResult(status=rc, index=None if rc == INFEASIBLE else int(r.index), cost=float(r.cost),
+                          max_latency_us=int(r.max_latency_us), config=cfg[:self.n_funcs],
+                          window=win[:self.n_funcs], n_decided=int(r.n_decided), n_full_evals=int(r.n_full_evals),
+                          eval_kernel_ms=0.0, total_device_ms=0.0, int64_path=False, launches=0), int(npaths.value)
 
     def evaluate(self, idx, arrivals, sla_us, windows_us, **kw) -> Tuple[np.ndarray, np.ndarray, np.ndarray]:
         a, keep = self._args(arrivals, sla_us, windows_us, **kw)

@@ -1156,3 +1156,67 @@ def test_c2_window0_subspace_matches_oracle_brute_force():
     full = pl.plan(arr, p.sla_us, p.windows_us)
     assert full.index == g["index_full_space"] and full.cost.hex() == g["cost_hex"]
     assert full.config.tolist() == g["config"] and (full.window == 0).all()
+
+
+# ---------------------------------------------------------------------------------------
+# NEXT-3 with model M: per-path exhaustive GPU plans + the paper's combine
+# ---------------------------------------------------------------------------------------
+
+def test_decompose_plan_golden_on_the_gpu():
+    """Golden P2m (hand-derived) through smiless_decompose_plan."""
+    import json, os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "P2m_decompose_model_m.json")))
+    ptr, idx = W.csr_from_preds(g["preds"])
+    p = W.Problem("t", ptr, idx, np.asarray(g["n_configs"], np.int32), np.asarray(g["exec_us"], np.int32),
+                  np.asarray(g["init_us"], np.int32), np.asarray(g["price_per_us"], np.float64),
+                  np.asarray(g["arrivals_us"], np.int64), g["sla_us"], np.asarray(g["windows_us"], np.int32))
+    r, n_paths = S.planner_for(p).decompose_plan(p.arrivals_us, p.sla_us, p.windows_us)
+    assert n_paths == 2 and r.feasible
+    assert r.config.tolist() == g["expected_configs"] and r.window.tolist() == [0] * 4
+    assert r.max_latency_us == g["expected_latency_us"] and r.cost == g["expected_cost"]
+
+
+def test_decompose_plan_matches_oracle_walk():
+    """Random DAGs (joins, several sinks, instances): the library's per-path GPU plans and
+    combine equal oracle/decompose_m.py step for step (configs, windows, cost bits)."""
+    from oracle.decompose_m import decompose_plan
+    rng = np.random.default_rng(808)
+    n_checked = n_feasible = 0
+    for t in range(60):
+        n = int(rng.integers(2, 6))
+        p = W.random_problem(rng, n, 3, int(rng.integers(1, 4)), int(rng.integers(2, 40)),
+                             sla_us=int(rng.integers(8_000, 40_000)))
+        if t % 2:
+            p = p.replace(instances=np.asarray([int(rng.integers(1, 3)) for _ in range(n)], np.int32))
+        pl = S.planner_for(p)
+        r, n_paths = pl.decompose_plan(p.arrivals_us, p.sla_us, p.windows_us)
+        cfg, win, cost, lat, ok, np_ = decompose_plan(p, OracleProblem)
+        assert n_paths == np_
+        assert r.feasible == ok
+        if ok:
+            assert r.config.tolist() == cfg and r.window.tolist() == win
+            assert r.cost == cost and r.max_latency_us == lat
+            n_feasible += 1
+        n_checked += 1
+        if n_checked == 30:
+            break
+    assert n_feasible >= 5
+
+
+@pytest.mark.parametrize("name", ["C3", "C5"])
+def test_decompose_plan_full_size(name):
+    """C3 / C5 at J = 10^4 with scale-out: the per-path decomposition yields a plan; if it is
+    feasible its cost is >= the exhaustive OPT's on the same space (C3) and it re-checks on
+    the oracle."""
+    p = W.make_config(name)
+    pl = S.planner_for(p)
+    r, n_paths = pl.decompose_plan(p.arrivals_us, p.sla_us, p.windows_us)
+    assert n_paths >= 2
+    if r.feasible:
+        Wn = len(p.windows_us)
+        kw = {}
+        oc, ol, of = OracleProblem(p).evaluate([r.index]) if name != "C5" else (None, None, None)
+        if name != "C5":
+            assert of[0] and oc[0] == r.cost
+            opt = pl.plan(p.arrivals_us, p.sla_us, p.windows_us)
+            assert opt.feasible and opt.cost <= r.cost

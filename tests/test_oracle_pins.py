@@ -659,3 +659,19 @@ def test_workload_instances_are_the_autoscalers(name):
     off = np.concatenate([[0], np.cumsum(p.n_configs)])
     fastest = [off[k] + int(np.argmin(p.exec_us[off[k]:off[k + 1]])) for k in range(n)]
     assert [n_o[r] for r in fastest] == list(W.SCALE_OUT_INSTANCES[name]) == list(p.instances)
+
+
+def test_decompose_model_m_on_diamond():
+    """Golden P2m (P:214-218 with exhaustive per-path optima under model M): the paths, each
+    path's optimum and latency, the F_s/F_e rule and the branch re-choice that moves F2 to
+    its cheaper configuration, and the combined plan's latency and cost."""
+    from oracle.decompose_m import decompose_plan
+    g = _golden("P2m_decompose_model_m.json")
+    p = mk(g["preds"], g["exec_us"], g["init_us"], g["arrivals_us"], g["windows_us"], sla=g["sla_us"],
+           prices=g["price_per_us"], n_configs=g["n_configs"])
+    tr = {}
+    cfg, win, cost, lat, ok, n_paths = decompose_plan(p, OracleProblem, trace=tr)
+    assert tr["paths"] == g["expected_paths"] and n_paths == 2
+    assert tr["path_configs"] == g["expected_path_configs"] and tr["path_latency"] == g["expected_path_latency"]
+    assert cfg == g["expected_configs"] and win == [0] * 4 and ok
+    assert lat == g["expected_latency_us"] and cost == g["expected_cost"]

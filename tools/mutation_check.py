@@ -26,6 +26,15 @@ MUTATIONS = [
      "if cfg[k] < 0 or I(k, m) < I(k, cfg[k]):", "if cfg[k] < 0 or I(k, m) > I(k, cfg[k]):"),
     ("decompose: branch functions not re-chosen after combining", "oracle/decompose.py",
      "            if n_on[k] != 1:\n                continue", "            if True:\n                continue"),
+    ("decompose (model M): F_s/F_e take the slowest of their paths' choices", "oracle/decompose_m.py",
+     "if cfg[k] < 0 or prob.exec_us[off[k] + c[q]] < prob.exec_us[off[k] + cfg[k]]:",
+     "if cfg[k] < 0 or prob.exec_us[off[k] + c[q]] > prob.exec_us[off[k] + cfg[k]]:"),
+    ("decompose (model M): no re-choice of branch functions", "oracle/decompose_m.py",
+     "            if n_on[k] != 1:\n                continue\n            R =", "            if True:\n                continue\n            R ="),
+    ("decompose (model M): re-choice may raise the path latency", "oracle/decompose_m.py",
+     "if lat[d] <= pl and (best is None or cost[d] < cost[best]):", "if (best is None or cost[d] < cost[best]):"),
+    ("scale-out: previous completion from request j-1 instead of j-n_k", "oracle/smiless_oracle.c",
+     "int64_t f = D[(int64_t)k * J + (j - n_inst[k])];", "int64_t f = D[(int64_t)k * J + (j - 1)];"),
     ("autoscale: ties go to the higher configuration", "oracle/autoscale.py",
      "if cost < best[3]:", "if cost <= best[3]:"),
     ("autoscale: smallest feasible batch instead of the largest", "oracle/autoscale.py",
