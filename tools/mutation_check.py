@@ -6,6 +6,7 @@ report which pins turn red.  A mutation no pin catches is a gap in the pins.
     python tools/mutation_check.py [--out profiles/r02_oracle_mutations.md]
 """
 import argparse
+import re
 import os
 import shutil
 import subprocess
@@ -90,6 +91,7 @@ def main():
         for mut in MUTATIONS:
             rc, failed = run_one(mut, tmp)
             caught = rc != 0 and failed
+            failed = [re.sub(r"\[/.*/tests/golden/", "[", f) for f in failed]
             rows.append((mut[0], mut[1], "caught" if caught else "SURVIVED", ", ".join(failed[:6])))
             print(rows[-1], flush=True)
     with open(args.out, "w") as fo:
