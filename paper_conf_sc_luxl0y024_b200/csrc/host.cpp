@@ -764,23 +764,12 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_NSLA " << ctx->nsla << "\n";
     s << "#define SM_ROWWIN " << (a->row_windows_us ? 1 : 0) << "\n";
     s << "#define SM_LBT " << (bound_lb_table(ctx, W) ? 1 : 0) << "\n";
-    const char *mask_env = getenv("SMILESS_MASK");   // tuning knob, see evaluator.cuh SM_MASK
-    s << "#define SM_MASK " << (mask_env ? atoi(mask_env) : 0) << "\n";
     s << "#define SM_XPF " << xpf_groups() << "\n";
-    // tuning knob, see evaluator.cuh SM_SELMASK; default: every window variant uses the IMAD.HI
-    // busy mask (measured best once the x stream is prefetched, profiles/r01k_sweep_variants.md)
-    const char *sel_env = getenv("SMILESS_SELMASK");
-    s << "#define SM_SELMASK " << (sel_env ? atoi(sel_env) : 0) << "\n";
     s << "#define SM_SPLITCOST " << (split_cost() ? 1 : 0) << "\n";
     // window variants of the memoised kernel walked in the positive-time form (evaluator.cuh
     // variants_step FM: ALU busy mask + full-rate IMAD instead of the quarter-rate IMAD.HI)
     const char *fm_env = getenv("SMILESS_FMASK");
     s << "#define SM_FMASK " << (fm_env ? strtoul(fm_env, nullptr, 0) : 0ul) << "u\n";
-    const char *vun_env = getenv("SMILESS_VUNROLL");
-    s << "#define SM_VUNROLL " << (vun_env ? atoi(vun_env) : 4) << "\n";
-    const char *alusul_env = getenv("SMILESS_ALUSUL"), *alug_env = getenv("SMILESS_ALUG");
-    s << "#define SM_ALUSUL " << (alusul_env ? atoi(alusul_env) : 0) << "\n#define SM_ALUG "
-      << (alug_env ? atoi(alug_env) : 0) << "\n";
     // scale-out (NEXT-4): any instance count > 1, the prologue length, the ring size
     s << "#define SM_INST " << (kd.virt ? 1 : 0) << "\n#define SM_PRO " << P << "\n#define SM_RG_ALLOC "
       << std::max(n_rg, 1) << "\n";
@@ -963,6 +952,7 @@ static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
 
 std::string full_source(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, bool off_smem,
                         int minb, int families = FAM_ALL) {
+    if (inst_mode(ctx, a)) families &= ~FAM_MEMO;       // scale-out plans never take the memo path
     return dag_spec_source(ctx, a, rp, off_smem, minb, families) + "\n" + smiless_evaluator_src;
 }
 

@@ -166,7 +166,10 @@ def test_nvrtc_specialises_every_config_for_sm100a(name):
     assert n > 0
     assert "0 bytes stack frame, 0 bytes spill stores, 0 bytes spill loads" in log, log
     src = pl.kernel_source(p.arrivals_us, p.sla_us, p.windows_us, n_fixed=nf, fixed_digits=[0] * nf)
-    assert "#define SM_N %d" % p.n_funcs in src and "smiless_plan_kernel" in src
+    # a scale-out plan (C3 / C5) is specialised for the DAG plus its virtual sink (DESIGN §5 item 13)
+    scale_out = p.instances is not None and max(p.instances) > 1
+    assert "#define SM_N %d" % (p.n_funcs + scale_out) in src and "smiless_plan_kernel" in src
+    assert ("#define SM_INST %d" % scale_out) in src
 
 
 def test_int64_path_selected_when_int32_range_fails():
