@@ -906,8 +906,8 @@ def test_branch_and_bound_shards_and_list_splits_are_exact(listcap, monkeypatch)
 def test_full_space_plan_shards_split_the_work(name, world):
     """The exact full-space plans of C2 (2^42) and C3 (7.2e15) sharded over `world` ranks
     (run one after the other on this GPU): every rank decides at least space / (2 world)
-    candidates and walks some to J, the shares sum to the space, and the best rank winner
-    is the single-rank OPT (which the oracle re-checks)."""
+    candidates, the shares sum to the space, and the best rank winner is the single-rank
+    OPT (which the oracle re-checks)."""
     import torch
     p = W.make_config(name)
     pl = S.planner_for(p)
@@ -921,7 +921,7 @@ def test_full_space_plan_shards_split_the_work(name, world):
     assert sum(r.n_decided for r in parts) == space
     for r in parts:
         assert r.n_decided >= space // (2 * world), [q.n_decided for q in parts]
-        assert r.n_full_evals > 0
+    assert sum(r.n_full_evals for r in parts) > 0      # (a rank's whole share may be pruned by the bounds)
     assert min((r.cost, r.index) for r in parts if r.feasible) == (one.cost, one.index)
 
 
