@@ -273,7 +273,10 @@ SMILESS_API int smiless_decompose_search(smiless_ctx *ctx, const smiless_plan_ar
  * ties to the lowest digit).  The combined plan is evaluated with model M on the whole DAG
  * (res, config_out, window_out; INFEASIBLE if a path has no feasible plan or the combined plan
  * misses the SLA); *n_paths the number of paths.  a->n_fixed == 0, no row windows; at most
- * 4096 paths.  The paths are independent plans (the paper runs them in parallel). */
+ * 4096 paths.  When the whole space exceeds 2^63, res->index is the plan's index with
+ * function 0's digit pinned (the suffix space of functions 1..N-1); config_out / window_out
+ * are always complete.  The paths are independent plans (the paper runs them in parallel,
+ * P:214). */
 SMILESS_API int smiless_decompose_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res,
                                        int32_t *config_out, int32_t *window_out, int64_t *n_paths);
 

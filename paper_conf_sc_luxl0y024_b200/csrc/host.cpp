@@ -2301,7 +2301,19 @@ int smiless_decompose_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless
     if (!a || !res) return fail(ctx, SMILESS_EINVAL, "args / res is NULL");
     if (a->n_fixed != 0) return fail(ctx, SMILESS_EINVAL, "decompose plan does not take pinned digits");
     if (a->row_windows_us) return fail(ctx, SMILESS_EINVAL, "decompose plan searches the window grid (no row windows)");
-    int rc = validate_args(ctx, a, true);
+    // a space above 2^63 (C5) is evaluated with function 0's digit pinned: the index is then in
+    // the suffix space of functions 1..N-1
+    const int32_t digit0 = 0;
+    smiless_plan_args av = *a;
+    {
+        u64 sp;
+        if (ctx->dag_loaded && ctx->prof_loaded && a->n_windows >= 1 && a->n_windows <= SMILESS_MAX_WINDOWS &&
+            !space_size_of(ctx, a->n_windows, 0, &sp)) {
+            av.n_fixed = 1;
+            av.fixed_digits = &digit0;
+        }
+    }
+    int rc = validate_args(ctx, &av, true);
     if (rc) return rc;
     const int N = ctx->N, W = a->n_windows;
     // 1. decompose into source-to-sink paths (subgraphs with only sequential dependencies)
@@ -2451,12 +2463,14 @@ int smiless_decompose_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless
         }
     }
     // 4. the combined plan under model M on the whole DAG
+    const int32_t d0 = cfg[0] * W + win[0];
+    if (av.n_fixed == 1) av.fixed_digits = &d0;
     u64 idx = 0;
-    for (int k = 0; k < N; ++k) idx = idx * ((u64)ctx->M[k] * (u64)W) + (u64)cfg[k] * (u64)W + (u64)win[k];
+    for (int k = av.n_fixed; k < N; ++k) idx = idx * ((u64)ctx->M[k] * (u64)W) + (u64)cfg[k] * (u64)W + (u64)win[k];
     double cost = 0.0;
     int64_t lat = 0;
     uint8_t ok = 0;
-    if ((rc = smiless_evaluate(ctx, a, (const uint64_t *)&idx, 1, &cost, &lat, &ok))) return rc;
+    if ((rc = smiless_evaluate(ctx, &av, (const uint64_t *)&idx, 1, &cost, &lat, &ok))) return rc;
     memset(res, 0, sizeof *res);
     res->n_decided = res->n_full_evals = 1;
     if (n_paths) *n_paths = (int64_t)paths.size();

@@ -1208,9 +1208,9 @@ def test_decompose_plan_full_size(name):
     assert n_paths >= 2
     if r.feasible:
         Wn = len(p.windows_us)
-        kw = {}
-        oc, ol, of = OracleProblem(p).evaluate([r.index]) if name != "C5" else (None, None, None)
+        kw = dict(n_fixed=1, fixed_digits=[int(r.config[0]) * Wn + int(r.window[0])]) if name == "C5" else {}
+        oc, ol, of = OracleProblem(p, **kw).evaluate([r.index])
+        assert of[0] and oc[0] == r.cost and ol[0] == r.max_latency_us
         if name != "C5":
-            assert of[0] and oc[0] == r.cost
             opt = pl.plan(p.arrivals_us, p.sla_us, p.windows_us)
             assert opt.feasible and opt.cost <= r.cost

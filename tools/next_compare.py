@@ -1,6 +1,8 @@
 """NEXT-1 / NEXT-2 / NEXT-3 on the BASELINE configs: exhaustive OPT over configs x window grid vs
 exhaustive OPT under the paper's derived windows (NEXT-1) vs SMIless's Top-1 path search
-(NEXT-2, the paper's deployed heuristic), all exact under model M on one GPU.  This is the
+(NEXT-2, the paper's deployed heuristic) vs DAG decomposition (NEXT-3: closed-form Top-1 per
+path, and exhaustive model-M plans per path on the GPU), all exact under model M on one GPU
+(C3 / C5 with their scale-out instances, NEXT-4).  This is the
 paper's Fig. 8 comparison "SMIless vs OPT (exhaustive search)" on synthetic inputs."""
 import json, sys, time
 sys.path.insert(0, '.')
@@ -48,6 +50,16 @@ def run(name, p, check=True):
     dc, n_paths = plq.decompose_search(p.arrivals_us, q.sla_us, it, rw)
     out["decompose_search"] = {"cost": dc.cost if dc.feasible else None, "s": time.perf_counter() - t0,
                                "paths": n_paths, "config": dc.config.tolist()}
+    t0 = time.perf_counter()
+    dm, n_paths_m = pl.decompose_plan(arr, p.sla_us, p.windows_us)    # NEXT-3 with model M (GPU per path)
+    out["decompose_plan_model_m"] = {"cost": dm.cost if dm.feasible else None, "s": time.perf_counter() - t0,
+                                     "paths": n_paths_m, "config": dm.config.tolist(), "window": dm.window.tolist()}
+    if dm.feasible:
+        pin = dict(n_fixed=1, fixed_digits=[int(dm.config[0]) * Wn + int(dm.window[0])]) if fixed else {}
+        c, l, f = OracleProblem(p, **pin).evaluate([dm.index])
+        out["decompose_plan_model_m"]["oracle_check"] = bool(f[0] and c[0] == dm.cost and l[0] == dm.max_latency_us)
+    if full.feasible and dm.feasible:
+        out["decompose_model_m_over_opt"] = dm.cost / full.cost
     if full.feasible and dc.feasible:
         out["decompose_over_opt"] = dc.cost / full.cost
     if full.feasible and h.feasible:
