@@ -768,8 +768,10 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_SPLITCOST " << (split_cost() ? 1 : 0) << "\n";
     // window variants of the memoised kernel walked in the positive-time form (evaluator.cuh
     // variants_step FM: ALU busy mask + full-rate IMAD instead of the quarter-rate IMAD.HI)
+    // default: every window variant (measured: 3.45e8 -> 3.81e8 candidates/s on the C2 slice,
+    // profiles/r02_sweep_fmask.md); the keep-alive variant needs no mask either way
     const char *fm_env = getenv("SMILESS_FMASK");
-    s << "#define SM_FMASK " << (fm_env ? strtoul(fm_env, nullptr, 0) : 0ul) << "u\n";
+    s << "#define SM_FMASK " << (fm_env ? strtoul(fm_env, nullptr, 0) : 0xfffffffful) << "u\n";
     // scale-out (NEXT-4): any instance count > 1, the prologue length, the ring size
     s << "#define SM_INST " << (kd.virt ? 1 : 0) << "\n#define SM_PRO " << P << "\n#define SM_RG_ALLOC "
       << std::max(n_rg, 1) << "\n";
