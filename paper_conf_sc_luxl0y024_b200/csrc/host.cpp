@@ -406,7 +406,7 @@ int ensure_device(smiless_ctx *ctx) {
     for (auto &ev : ctx->ev) CK(cudaEventCreate(&ev), "cudaEventCreate");
     CK(cudaMallocHost((void **)&ctx->hRes, sizeof(ResBlock) * SMILESS_MAX_SLAS), "cudaMallocHost");
     CK(ctx->dRes.ensure(SMILESS_MAX_SLAS), "cudaMalloc");
-    CK(ctx->dScal.ensure(34), "cudaMalloc");          // [0] R, [1] o_last, [2..34) scale-out tail sums
+    CK(ctx->dScal.ensure(546), "cudaMalloc");         // [0] R, [1] o_last, [2..546) scale-out sums (prep_tail)
     CK(ctx->dErr.ensure(1), "cudaMalloc");
     CK(ctx->dCounter.ensure(1), "cudaMalloc");
     CK(ctx->dStats.ensure(2), "cudaMalloc");
@@ -622,7 +622,6 @@ struct KDag {
     std::vector<std::vector<int>> preds;
     std::vector<int> M, row0, inst;
     u64 sink = 0;
-    std::vector<char> taint;     // scale-out function or downstream of one (bound kernel: lower bounds)
 };
 
 KDag kernel_dag(const smiless_ctx *ctx, const smiless_plan_args *a) {
@@ -633,7 +632,6 @@ KDag kernel_dag(const smiless_ctx *ctx, const smiless_plan_args *a) {
     d.M.resize(d.N);
     d.row0.resize(d.N);
     d.inst.resize(d.N, 1);
-    d.taint.resize(d.N, 0);
     for (int k = 0; k < ctx->N; ++k) {
         for (int e = ctx->pred_ptr[k]; e < ctx->pred_ptr[k + 1]; ++e) d.preds[k].push_back(ctx->pred_idx[e]);
         d.M[k] = ctx->M[k];
@@ -649,10 +647,6 @@ KDag kernel_dag(const smiless_ctx *ctx, const smiless_plan_args *a) {
         d.sink = 1ull << v;
     } else {
         d.sink = ctx->sinkmask;
-    }
-    for (int k = 0; k < d.N; ++k) {
-        d.taint[k] = d.inst[k] > 1;
-        for (int q : d.preds[k]) d.taint[k] |= d.taint[q];
     }
     return d;
 }
@@ -921,29 +915,34 @@ static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
         for (int k = 0; k < N; ++k)
             if ((kd.sink >> k) & 1ull) s << "  nl = vminz(nl, NF[" << k << "], z);\n";
         s << "  (void)z;\n}\n";
-        // Lower bounds of every done time: an assigned function (k < DD) is exact under model M
-        // only if no scale-out function is it or upstream of it (a scale-out function is
-        // bounded, and model M's start is not monotone in f); otherwise every branch of model M
-        // has start >= max(x, f) (one instance) or start >= x (several), so keep-alive with
-        // max(x, f) + I (one instance) or x + I (several) is a lower bound, monotone in its
-        // lower-bounded inputs.  Relaxed functions (k >= DD) take their smallest exec time.
-        s << "template <int DD, int A> static __device__ __forceinline__ void dag_bstep(tm_t (&NF)[A], const tm_t "
-             "(&NI)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], const tm_t o, tm_t &nl, const tm_t z) {\n"
-             "  tm_t su = 0;\n";
+        // Lower bounds of every done time.  An assigned function (k < DD) has exact inputs (all its
+        // predecessors are assigned) and runs model M exactly, with its instance ring.  A relaxed
+        // function (k >= DD) runs keep-alive on its smallest exec time: max(x', D'_{j-n}) + I_min
+        // (a ring of n_k - 1 older bounds for n_k > 1; the first request of an instance x' + I_min)
+        // -- in every branch of model M start >= max(x, D_{j-n}), and that bound is monotone in its
+        // lower-bounded inputs.
+        s << "template <int DD, int JJ, int A, int R> static __device__ __forceinline__ void dag_bstep(tm_t (&NF)[A], "
+             "tm_t (&RG)[R], const tm_t (&NI)[A], const tm_t (&Te)[A], const tm_t (&Wn)[A], const tm_t o, tm_t &nl, "
+             "const tm_t z) {\n  tm_t su = 0;\n";
         for (int k = 0; k < N; ++k) {
-            const std::string g = is_src(k) ? "o + NF[" + ks(k) + "]" : "NF[" + ks(k) + "] - " + nf_min(k);
+            const int n = kd.inst[k];
             const std::string nx = is_src(k) ? std::string("opaque_sub(z, o)") : nf_min(k);
-            if (kd.inst[k] > 1) {
-                s << "  NF[" << k << "] = NI[" << k << "] + " << nx << ";\n";
-            } else if (kd.taint[k]) {
-                s << "  { const tm_t g = " << g << "; NF[" << k << "] = NF[" << k << "] + NI[" << k
-                  << "] - vmax(g, (tm_t)0); }\n";
-            } else {
-                // assigned (k < DD): model M; relaxed: keep-alive (start - f = max(g, 0)), smallest exec
+            if (n == 1) {
+                const std::string g = is_src(k) ? "o + NF[" + ks(k) + "]" : "NF[" + ks(k) + "] - " + nf_min(k);
                 s << "  if (" << k << " < DD) fstep(NF[" << k << "], su, " << g << ", NI[" << k << "], Te[" << k
                   << "], Wn[" << k << "]);\n  else { const tm_t g = " << g << "; NF[" << k << "] = NF[" << k
                   << "] + NI[" << k << "] - vmax(g, (tm_t)0); }\n";
+                continue;
             }
+            const std::string g = is_src(k) ? std::string("o + nf") : "nf - " + nf_min(k);
+            s << "  {\n    tm_t nf = RG[" << rg0[k] << "];\n";
+            for (int r = 0; r + 1 < n - 1; ++r) s << "    RG[" << rg0[k] + r << "] = RG[" << rg0[k] + r + 1 << "];\n";
+            s << "    RG[" << rg0[k] + n - 2 << "] = NF[" << k << "];\n";
+            s << "    if (JJ != 0 && JJ < " << n << ") NF[" << k << "] = NI[" << k << "] + " << nx << ";\n";
+            s << "    else if (" << k << " < DD) { fstep(nf, su, " << g << ", NI[" << k << "], Te[" << k << "], Wn[" << k
+              << "]); NF[" << k << "] = nf; }\n";
+            s << "    else { const tm_t g = " << g << "; NF[" << k << "] = nf + NI[" << k << "] - vmax(g, (tm_t)0); }\n";
+            s << "  }\n";
         }
         for (int k = 0; k < N; ++k)
             if ((kd.sink >> k) & 1ull) s << "  nl = vaddmin(NF[" << k << "], o, nl);\n";

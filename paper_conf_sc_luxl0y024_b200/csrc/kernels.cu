@@ -76,6 +76,19 @@ __global__ void prep_tail_kernel(const i64 *__restrict__ arr, i64 J, i64 d_cap, 
         }
         scal[18 + i] = o;
     }
+    // per instance count n = 1..16 and instance i < n (requests i, i + n, ...): the real span
+    // R_i = r_{last_i} - r_i at scal[34 + (n-1)*16 + i] and the request count c_i at
+    // scal[290 + (n-1)*16 + i] (0 when i >= J): the static cost bound of a scale-out function
+    for (int n = 1; n <= 16; ++n)
+        for (int i = 0; i < 16; ++i) {
+            i64 span = 0, cnt = 0;
+            if (i < n && i < J) {
+                cnt = (J - 1 - i) / n + 1;
+                span = arr[i + (cnt - 1) * n] - arr[i];
+            }
+            scal[34 + (n - 1) * 16 + i] = span;
+            scal[290 + (n - 1) * 16 + i] = cnt;
+        }
 }
 
 __device__ __forceinline__ bool key_less(u64 ca, u64 ia, u64 cb, u64 ib) {
