@@ -55,6 +55,8 @@ def main():
                 kw["cost_cap"] = best[0]
             r = pl.plan(arr, p.sla_us, p.windows_us, **kw)
             per_digit.append(round((time.perf_counter() - td) * 1e3, 3))
+            print(f"digit {d}: {per_digit[-1]} ms, feasible {r.feasible}, decided {r.n_decided}, "
+                  f"full {r.n_full_evals}, best {best[0] if best else None}", file=sys.stderr, flush=True)
             decided += r.n_decided
             full += r.n_full_evals
             launches += r.launches
