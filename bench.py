@@ -433,7 +433,8 @@ def run_reference(args):
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "i64+f64",
         "data": "synthetic", "config": config_block(p, kw, args),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
-                         "sample": f"{n_step} consecutive candidates of the slice per step"},
+                         "sample": f"{n_step} consecutive candidates of the slice per step",
+                         "cpu_model": host_cpu()["model"], "cpu_mhz": host_cpu()["mhz"]},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
