@@ -130,8 +130,27 @@ __global__ void reduce_best_kernel(const u64 *__restrict__ slots, int n, int str
 // one iteration of the warp instead of N dependent steps of one thread.
 #define EXACT_WARPS 4
 
+// arrivals staged per warp in a shared ring of 512 (4 blocks of 128), each block fetched with
+// cp.async 256 invocations before it is read (the lanes read j in [it - 31, it])
+#define EXACT_ARR_RING 512
+#define EXACT_ARR_BLOCK 128
+
+__device__ __forceinline__ void exact_fetch_block(long long *ring_arr, const long long *arr, i64 J, i64 b, int lane) {
+    // block b = arrivals [b * 128, b * 128 + 128): 8-byte copies (any int64-aligned source), 4 per
+    // lane; past J: nothing
+    for (int q = lane; q < EXACT_ARR_BLOCK; q += 32) {
+        const i64 j0 = b * EXACT_ARR_BLOCK + q;
+        if (j0 < J) {
+            const unsigned dst = (unsigned)__cvta_generic_to_shared(ring_arr + (j0 & (EXACT_ARR_RING - 1)));
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(dst), "l"(arr + j0) : "memory");
+        }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
 __global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParams p) {
     __shared__ long long ring[EXACT_WARPS][SMILESS_DEV_MAX_FUNCS][32];   // [warp][function][j % 32]
+    __shared__ __align__(16) long long ring_arr[EXACT_WARPS][EXACT_ARR_RING];
     const unsigned FULL = 0xffffffffu;
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const i64 t = ((i64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;   // candidate of this warp
@@ -188,12 +207,23 @@ __global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParam
     long long (*rg)[32] = ring[wib];
     const i64 J = p.J;
     i64 D = 0, billed = 0, maxlat = INT64_MIN;
-    i64 rcur = act ? p.arr[0] : 0;                        // r_j of this lane's next invocation
+    long long *ra = ring_arr[wib];
+    // blocks 0, 1 now (waited for), block m + 2 at iteration 128 m (waited for 128 iterations later)
+    exact_fetch_block(ra, p.arr, J, 0, lane);
+    exact_fetch_block(ra, p.arr, J, 1, lane);
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    __syncwarp();
     for (i64 it = 0; it < J + nlev - 1; ++it) {
+        if ((it & (EXACT_ARR_BLOCK - 1)) == 0) {
+            // the previous fetch (block it / 128 + 1, read from the next block boundary on) has
+            // landed once at most the newest group is pending; then fetch block it / 128 + 2
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
+            __syncwarp();
+            exact_fetch_block(ra, p.arr, J, it / EXACT_ARR_BLOCK + 2, lane);
+        }
         const i64 j = it - lvl;
         const bool on = act && j >= 0 && j < J;
-        const i64 r = rcur;
-        if (on && j + 1 < J) rcur = p.arr[j + 1];          // prefetch for the next iteration
+        const i64 r = on ? ra[j & (EXACT_ARR_RING - 1)] : 0;
         if (on) {
             i64 x = r;                                    // sources: the request's arrival
             const int sl = (int)(j & 31);
