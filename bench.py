@@ -155,7 +155,7 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier, sla=
     import torch
     import torch.distributed as dist
     from paper_conf_sc_luxl0y024_b200.dist import (cost_bits, bits_cost, reduce_lex, plan_pinned_rounds,
-                                                   plan_range_rounds, INF_BITS)
+                                                   plan_range_rounds, plan_digits_sharded, INF_BITS)
     rounds = int(os.environ.get("SMILESS_BENCH_ROUNDS", "1" if world == 1 else "2"))
     p = W.make_config(name)
     if sla is not None:
@@ -188,10 +188,19 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier, sla=
         cap0 = bits_cost(int(cb.item())) if int(cb.item()) != INF_BITS else None
         seed_ms = (time.perf_counter() - ts) * 1e3
     if pinned:
-        best, decided, full_evals, _ = plan_pinned_rounds(
-            lambda d0, cap: pl.plan(arr, p.sla_us, p.windows_us, n_fixed=1, fixed_digits=[d0],
-                                    **({"cost_cap": cap} if cap is not None else {})),
-            digits, rank, world, xdev, initial_cap=cap0)
+        # every rank plans every function-0 digit on its interleaved shard, incumbent exchanged
+        # after each digit (a heavy digit is split across the GPUs); SMILESS_BENCH_DIGITS=rr
+        # deals whole digits round-robin instead (dist.plan_pinned_rounds)
+        if os.environ.get("SMILESS_BENCH_DIGITS", "sharded") == "rr":
+            best, decided, full_evals, _ = plan_pinned_rounds(
+                lambda d0, cap: pl.plan(arr, p.sla_us, p.windows_us, n_fixed=1, fixed_digits=[d0],
+                                        **({"cost_cap": cap} if cap is not None else {})),
+                digits, rank, world, xdev, initial_cap=cap0)
+        else:
+            best, decided, full_evals, _ = plan_digits_sharded(
+                lambda d0, cap: pl.plan(arr, p.sla_us, p.windows_us, n_fixed=1, fixed_digits=[d0], shard=rank,
+                                        n_shards=world, **({"cost_cap": cap} if cap is not None else {})),
+                digits, rank, world, xdev, initial_cap=cap0)
     else:
         # one exact plan, every rank on its interleaved share of every B&B survivor's subtree;
         # with N > 1 the index range runs in `rounds` pieces and the ranks exchange the

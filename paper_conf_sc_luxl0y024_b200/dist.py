@@ -162,3 +162,32 @@ def plan_range_rounds(plan_range, space, rounds, rank, world, device, group=None
             dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
             cap_bits = int(t.item())
     return best, decided, full_evals, caps
+
+
+def plan_digits_sharded(plan_digit, digits, rank, world, device, group=None, initial_cap=None):
+    """Sub-spaces (one per value of a pinned leading digit, e.g. C5's 2^70 = 128 x 2^63) planned
+    one after the other by EVERY rank on its interleaved shard (plan_digit(d, cap) calls
+    smiless_plan with shard=rank, n_shards=world), so a heavy digit is split across the GPUs
+    like any single plan.  After every digit the ranks MIN-all-reduce
+    their cheapest feasible cost and pass it as the next digit's cost cap (exact for any cap
+    >= OPT, see plan_range_rounds).
+
+    Returns (best, decided, full_evals, caps) like plan_pinned_rounds: best = (cost, digit,
+    index, max_latency) of this rank or None."""
+    best, decided, full_evals, caps = None, 0, 0, []
+    cap_bits = cost_bits(initial_cap) if initial_cap is not None else INF_BITS
+    for i, d0 in enumerate(digits):
+        cap = bits_cost(cap_bits) if cap_bits != INF_BITS else None
+        caps.append(cap)
+        r = plan_digit(d0, cap)
+        decided += r.n_decided
+        full_evals += r.n_full_evals
+        if r.feasible and (best is None or (r.cost, d0, r.index) < best[:3]):
+            best = (r.cost, d0, r.index, r.max_latency_us)
+        if best is not None:
+            cap_bits = min(cap_bits, cost_bits(best[0]))
+        if world > 1 and i + 1 < len(digits):
+            t = torch.tensor([cap_bits], dtype=torch.int64, device=device)
+            dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+            cap_bits = int(t.item())
+    return best, decided, full_evals, caps

@@ -274,3 +274,65 @@ def test_range_rounds_with_in_plan_incumbent_exchange(world, rounds, zero_prices
         assert len(caps) == rounds and all(cp is None or cp >= ref_cost for cp in caps)
         if rounds > 1:
             assert caps[-1] is not None       # the global incumbent reached every rank's last round
+
+
+def _digits_sharded_worker(rank, world, port, zero_prices, out_q):
+    """C1 as 16 function-0 digits, EVERY rank planning every digit on its interleaved shard
+    (emulated on the oracle's per-candidate costs with the library's semantics), the
+    incumbent exchanged after each digit."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import workloads as W
+    from oracle import OracleProblem
+    from paper_conf_sc_luxl0y024_b200.dist import plan_digits_sharded, reduce_lex
+    p = W.make_config("C1", n_arrivals=40)
+    if zero_prices:
+        p = p.replace(price_per_us=np.zeros_like(p.price_per_us))
+    c, l, f = OracleProblem(p).evaluate(np.arange(4096, dtype=np.uint64))
+
+    def plan_digit(d, cap):
+        s_ = np.arange(256)
+        s_ = s_[s_ % world == rank]                     # this rank's share of the digit
+        g = d * 256 + s_
+        ok = f[g] & (c[g] <= (np.inf if cap is None else cap))
+        if not ok.any():
+            return _Res(False, float("inf"), None, -1, len(s_))
+        k = s_[ok][np.lexsort((s_[ok], c[g][ok]))[0]]
+        return _Res(True, float(c[d * 256 + k]), int(k), int(l[d * 256 + k]), len(s_))
+
+    best, dec, _, caps = plan_digits_sharded(plan_digit, list(range(16)), rank, world, "cpu")
+    keys = [cost_bits(best[0]) if best else INF_BITS, best[1] if best else 0, best[2] if best else 0]
+    keys, pay = reduce_lex(keys, [best[3] if best else -1], "cpu")
+    out_q.put((rank, (keys, pay, dec, caps)))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,zero_prices", [(2, False), (3, False), (2, True)])
+def test_digits_sharded_with_global_cost_cap(world, zero_prices):
+    """bench.py's C5 driver (dist.plan_digits_sharded): every rank decides its share of every
+    digit, the caps are real feasible costs, and the reduced (cost, digit, index) is the
+    oracle's OPT with the lowest-index tie-break."""
+    import workloads as W
+    from oracle import OracleProblem
+    p = W.make_config("C1", n_arrivals=40)
+    if zero_prices:
+        p = p.replace(price_per_us=np.zeros_like(p.price_per_us))
+    ref_idx, ref_cost, ref_lat = OracleProblem(p).plan()
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_digits_sharded_worker, args=(r, world, port, zero_prices, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    out = dict(q.get(timeout=180) for _ in range(world))
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    assert sum(out[r][2] for r in range(world)) == 4096
+    for r in range(world):
+        keys, pay, dec, caps = out[r]
+        assert dec >= 4096 // (2 * world)
+        assert bits_cost(keys[0]) == ref_cost and keys[1] * 256 + keys[2] == ref_idx and pay[0] == ref_lat
+        assert all(cp is None or cp >= ref_cost for cp in caps)
