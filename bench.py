@@ -240,7 +240,7 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier, sla=
     cost = bits_cost(keys[0])
     out = {"candidates": decided, "time_to_optimal_s": sec, "wall_s": wall, "decided_per_s": decided / sec,
            "sla_us": p.sla_us, "instances": None if p.instances is None else p.instances.tolist(),
-           "full_evals_local": full_evals, "decided_per_rank": per_rank, "full_evals_per_rank": per_rank_full,
+           "full_evals_local": full_evals, "digits": ("rr" if os.environ.get("SMILESS_BENCH_DIGITS") == "rr" else "sharded") if pinned else None, "decided_per_rank": per_rank, "full_evals_per_rank": per_rank_full,
            "rounds": 1 if pinned else rounds,
            "cost": cost, "max_latency_us": lat if cost is not None else -1,
            "seed_cap": {"enabled": seed, "cap": cap0, "wall_ms": seed_ms}}
