@@ -280,6 +280,19 @@ SMILESS_API int smiless_decompose_search(smiless_ctx *ctx, const smiless_plan_ar
 SMILESS_API int smiless_decompose_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res,
                                        int32_t *config_out, int32_t *window_out, int64_t *n_paths);
 
+/* Multi-GPU form of smiless_decompose_plan ("the Strategy Optimizer executes the basic
+ * algorithm in parallel for each subgraph"): every rank calls it with a->shard /
+ * a->n_shards; each path's exhaustive plan then covers this rank's interleaved share of the
+ * path's space, and after each path the library calls reduce(user, path, res) -- the caller's
+ * collective, which must replace res->index / cost / max_latency_us with the ranks' global
+ * lexicographic (cost, index) winner (index UINT64_MAX if no rank has a feasible one) and
+ * return 0.  The library decodes that winner and every rank then combines identically.  The
+ * library itself never communicates.  reduce == NULL is smiless_decompose_plan. */
+typedef int (*smiless_path_reduce_fn)(void *user, int32_t path, smiless_plan_result *res);
+SMILESS_API int smiless_decompose_plan_sharded(smiless_ctx *ctx, const smiless_plan_args *a,
+                                               smiless_path_reduce_fn reduce, void *user, smiless_plan_result *res,
+                                               int32_t *config_out, int32_t *window_out, int64_t *n_paths);
+
 /* SLA sweep (C4: "impact of SLA settings"): ONE evaluation of the space
  * with one argmin key per SLA in slas[0..n_sla) (1 <= n_sla <= SMILESS_MAX_SLAS); pruning uses
  * their maximum; a->sla_us is ignored and a->cost_out must be NULL.  res[n_sla] and, when not

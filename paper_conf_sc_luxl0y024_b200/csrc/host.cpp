@@ -2295,8 +2295,9 @@ int smiless_decompose_search(smiless_ctx *ctx, const smiless_plan_args *a, int64
     return SMILESS_OK;
 }
 
-int smiless_decompose_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res,
-                           int32_t *config_out, int32_t *window_out, int64_t *n_paths) {
+int smiless_decompose_plan_sharded(smiless_ctx *ctx, const smiless_plan_args *a, smiless_path_reduce_fn reduce,
+                                   void *user, smiless_plan_result *res, int32_t *config_out, int32_t *window_out,
+                                   int64_t *n_paths) {
     if (!ctx) return SMILESS_EINVAL;
     ctx->err.clear();
     if (!a || !res) return fail(ctx, SMILESS_EINVAL, "args / res is NULL");
@@ -2381,6 +2382,7 @@ int smiless_decompose_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless
         pa.shard = 0;
         pa.n_shards = 0;
         pa.cost_out = nullptr;
+        pa.cost_cap = 0.0;
         pa.flags = a->flags & (SMILESS_FLAG_ARRIVALS_ON_DEVICE | SMILESS_FLAG_FORCE_INT64);
         inst.clear();
         for (int k : P) inst.push_back(inst_of(a, k));
@@ -2396,10 +2398,27 @@ int smiless_decompose_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless
         smiless_ctx *c = nullptr;
         if ((rc = sub_for(P, &c))) return rc;
         smiless_plan_args pa = path_args(P, inst);
+        if (reduce) {                                    // this rank's interleaved share of the path
+            pa.shard = a->shard;
+            pa.n_shards = a->n_shards;
+        }
         smiless_plan_result pr;
         std::vector<int32_t> co(P.size()), wo(P.size());
         rc = smiless_plan(c, &pa, &pr, co.data(), wo.data());
         if (rc < 0) return fail(ctx, rc, "decompose: path plan: %s", smiless_last_error(c));
+        if (reduce) {
+            // the caller reduces the ranks' path winners (its collective) into pr
+            const int rr = reduce(user, (int32_t)pi, &pr);
+            if (rr) return fail(ctx, SMILESS_EINVAL, "decompose: path reduce callback returned %d", rr);
+            rc = pr.index == ~0ull ? SMILESS_INFEASIBLE : SMILESS_OK;
+            if (rc == SMILESS_OK) {
+                pa.shard = 0;
+                pa.n_shards = 0;
+                const int dr = smiless_decode(c, W, pr.index, &pa, co.data(), wo.data());
+                if (dr) return fail(ctx, dr, "decompose: reduced path winner %llu does not decode",
+                                    (unsigned long long)pr.index);
+            }
+        }
         if (rc == SMILESS_INFEASIBLE) {                  // no plan meets the SLA on this path alone
             memset(res, 0, sizeof *res);
             res->index = ~0ull;
@@ -2435,7 +2454,7 @@ int smiless_decompose_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless
         const auto &P = paths[pi];
         smiless_ctx *c = nullptr;
         if ((rc = sub_for(P, &c))) return rc;
-        smiless_plan_args pa = path_args(P, inst);
+        smiless_plan_args pa = path_args(P, inst);         // (every rank evaluates these itself)
         for (size_t q = 0; q < P.size(); ++q) {
             const int k = P[q];
             if (n_on[k] != 1) continue;
@@ -2489,6 +2508,11 @@ int smiless_decompose_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless
     res->cost = cost;
     res->max_latency_us = lat;
     return SMILESS_OK;
+}
+
+int smiless_decompose_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res,
+                           int32_t *config_out, int32_t *window_out, int64_t *n_paths) {
+    return smiless_decompose_plan_sharded(ctx, a, nullptr, nullptr, res, config_out, window_out, n_paths);
 }
 
 int smiless_plan_sla_sweep(smiless_ctx *ctx, const smiless_plan_args *a, const int64_t *slas, int32_t n_sla,

@@ -191,3 +191,25 @@ def plan_digits_sharded(plan_digit, digits, rank, world, device, group=None, ini
             dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
             cap_bits = int(t.item())
     return best, decided, full_evals, caps
+
+
+def decompose_plan_distributed(planner, arrivals, sla_us, windows_us, group=None, device=None, **kw):
+    """NEXT-3 with model M on N GPUs: every rank plans its interleaved share of each source-to-
+    sink path (smiless_decompose_plan_sharded) and the path winners are reduced with the same
+    two MIN all-reduces as a plan (reduce_best), inside the library's callback.  Every rank
+    returns the same combined plan: (PlanResult, number of paths)."""
+    rank = dist.get_rank(group)
+    world = dist.get_world_size(group)
+    if device is None:
+        device = torch.device("cuda", torch.cuda.current_device()) if torch.cuda.is_available() else "cpu"
+
+    def reduce(path, res):
+        feasible = res.index != (1 << 64) - 1
+        cost, index, lat, _ = reduce_best(res.cost if feasible else None, res.index if feasible else None,
+                                          res.max_latency_us, res.n_decided, device, group)
+        if index is None:
+            res.index, res.cost, res.max_latency_us = (1 << 64) - 1, float("inf"), -1
+        else:
+            res.index, res.cost, res.max_latency_us = index, cost, lat
+
+    return planner.decompose_plan(arrivals, sla_us, windows_us, reduce=reduce, shard=rank, n_shards=world, **kw)

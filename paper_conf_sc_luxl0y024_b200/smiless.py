@@ -26,6 +26,7 @@ _NAMES = {0: "OK", 1: "INFEASIBLE", -1: "EINVAL", -2: "ENOTTOPO", -3: "ERANGE", 
 EXPORTS = ("smiless_create", "smiless_set_stream", "smiless_destroy", "smiless_last_error",
            "smiless_load_dag", "smiless_load_profiles", "smiless_space_size", "smiless_plan",
            "smiless_plan_sla_sweep", "smiless_derive_windows", "smiless_top1_search", "smiless_decompose_search", "smiless_decompose_plan",
+           "smiless_decompose_plan_sharded",
            "smiless_autoscale", "smiless_autoscale_rows",
            "smiless_evaluate",
            "smiless_decode",
@@ -73,6 +74,10 @@ class PlanResultC(ctypes.Structure):
         ("h2d_bytes", ctypes.c_uint64),
         ("d2h_bytes", ctypes.c_uint64),
     ]
+
+
+# int (*smiless_path_reduce_fn)(void *user, int32_t path, smiless_plan_result *res)
+PATH_REDUCE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(PlanResultC))
 
 
 @dataclasses.dataclass
@@ -132,6 +137,8 @@ def load_library(build_if_missing: bool = True):
                                         ctypes.POINTER(ctypes.c_int64)]
     lib.smiless_decompose_plan.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.POINTER(PlanResultC), vp, vp,
                                            ctypes.POINTER(ctypes.c_int64)]
+    lib.smiless_decompose_plan_sharded.argtypes = [vp, ctypes.POINTER(PlanArgs), PATH_REDUCE_FN, vp,
+                                                   ctypes.POINTER(PlanResultC), vp, vp, ctypes.POINTER(ctypes.c_int64)]
     lib.smiless_evaluate.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i64, vp, vp, vp]
     lib.smiless_decode.argtypes = [vp, i32, u64, ctypes.POINTER(PlanArgs), vp, vp]
     lib.smiless_kernel_source.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.c_char_p, ctypes.c_size_t,
@@ -351,17 +358,33 @@ class Planner:
                           window=win[:self.n_funcs], n_decided=1, n_full_evals=1, eval_kernel_ms=0.0,
                           total_device_ms=0.0, int64_path=False, launches=0), int(n.value)
 
-    def decompose_plan(self, arrivals, sla_us, windows_us, **kw):
+    def decompose_plan(self, arrivals, sla_us, windows_us, reduce=None, **kw):
         """NEXT-3 with model M (smiless_decompose_plan): exhaustive GPU plan per source-to-sink
-        path, the paper's combine; returns (PlanResult, number of paths)."""
+        path, the paper's combine; returns (PlanResult, number of paths).  With `reduce`
+        (a callable (path, PlanResultC) -> None that replaces the result's index / cost /
+        max_latency_us with the ranks' global winner) and shard / n_shards in kw, the path
+        plans are sharded over ranks (smiless_decompose_plan_sharded)."""
         a, keep = self._args(arrivals, sla_us, windows_us, **kw)
         r = PlanResultC()
         cfg = np.zeros(max(self.n_funcs, 1), np.int32)
         win = np.zeros(max(self.n_funcs, 1), np.int32)
         npaths = ctypes.c_int64()
-        rc = self._check(self._lib.smiless_decompose_plan(self._ctx, ctypes.byref(a), ctypes.byref(r), cfg.ctypes.data,
-                                                          win.ctypes.data, ctypes.byref(npaths)),
-                         allow=(OK, INFEASIBLE))
+        if reduce is None:
+            rc = self._check(self._lib.smiless_decompose_plan(self._ctx, ctypes.byref(a), ctypes.byref(r),
+                                                              cfg.ctypes.data, win.ctypes.data, ctypes.byref(npaths)),
+                             allow=(OK, INFEASIBLE))
+        else:
+            def _cb(user, path, res_p):
+                try:
+                    reduce(int(path), res_p.contents)
+                    return 0
+                except Exception:               # pragma: no cover  (reported as EINVAL by the library)
+                    return 1
+            cb = PATH_REDUCE_FN(_cb)
+            rc = self._check(self._lib.smiless_decompose_plan_sharded(self._ctx, ctypes.byref(a), cb, None,
+                                                                      ctypes.byref(r), cfg.ctypes.data,
+                                                                      win.ctypes.data, ctypes.byref(npaths)),
+                             allow=(OK, INFEASIBLE))
         del keep
         return PlanResult(status=rc, index=None if rc == INFEASIBLE else int(r.index), cost=float(r.cost),
                           max_latency_us=int(r.max_latency_us), config=cfg[:self.n_funcs],

@@ -1214,3 +1214,49 @@ def test_decompose_plan_full_size(name):
         if name != "C5":
             opt = pl.plan(p.arrivals_us, p.sla_us, p.windows_us)
             assert opt.feasible and opt.cost <= r.cost
+
+
+def _decompose_rank(rank, world, port, name, out_q):
+    import os
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    torch.cuda.set_device(0)
+    from paper_conf_sc_luxl0y024_b200.dist import decompose_plan_distributed
+    p = W.make_config(name) if name != "rand" else W.random_problem(np.random.default_rng(9), 5, 3, 2, 60,
+                                                                    sla_us=30_000)
+    pl = S.planner_for(p)
+    r, n_paths = decompose_plan_distributed(pl, p.arrivals_us, p.sla_us, p.windows_us, device="cpu")
+    out_q.put((rank, (r.status, r.index, r.cost, r.max_latency_us, r.config.tolist(), r.window.tolist(), n_paths)))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("name,world", [("C3", 2), ("C2", 3), ("rand", 2)])
+def test_decompose_plan_sharded_over_ranks(name, world):
+    """NEXT-3 per-path GPU sharding: `world` ranks (processes on this one GPU,
+    gloo collectives inside the library's reduce callback) each plan their share of every
+    path; every rank returns the single-rank decomposition exactly."""
+    import socket
+    import torch.multiprocessing as mp
+    p = W.make_config(name) if name != "rand" else W.random_problem(np.random.default_rng(9), 5, 3, 2, 60,
+                                                                    sla_us=30_000)
+    one, n_paths = S.planner_for(p).decompose_plan(p.arrivals_us, p.sla_us, p.windows_us)
+    sock = socket.socket()
+    sock.bind(("127.0.0.1", 0))
+    port = sock.getsockname()[1]
+    sock.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_decompose_rank, args=(r, world, port, name, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    out = dict(q.get(timeout=600) for _ in range(world))
+    for pr in procs:
+        pr.join(timeout=120)
+        assert pr.exitcode == 0
+    want = (one.status, one.index, one.cost, one.max_latency_us, one.config.tolist(), one.window.tolist(), n_paths)
+    for r in range(world):
+        assert out[r] == want
