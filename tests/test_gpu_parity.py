@@ -1260,3 +1260,20 @@ def test_decompose_plan_sharded_over_ranks(name, world):
     want = (one.status, one.index, one.cost, one.max_latency_us, one.config.tolist(), one.window.tolist(), n_paths)
     for r in range(world):
         assert out[r] == want
+
+
+def test_arrivals_device_view_at_8_byte_offset():
+    """Arrivals as a device tensor view 8 bytes into its allocation (only int64-aligned):
+    the plan, its exact winner re-check (cp.async arrival ring) and smiless_evaluate agree
+    with the oracle."""
+    import torch
+    p = W.make_config("C1")
+    full = torch.as_tensor(np.concatenate([[0], p.arrivals_us])).cuda()
+    view = full[1:]
+    assert view.data_ptr() % 16 == 8
+    pl = S.planner_for(p)
+    g = pl.plan(view, p.sla_us, p.windows_us)
+    o = OracleProblem(p)
+    assert_same_plan(g, o.plan(), o)
+    idx = np.arange(0, 4096, 13, dtype=np.uint64)
+    assert_same_eval(*pl.evaluate(idx, view, p.sla_us, p.windows_us), *o.evaluate(idx))
