@@ -346,16 +346,17 @@ def measured_peaks():
         return {}
 
 
-def ncu_traffic(memo: bool, plan_launches: int):
+def ncu_traffic(memo: bool, plan_launches: int, split: bool = True):
     """DRAM bytes of the timed kernels per plan call (the unit `achieved` uses), from the
     committed ncu --set full summaries.  Memo path: one plan call = prep + B x (upstream,
-    variants) + reduce + exact, so B = (launches - 3) / 2 pairs, each pair moving the
-    upstream kernel's x-buffer write and the variants kernel's read of it."""
+    variants[, variants cost]) + reduce + exact, so B = (launches - 3) / 3 batches with the
+    split cost (2 without), each moving the upstream kernel's x-buffer write and the variants
+    kernel's read of it (the cost pass re-reads the few units with a feasible candidate)."""
     try:
         if memo:
             d = json.load(open(os.path.join(ROOT, "profiles", "ncu_memo_summary.json")))
             pair = sum(k["dram_bytes_per_launch"] for k in d["launches"])
-            return pair * max(1, (plan_launches - 3) // 2)
+            return pair * max(1, (plan_launches - 3) // (3 if split else 2))
         d = json.load(open(os.path.join(ROOT, "profiles", "ncu_evaluator_summary.json")))
         return d.get("dram_bytes_per_launch")
     except Exception:
@@ -694,8 +695,9 @@ def main():
                 "bytes_basis": "counted by the library per smiless_plan call (smiless_plan_result)"},
         "clocks": clocks,
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_ops, "unit": "int-ops/s",
-                     "frac": achieved / peak_ops, "traffic": ncu_traffic(memo, res.launches),
-                     "traffic_basis": "ncu dram__bytes_read+write per plan call (profiles/ncu_memo_summary.json)",
+                     "frac": achieved / peak_ops, "traffic": ncu_traffic(memo, res.launches, split),
+                     "traffic_basis": "ncu dram__bytes_read+write per plan call (profiles/ncu_memo_summary.json): "
+                                      "the memoised x-buffer round trip, ~5.4 GB per 65,536-prefix batch",
                      "kernel": ("smiless_variants_kernel + smiless_upstream_kernel (prefix memoisation)"
                                 if memo else "smiless_plan_kernel"),
                      "kernel_ms_per_launch": kernel_ms_per_step,
