@@ -579,6 +579,10 @@ int inst_max(const smiless_ctx *ctx, const smiless_plan_args *a) {
     return m;
 }
 bool inst_mode(const smiless_ctx *ctx, const smiless_plan_args *a) { return inst_max(ctx, a) > 1; }
+// the virtual sink (DESIGN.md section 5 item 13) is needed only when the LAST function scales
+// out: otherwise its window variants keep sink sharing and the memoised throughput path, and
+// only the upstream functions carry instance rings
+bool virt_sink(const smiless_ctx *ctx, const smiless_plan_args *a) { return inst_of(a, ctx->N - 1) > 1; }
 // prologue steps j = 1 .. P of a scale-out plan (the first request of instances 2 .. n_k), a
 // multiple of 4 so that the main loop keeps its 16-byte aligned offset loads
 int inst_prologue(const smiless_ctx *ctx, const smiless_plan_args *a) {
@@ -587,7 +591,7 @@ int inst_prologue(const smiless_ctx *ctx, const smiless_plan_args *a) {
 }
 
 int configs_per_lane(const smiless_ctx *ctx, const smiless_plan_args *a) {
-    if (inst_mode(ctx, a)) return 1;                 // last kernel function = the virtual sink (M = 1)
+    if (virt_sink(ctx, a)) return 1;                 // last kernel function = the virtual sink (M = 1)
     const int M = ctx->M[ctx->N - 1], W = a->n_windows;
     int G = 1;
     const char *env = getenv("SMILESS_G");
@@ -601,11 +605,11 @@ int configs_per_lane(const smiless_ctx *ctx, const smiless_plan_args *a) {
 // candidates per evaluator unit (lane): G configs x W windows of the last function; 1 for a
 // scale-out plan, whose last kernel function is the virtual sink (one variant)
 u64 unit_cands(const smiless_ctx *ctx, const smiless_plan_args *a) {
-    return inst_mode(ctx, a) ? 1 : (u64)a->n_windows * (u64)configs_per_lane(ctx, a);
+    return virt_sink(ctx, a) ? 1 : (u64)a->n_windows * (u64)configs_per_lane(ctx, a);
 }
 // window variants of the last kernel function
 int variant_windows(const smiless_ctx *ctx, const smiless_plan_args *a) {
-    return inst_mode(ctx, a) ? 1 : a->n_windows;
+    return virt_sink(ctx, a) ? 1 : a->n_windows;
 }
 
 // The DAG the evaluator kernels are specialised for.  Normally the application DAG.  For a
@@ -626,7 +630,7 @@ struct KDag {
 
 KDag kernel_dag(const smiless_ctx *ctx, const smiless_plan_args *a) {
     KDag d;
-    d.virt = inst_mode(ctx, a);
+    d.virt = virt_sink(ctx, a);
     d.N = ctx->N + (d.virt ? 1 : 0);
     d.preds.resize(d.N);
     d.M.resize(d.N);
@@ -767,7 +771,8 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     const char *fm_env = getenv("SMILESS_FMASK");
     s << "#define SM_FMASK " << (fm_env ? strtoul(fm_env, nullptr, 0) : 0xfffffffful) << "u\n";
     // scale-out (NEXT-4): any instance count > 1, the prologue length, the ring size
-    s << "#define SM_INST " << (kd.virt ? 1 : 0) << "\n#define SM_PRO " << P << "\n#define SM_RG_ALLOC "
+    s << "#define SM_INST " << (inst_mode(ctx, a) ? 1 : 0) << "\n#define SM_VIRT " << (kd.virt ? 1 : 0)
+      << "\n#define SM_PRO " << P << "\n#define SM_RG_ALLOC "
       << std::max(n_rg, 1) << "\n";
     s << "#define SM_NINST(k) (";
     for (int k = 0; k < N; ++k) s << "(k)==" << k << "?" << kd.inst[k] << ":";
@@ -953,7 +958,7 @@ static __device__ __forceinline__ tm_t vmax(tm_t a, tm_t b);
 
 std::string full_source(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, bool off_smem,
                         int minb, int families = FAM_ALL) {
-    if (inst_mode(ctx, a)) families &= ~FAM_MEMO;       // scale-out plans never take the memo path
+    if (virt_sink(ctx, a)) families &= ~FAM_MEMO;       // a scaled-out last function: no memo path
     return dag_spec_source(ctx, a, rp, off_smem, minb, families) + "\n" + smiless_evaluator_src;
 }
 
@@ -966,8 +971,8 @@ size_t smem_memo_up(const smiless_ctx *ctx, const RangePlan &rp, i64 n_off) {
 }
 size_t smem_memo_var(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off);
 // table rows the plan / bound kernels stage: a scale-out plan adds the virtual sink's zero row
-int kernel_rows(const smiless_ctx *ctx, const smiless_plan_args *a) { return ctx->sumM + (inst_mode(ctx, a) ? 1 : 0); }
-int kernel_funcs(const smiless_ctx *ctx, const smiless_plan_args *a) { return ctx->N + (inst_mode(ctx, a) ? 1 : 0); }
+int kernel_rows(const smiless_ctx *ctx, const smiless_plan_args *a) { return ctx->sumM + (virt_sink(ctx, a) ? 1 : 0); }
+int kernel_funcs(const smiless_ctx *ctx, const smiless_plan_args *a) { return ctx->N + (virt_sink(ctx, a) ? 1 : 0); }
 
 size_t smem_bound_bytes(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off) {
     const int rows = kernel_rows(ctx, a);
@@ -1476,7 +1481,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         const bool prune_mode = !(a->flags & SMILESS_FLAG_NO_PRUNE);
         const char *memo_env0 = getenv("SMILESS_MEMO");
         const bool memo_path = !prune_mode && a->n_fixed < ctx->N && (!memo_env0 || atoi(memo_env0) != 0) &&
-                               !inst_mode(ctx, a) &&
+                               !virt_sink(ctx, a) &&
                                smem_memo_up(ctx, rp, n_off) <= 227 * 1024 &&
                                smem_memo_var(ctx, a, rp, n_off) <= 227 * 1024;
         const bool bnb_path = !memo_path && bb_depth(ctx, a) > 0 && smem_bound_bytes(ctx, a, rp, n_off) <= 227 * 1024;
