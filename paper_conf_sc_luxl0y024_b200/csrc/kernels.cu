@@ -183,9 +183,9 @@ __global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParam
     const int nin = act ? p.inst[k] : 1;                // instances (request j on instance j mod nin)
     const int e0 = act ? p.pred_ptr[k] : 0, deg = act ? p.pred_ptr[k + 1] - e0 : 0;
     const bool sink = act && ((p.sinkmask >> k) & 1u);
-    int pc[4];                                            // first predecessors, in registers
+    int pc[8];                                            // first predecessors, in registers
 #pragma unroll
-    for (int e = 0; e < 4; ++e) pc[e] = e < deg ? p.pred_idx[e0 + e] : 0;
+    for (int e = 0; e < 8; ++e) pc[e] = e < deg ? p.pred_idx[e0 + e] : 0;
     int maxdeg = deg;
 #pragma unroll
     for (int m = 16; m > 0; m >>= 1) maxdeg = max(maxdeg, __shfl_xor_sync(FULL, maxdeg, m));
@@ -228,13 +228,13 @@ __global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParam
             i64 x = r;                                    // sources: the request's arrival
             const int sl = (int)(j & 31);
 #pragma unroll
-            for (int e = 0; e < 4; ++e) {                 // AND-join: max over predecessors
+            for (int e = 0; e < 8; ++e) {                 // AND-join: max over predecessors
                 if (e < deg) {
                     const i64 d = rg[pc[e]][sl];
                     x = e == 0 ? d : max(x, d);
                 }
             }
-            for (int e = 4; e < deg; ++e) x = max(x, rg[p.pred_idx[e0 + e]][sl]);
+            for (int e = 8; e < deg; ++e) x = max(x, rg[p.pred_idx[e0 + e]][sl]);
             // the case split of model M as selects (lanes of one warp take different cases;
             // straight-line code keeps them converged)
             // previous completion on this request's instance: D[k][j - nin] (own ring slot,
