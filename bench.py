@@ -270,7 +270,7 @@ def plan_kernel_ops_per_candidate(p) -> float:
     listed = set(int(v) for v in p.pred_idx)
     sinks = [k for k in range(n) if k not in listed]
     joins = sum(max(0, len(p.preds(k)) - 1) for k in range(n))
-    if p.instances is not None and max(p.instances) > 1:
+    if virtual_sink(p):
         upstream = 7 * n + joins + (len(sinks) - 1)       # + the virtual sink's join
         per_unit = 3 + 4                                   # one keep-alive variant
         share = 1
@@ -285,6 +285,12 @@ def plan_kernel_ops_per_candidate(p) -> float:
 
 
 SLICE_PINNED = {"C3": 4, "C5": 6, "C3s": 4, "C5s": 6}   # leading functions pinned (fastest, keep-alive)
+
+
+def virtual_sink(p) -> bool:
+    """Mirror of host.cpp virt_sink: a scaled-out LAST function makes the kernels append the
+    virtual sink (no sink sharing, no memoised path); scaled-out upstream functions do not."""
+    return p.instances is not None and int(p.instances[-1]) > 1
 
 
 def throughput_slice(name, S, dev, stream, local, steps=2, n_cand=1 << 24):
@@ -313,7 +319,7 @@ def throughput_slice(name, S, dev, stream, local, steps=2, n_cand=1 << 24):
     b.record(stream)
     torch.cuda.synchronize(dev)
     sec = a.elapsed_time(b) / 1e3
-    scale_out = p.instances is not None and max(p.instances) > 1
+    scale_out = virtual_sink(p)
     ops = (plan_kernel_ops_per_candidate(p) if scale_out else
            algorithmic_ops_per_candidate(p, memo=os.environ.get("SMILESS_MEMO", "1") != "0",
                                          split=os.environ.get("SMILESS_SPLITCOST", "1") != "0"))
@@ -321,7 +327,8 @@ def throughput_slice(name, S, dev, stream, local, steps=2, n_cand=1 << 24):
     return {"candidates_per_step": r.n_decided, "value": value, "unit": UNIT,
             "function_steps_per_s": value * p.n_funcs * (len(p.arrivals_us) - 1),
             "slice": f"first {n_cand} candidates, functions 0..{nf - 1} pinned to digits {fixed}",
-            "kernel": "smiless_plan_kernel (scale-out)" if scale_out else "memoised upstream + variants",
+            "kernel": ("smiless_plan_kernel (scaled-out last function: virtual sink)" if scale_out else
+                       "memoised upstream + variants" + (" (scale-out upstream rings)" if p.instances is not None else "")),
             "int_ops_per_candidate": ops, "achieved_int_ops_per_s": ops * r.n_decided / (kms / steps / 1e3),
             "instances": None if p.instances is None else p.instances.tolist(),
             "winner": {"index": r.index, "cost": r.cost} if r.feasible else None}
