@@ -34,6 +34,18 @@ plq.plan(q.arrivals_us, q.sla_us, q.windows_us, flags=S.FLAG_NO_PRUNE)
 w = W.random_problem(rng, 32, 2, 2, 100, max_preds=8, sla_us=5 * 10**8)
 S.planner_for(w).evaluate(rng.integers(0, w.space_size(), size=8, dtype=np.uint64), w.arrivals_us, w.sla_us,
                           w.windows_us)
+# round 2: scale-out rings + prologue (plan, bound, memo upstream, virtual sink, exact),
+# sharded B&B with split survivor lists, positive-time variants, the decomposition
+for inst in ([2, 1, 3, 1, 2], [1, 2, 1, 1, 3]):       # last function 1 (memo, sink sharing) / 3 (virtual sink)
+    plq.plan(q.arrivals_us, q.sla_us, q.windows_us, instances=inst)
+    plq.plan(q.arrivals_us, q.sla_us, q.windows_us, instances=inst, flags=S.FLAG_NO_PRUNE)
+    plq.evaluate(np.arange(32, dtype=np.uint64), q.arrivals_us, q.sla_us, q.windows_us, instances=inst)
+os.environ.update(SMILESS_BB_DEPTH="3", SMILESS_BB_DEPTH_A="1", SMILESS_BB_LISTCAP="3")
+for s_ in range(2):
+    plq.plan(q.arrivals_us, q.sla_us, q.windows_us, shard=s_, n_shards=2, instances=[2, 1, 3, 1, 2])
+for k in ("SMILESS_BB_DEPTH", "SMILESS_BB_DEPTH_A", "SMILESS_BB_LISTCAP"):
+    os.environ.pop(k)
+plq.decompose_plan(q.arrivals_us, q.sla_us, q.windows_us)
 print("sanitize workload done")
 PY
 for tool in memcheck racecheck synccheck initcheck; do
