@@ -213,7 +213,11 @@ __global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParam
     exact_fetch_block(ra, p.arr, J, 1, lane);
     asm volatile("cp.async.wait_group 0;" ::: "memory");
     __syncwarp();
-    for (i64 it = 0; it < J + nlev - 1; ++it) {
+    const i64 wT = w + T;                                 // per-lane constants of the case split
+    const bool keep = w == 0;                             // keep-alive (Case II)
+    const int n_it = (int)(J + nlev - 1);                 // J <= 2^31 (validated): 32-bit step counters
+    const int Ji = (int)J;
+    for (int it = 0; it < n_it; ++it) {
         if ((it & (EXACT_ARR_BLOCK - 1)) == 0) {
             // the previous fetch (block it / 128 + 1, read from the next block boundary on) has
             // landed once at most the newest group is pending; then fetch block it / 128 + 2
@@ -221,12 +225,12 @@ __global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParam
             __syncwarp();
             exact_fetch_block(ra, p.arr, J, it / EXACT_ARR_BLOCK + 2, lane);
         }
-        const i64 j = it - lvl;
-        const bool on = act && j >= 0 && j < J;
+        const int j = it - lvl;
+        const bool on = act && j >= 0 && j < Ji;
         const i64 r = on ? ra[j & (EXACT_ARR_RING - 1)] : 0;
         if (on) {
             i64 x = r;                                    // sources: the request's arrival
-            const int sl = (int)(j & 31);
+            const int sl = j & 31;
 #pragma unroll
             for (int e = 0; e < 8; ++e) {                 // AND-join: max over predecessors
                 if (e < deg) {
@@ -239,13 +243,13 @@ __global__ void __launch_bounds__(32 * EXACT_WARPS) eval_exact_kernel(ExactParam
             // straight-line code keeps them converged)
             // previous completion on this request's instance: D[k][j - nin] (own ring slot,
             // nin <= 16 < 32 so it is still there), or the register copy for one instance
-            const i64 f = nin == 1 ? D : rg[k][(j - nin) & 31], g = x - f, s = f + w;
+            const i64 f = nin == 1 ? D : rg[k][(j - nin) & 31], g = x - f;
+            // s = f + w: x < s <=> g < w, x < s + T <=> g < w + T (compared on g, no s formed)
             const bool busy = g <= 0;                     // busy: FIFO, stays warm (G6)
-            const bool keep = w == 0;                     // keep-alive (Case II)
-            const bool cold = x < s;                      // pre-warm not begun: cold (G3)
-            const bool part = x < s + T;                  // init partly covered (G4); else covered (Case I)
-            i64 start = busy ? f : keep ? x : cold ? x + T : part ? s + T : x;
-            i64 bill = busy ? 0 : keep ? g : (cold || part) ? T : x - s;
+            const bool cold = g < w;                      // pre-warm not begun: cold (G3)
+            const bool part = g < wT;                     // init partly covered (G4); else covered (Case I)
+            i64 start = busy ? f : keep ? x : cold ? x + T : part ? f + wT : x;
+            i64 bill = busy ? 0 : keep ? g : part ? T : g - w;
             if (j < nin) {                                // first invocation of an instance pre-warmed (G5)
                 start = x;
                 bill = T;
