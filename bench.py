@@ -346,6 +346,18 @@ def gap_fractions(p):
     return {"per_function_over_configs": per_fn, "gaps": int(len(gaps))}
 
 
+# The paper's own numbers (BASELINE.md sections 1-2), quoted as context: other hardware, other
+# quantities (its planner is a heuristic with a closed-form latency, no per-candidate walk)
+PAPER_CONTEXT = {
+    "hardware": "8-node cluster, 2x Intel Xeon Gold 5320 + 1x RTX 3090 per node, 10 GbE (PAPER.md:299)",
+    "top1_strategy_search": "< 20 ms for a DAG whose longest path has 12 functions (PAPER.md:367, Fig. 16a)",
+    "autoscaler_solve": "< 0.1 ms per function (PAPER.md:367, Fig. 16b)",
+    "cost_vs_icebreaker": "up to 5.73x lower cost with 0 SLA violations (PAPER.md:17, :305-311)",
+    "vs_opt": "OPT by exhaustive search; 'additional total cost of 50%' (PAPER.md:305, likely garbled)",
+    "default_sla": "2 s (PAPER.md:283)",
+}
+
+
 def measured_peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -696,6 +708,7 @@ def main():
         "time_to_optimal_full_space": full,
         "c4_sla_sweep_replanning": c4,
         "extra": extra,
+        "paper_context": PAPER_CONTEXT,
         "gpu_launches": launches,
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(res_e2e.h2d_bytes),
                 "d2h_bytes_per_step": int(res_e2e.d2h_bytes), "steps": steps_e2e,
