@@ -119,6 +119,8 @@ def test_plan_argument_validation_before_any_gpu_work():
         (dict(cost_cap=float("nan")), S.EINVAL),
         (dict(cost_cap=-1.0), S.EINVAL),
         (dict(cost_cap=1.0, flags=S.FLAG_NO_PRUNE), S.EINVAL),      # the cap is a prune-mode argument
+        (dict(instances=[1, 0, 1]), S.EINVAL),                      # scale-out: >= 1 instance
+        (dict(instances=[1, 17, 1]), S.EINVAL),                     # <= SMILESS_MAX_INSTANCES
     ]
     for over, code in cases:
         kw = dict(ok)
@@ -126,6 +128,15 @@ def test_plan_argument_validation_before_any_gpu_work():
         with pytest.raises(S.SmilessError) as e:
             pl.plan(**kw)
         assert e.value.code == code, over
+
+
+def test_negative_zero_price_rejected():
+    """-0.0 would give cost bits with the sign set: rejected like a negative price."""
+    pl = S.Planner(device=0)
+    pl.load_dag(*W.csr_from_preds([[], [0]]))
+    with pytest.raises(S.SmilessError) as e:
+        pl.load_profiles([1, 1], [10, 10], [5, 5], [1.0, -0.0])
+    assert e.value.code == S.EINVAL
 
 
 def test_space_size_and_erange():
