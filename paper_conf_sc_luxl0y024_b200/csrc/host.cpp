@@ -582,7 +582,14 @@ bool inst_mode(const smiless_ctx *ctx, const smiless_plan_args *a) { return inst
 // the virtual sink (DESIGN.md section 5 item 13) is needed only when the LAST function scales
 // out: otherwise its window variants keep sink sharing and the memoised throughput path, and
 // only the upstream functions carry instance rings
-bool virt_sink(const smiless_ctx *ctx, const smiless_plan_args *a) { return inst_of(a, ctx->N - 1) > 1; }
+// SMILESS_LRING=1: a scaled-out last function keeps its window variants with instance rings
+// (evaluator.cuh variants_step_ring: sink sharing and the memoised path stay) instead of the
+// virtual sink
+bool lring_on() {
+    const char *e = getenv("SMILESS_LRING");
+    return e && atoi(e) != 0;
+}
+bool virt_sink(const smiless_ctx *ctx, const smiless_plan_args *a) { return inst_of(a, ctx->N - 1) > 1 && !lring_on(); }
 // prologue steps j = 1 .. P of a scale-out plan (the first request of instances 2 .. n_k), a
 // multiple of 4 so that the main loop keeps its 16-byte aligned offset loads
 int inst_prologue(const smiless_ctx *ctx, const smiless_plan_args *a) {
@@ -774,6 +781,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_INST " << (inst_mode(ctx, a) ? 1 : 0) << "\n#define SM_VIRT " << (kd.virt ? 1 : 0)
       << "\n#define SM_PRO " << P << "\n#define SM_RG_ALLOC "
       << std::max(n_rg, 1) << "\n";
+    s << "#define SM_NL " << (kd.virt ? 1 : kd.inst[N - 1]) << "\n";   // instances of the variants' function
     s << "#define SM_NINST(k) (";
     for (int k = 0; k < N; ++k) s << "(k)==" << k << "?" << kd.inst[k] << ":";
     s << "1)\n";

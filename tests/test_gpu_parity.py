@@ -1022,8 +1022,11 @@ def test_every_int32_chunk_length_is_exact(K, monkeypatch):
 # NEXT-4 inside model M: scale-out instances (reading G26) on every kernel path
 # ---------------------------------------------------------------------------------------
 
-def test_scale_out_golden_on_the_gpu():
-    """Golden S_E7 (hand-worked) through smiless_evaluate and smiless_plan."""
+@pytest.mark.parametrize("lring", ["0", "1"])
+def test_scale_out_golden_on_the_gpu(lring, monkeypatch):
+    """Golden S_E7 (hand-worked) through smiless_evaluate and smiless_plan, with the
+    scaled-out last function as the virtual sink (lring 0) or as ring variants (lring 1)."""
+    monkeypatch.setenv("SMILESS_LRING", lring)
     import json, os
     g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "S_E7_scale_out.json")))
     for case in g["cases"]:
@@ -1039,12 +1042,15 @@ def test_scale_out_golden_on_the_gpu():
             assert r.index == 0 and r.cost == c[0] and r.max_latency_us == l[0]
 
 
+@pytest.mark.parametrize("lring", ["0", "1"])
 @pytest.mark.parametrize("flags", [0, S.FLAG_NO_PRUNE, S.FLAG_FORCE_INT64, S.FLAG_NO_PRUNE | S.FLAG_FORCE_INT64])
-def test_scale_out_random_dags_per_candidate_costs(flags):
+def test_scale_out_random_dags_per_candidate_costs(flags, lring, monkeypatch):
     """Random DAGs with 1-4 round-robin instances per function (rings, prologue, virtual
     sink, scale-out billing): every candidate's cost bits and feasibility equal the oracle's,
     the winner is the oracle's OPT, and smiless_evaluate (the independent exact kernel)
-    agrees too."""
+    agrees too.  lring: a scaled-out last function as ring variants instead of the virtual
+    sink (SMILESS_LRING)."""
+    monkeypatch.setenv("SMILESS_LRING", lring)
     rng = np.random.default_rng(400 + flags)
     n_checked = 0
     for t in range(80):
@@ -1070,9 +1076,11 @@ def test_scale_out_random_dags_per_candidate_costs(flags):
     assert n_checked >= 15
 
 
-def test_scale_out_branch_and_bound_and_shards(monkeypatch):
+@pytest.mark.parametrize("lring", ["0", "1"])
+def test_scale_out_branch_and_bound_and_shards(lring, monkeypatch):
     """B&B depths with scale-out functions (lower-bound relaxation downstream of them),
     2 shards, and the cost bound: per-candidate parity and the oracle's OPT."""
+    monkeypatch.setenv("SMILESS_LRING", lring)
     rng = np.random.default_rng(77)
     n_checked = 0
     for t in range(40):
@@ -1110,11 +1118,13 @@ def test_scale_out_branch_and_bound_and_shards(monkeypatch):
     assert n_checked >= 5
 
 
+@pytest.mark.parametrize("lring", ["0", "1"])
 @pytest.mark.parametrize("K", ["64", "16", "8"])
-def test_scale_out_chunk_lengths(K, monkeypatch):
+def test_scale_out_chunk_lengths(K, lring, monkeypatch):
     """The prologue must sit inside chunk 0 (K >= prologue) and the rings span chunk
     rebases: forced K with up to 8 instances (prologue 8) against the oracle."""
     monkeypatch.setenv("SMILESS_FORCE_K", K)
+    monkeypatch.setenv("SMILESS_LRING", lring)
     rng = np.random.default_rng(500 + int(K))
     for t in range(30):
         n = int(rng.integers(1, 5))
