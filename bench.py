@@ -288,10 +288,11 @@ SLICE_PINNED = {"C3": 4, "C5": 6, "C3s": 4, "C5s": 6}   # leading functions pinn
 
 
 def virtual_sink(p) -> bool:
-    """Mirror of host.cpp virt_sink: a scaled-out LAST function makes the kernels append the
-    virtual sink (no sink sharing, no memoised path); scaled-out upstream functions do not."""
+    """Mirror of host.cpp virt_sink: with SMILESS_LRING=0 a scaled-out LAST function makes the
+    kernels append the virtual sink (no sink sharing, no memoised path); by default its window
+    variants carry instance rings instead."""
     return (p.instances is not None and int(p.instances[-1]) > 1 and
-            os.environ.get("SMILESS_LRING", "0") == "0")
+            os.environ.get("SMILESS_LRING", "1") == "0")
 
 
 def throughput_slice(name, S, dev, stream, local, steps=2, n_cand=1 << 24):

@@ -180,7 +180,7 @@ def test_nvrtc_specialises_every_config_for_sm100a(name):
     # scale-out plans (C3 / C5) carry instance rings; a scaled-out LAST function (C5) adds the
     # virtual sink to the kernel DAG (DESIGN §5 item 13)
     scale_out = p.instances is not None and max(p.instances) > 1
-    virt = p.instances is not None and p.instances[-1] > 1
+    virt = False        # the default keeps a scaled-out last function's variants (ring form)
     assert "#define SM_N %d" % (p.n_funcs + virt) in src and "smiless_plan_kernel" in src
     assert ("#define SM_INST %d" % scale_out) in src and ("#define SM_VIRT %d" % virt) in src
 
