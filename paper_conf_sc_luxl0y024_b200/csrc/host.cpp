@@ -1408,6 +1408,12 @@ struct HostProf {
     HostProf() : on(getenv("SMILESS_PROFILE_HOST") != nullptr) {
         if (on) t0 = last = std::chrono::steady_clock::now();
     }
+    void note(const char *what, unsigned long long v) {
+        if (!on) return;
+        char b[96];
+        snprintf(b, sizeof b, " %s=%llu", what, v);
+        line += b;
+    }
     void mark(const char *what) {
         if (!on) return;
         const auto now = std::chrono::steady_clock::now();
@@ -1762,6 +1768,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                     ctx->d2h += sizeof n_a;
                     CK(cudaStreamSynchronize(st), "count");
                     hp.mark("sync_a");
+                    hp.note("n_a", n_a);
                     // deep launches (first survivor entry, entries, first child, children per entry):
                     // at most list_cap ordinals each.  With the cost bound on, the first launch is small:
                     // its evaluation sets the incumbent the static prefix bound of every later launch
