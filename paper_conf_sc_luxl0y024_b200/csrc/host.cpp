@@ -233,6 +233,7 @@ struct BoundParamsHost {
     unsigned *overflow;            // set to 1 if a launch would exceed list_cap (never, by sizing)
     int shard, n_shards;           // ordinals c = c' * n_shards + shard of the launch
     int attr_shard, attr_n;        // replicated level: decided counted for c % attr_n == attr_shard
+    u64 *list_key;                 // optional static cost lower bound per survivor (best-first order)
     int fixed[SMILESS_MAX_FUNCS];
 };
 
@@ -341,7 +342,7 @@ struct smiless_ctx {
     DevBuf<i64> dLat;
     DevBuf<unsigned char> dFeas;
     DevBuf<double> dDump;
-    DevBuf<u64> dList, dListA, dCostList;
+    DevBuf<u64> dList, dListA, dCostList, dListKeyA;
     DevBuf<unsigned> dCostN;
     DevBuf<unsigned> dListCnt, dListCntA, dChunkCnt;
     DevBuf<int> dW;                          // per-row windows of the current plan (padded)
@@ -1222,7 +1223,7 @@ void smiless_destroy(smiless_ctx *ctx) {
         ctx->dCounter.release(); ctx->dStats.release(); ctx->dInc.release(); ctx->dBlk.release(); ctx->dIdxEval.release();
         ctx->dCost.release(); ctx->dLat.release(); ctx->dFeas.release(); ctx->dRes.release(); ctx->dDump.release();
         ctx->dList.release(); ctx->dListCnt.release(); ctx->dW.release();
-        ctx->dListA.release(); ctx->dListCntA.release(); ctx->dChunkCnt.release();
+        ctx->dListA.release(); ctx->dListCntA.release(); ctx->dChunkCnt.release(); ctx->dListKeyA.release();
         ctx->dCostList.release(); ctx->dCostN.release();
         ctx->dX.release(); ctx->dRecNx.release(); ctx->dRecNlu.release(); ctx->dRecPre.release();
         if (ctx->hRes) cudaFreeHost(ctx->hRes);
@@ -1739,6 +1740,14 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 const u64 a_lo = cb / SA, a_hi = (ce + SA - 1) / SA;
                 CK(ctx->dListA.ensure((size_t)batch), "cudaMalloc list");
                 CK(ctx->dListCntA.ensure(1), "cudaMalloc");
+                // best-first: with the cost bound on, the shallow survivors are sorted by their
+                // static cost lower bound so the first deep launch sets a good incumbent early
+                // (SMILESS_BB_SORT=0: atomic append order)
+                const char *sort_env = getenv("SMILESS_BB_SORT");
+                const bool bb_sort = pp.cost_prune && (!sort_env || atoi(sort_env) != 0);
+                if (bb_sort) CK(ctx->dListKeyA.ensure((size_t)batch), "cudaMalloc keys");
+                std::vector<u64> h_pref, h_key;
+                std::vector<uint32_t> h_ord;
                 for (u64 b0 = a_lo; b0 < a_hi; b0 += batch) {
                     const u64 b1 = std::min(a_hi, b0 + batch);
                     CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
@@ -1758,6 +1767,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                     bp.n_shards = 1;
                     bp.attr_shard = shard;                        // ... its pruned prefixes counted once
                     bp.attr_n = n_shards;
+                    bp.list_key = bb_sort ? ctx->dListKeyA.p : nullptr;
                     {
                         NvtxRange nv("bnb shallow level");
                         if ((rc = run_bound(jk->fn_bound_a))) return rc;
@@ -1769,6 +1779,29 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                     CK(cudaStreamSynchronize(st), "count");
                     hp.mark("sync_a");
                     hp.note("n_a", n_a);
+                    bp.list_key = nullptr;
+                    if (bb_sort && n_a > 1 && n_a <= (1u << 18)) {
+                        // (key, prefix) ascending; ties by prefix: a deterministic order on every rank
+                        h_pref.resize(n_a);
+                        h_key.resize(n_a);
+                        CK(cudaMemcpyAsync(h_pref.data(), ctx->dListA.p, n_a * sizeof(u64), cudaMemcpyDeviceToHost, st),
+                           "D2H survivors");
+                        CK(cudaMemcpyAsync(h_key.data(), ctx->dListKeyA.p, n_a * sizeof(u64), cudaMemcpyDeviceToHost, st),
+                           "D2H keys");
+                        CK(cudaStreamSynchronize(st), "survivors");
+                        h_ord.resize(n_a);
+                        for (uint32_t q = 0; q < n_a; ++q) h_ord[q] = q;
+                        std::sort(h_ord.begin(), h_ord.end(), [&](uint32_t x, uint32_t y) {
+                            return h_key[x] != h_key[y] ? h_key[x] < h_key[y] : h_pref[x] < h_pref[y];
+                        });
+                        std::vector<u64> sorted(n_a);
+                        for (uint32_t q = 0; q < n_a; ++q) sorted[q] = h_pref[h_ord[q]];
+                        CK(cudaMemcpyAsync(ctx->dListA.p, sorted.data(), n_a * sizeof(u64), cudaMemcpyHostToDevice, st),
+                           "H2D survivors");
+                        ctx->d2h += 2 * (u64)n_a * sizeof(u64);
+                        ctx->h2d += (u64)n_a * sizeof(u64);
+                        hp.mark("sort_a");
+                    }
                     // deep launches (first survivor entry, entries, first child, children per entry):
                     // at most list_cap ordinals each.  With the cost bound on, the first launch is small:
                     // its evaluation sets the incumbent the static prefix bound of every later launch
