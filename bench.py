@@ -9,11 +9,13 @@ Step (BASELINE.json metric, configs[1]): one smiless_plan call = the whole hot p
 re-evaluation of the winner) over the fixed 2^28-candidate slice of C2 (IPA-6 DAG,
 16 configs x 8 windows, 10^4 Poisson arrivals; functions 0 and 1 pinned to
 GPU-100% / keep-alive), in throughput mode (no pruning: every candidate walked through
-all 10^4 arrivals).  N GPUs split that fixed slice (strong scaling: time-to-optimal
-of the slice); each rank plans its interleaved chunks and the ranks exchange the
-winner with NCCL MIN all-reduces.
+all 10^4 arrivals).  Weak scaling (the candidate space partitions, so per-GPU work is
+fixed): rank r plans its own 2^28-candidate slice, function 1 pinned to config 15 - r
+(rank 0 = the single-GPU slice), and the ranks exchange the winner of the union with
+NCCL MIN all-reduces (16 bytes; no data-path collective).  SMILESS_BENCH_SCALING=strong
+splits the one rank-0 slice over the ranks instead.
 
-`value` = candidates of the slice / max-over-ranks device time per step (inputs resident
+`value` = candidates of all ranks' slices / max-over-ranks device time per step (inputs resident
 in HBM: arrivals passed as a device tensor).  `e2e` = the same through the public API
 with the arrivals in pinned host memory (H2D inside the timed region) and the result
 read back to the host.  Only rank 0 at N=1 times the CPU oracle (cpu_baseline) on a
@@ -42,13 +44,16 @@ UNIT = "candidates/s"
 ISSUE_LANES_PER_CLK_PER_SM = 4 * 32      # 4 SMSPs x 1 warp-instruction/clk x 32 lanes
 
 
-def workload(name: str = "C2"):
-    """(Problem, plan kwargs) of the timed step.  Shared with tests/test_gpu_parity.py."""
+def workload(name: str = "C2", rank: int = 0):
+    """(Problem, plan kwargs) of the timed step.  Shared with tests/test_gpu_parity.py.
+    rank r > 0 (weak scaling): function 1 pinned to config 15 - r instead of 15."""
     if name == "C2":
         p = W.make_config("C2")
         Wn = len(p.windows_us)
         gpu100 = 15                        # CONFIG_GRIDS[16][15] = ("gpu", 1.0)
-        fixed = [gpu100 * Wn + 0, gpu100 * Wn + 0]   # SR, IR on GPU-100%, keep-alive
+        if not 0 <= rank < 16:
+            raise ValueError("weak-scaling slices exist for ranks 0..15")
+        fixed = [gpu100 * Wn + 0, (gpu100 - rank) * Wn + 0]   # SR, IR on GPU configs, keep-alive
         return p, dict(n_fixed=2, fixed_digits=fixed)
     if name == "C1":
         return W.make_config("C1"), dict(n_fixed=0, fixed_digits=[])
@@ -440,6 +445,7 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
+    weak = os.environ.get("SMILESS_BENCH_SCALING", "weak") != "strong" and args.workload == "C2"
     p, kw = workload(args.workload)
     from oracle import OracleProblem
     threads = os.cpu_count() or 1
@@ -461,8 +467,8 @@ def run_reference(args):
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
-        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "i64+f64",
-        "data": "synthetic", "config": config_block(p, kw, args),
+        "higher_is_better": True, "scaling": "weak" if weak else "strong", "vs_baseline": None,
+        "dtype": "i64+f64", "data": "synthetic", "config": config_block(p, kw, args, weak),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
                          "sample": f"{n_step} consecutive candidates of the slice per step",
                          "cpu_model": host_cpu()["model"], "cpu_mhz": host_cpu()["mhz"]},
@@ -472,19 +478,23 @@ def run_reference(args):
     return 0
 
 
-def config_block(p, kw, args):
+def config_block(p, kw, args, weak=False):
     space = 1
     for k in range(kw["n_fixed"], p.n_funcs):
         space *= int(p.n_configs[k]) * len(p.windows_us)
+    n_slices = args.gpus if weak else 1
+    per_rank = (f"; rank r plans the slice with function 1 on config 15 - r (digit {kw['fixed_digits'][1]} - 8r)"
+                if weak and args.gpus > 1 else "")
     return {
         "workload": f"{p.name}: {p.n_funcs}-function DAG, {int(p.n_configs[0])} configs x {len(p.windows_us)} "
                     f"windows, J={len(p.arrivals_us)} arrivals, SLA {p.sla_us} us; slice of {space} candidates "
-                    f"(functions 0..{kw['n_fixed'] - 1} pinned to digits {list(kw['fixed_digits'])}); "
+                    f"(functions 0..{kw['n_fixed'] - 1} pinned to digits {list(kw['fixed_digits'])}){per_rank}; "
                     f"throughput mode (no pruning)",
-        "candidates_per_step": space,
+        "candidates_per_step": space * n_slices,
         "arrivals": len(p.arrivals_us),
         "l2": "256 MiB buffer written between timed steps (L2 flushed); working set < 1 MB",
-        "parallelism": f"candidate-space sharding x{args.gpus}",
+        "parallelism": (f"weak scaling: one {space}-candidate slice per rank x{args.gpus}" if weak
+                        else f"candidate-space sharding x{args.gpus}"),
     }
 
 
@@ -528,18 +538,27 @@ def main():
         else:
             dist.init_process_group("nccl", device_id=dev)
 
-    p, kw = workload(args.workload)
+    weak = os.environ.get("SMILESS_BENCH_SCALING", "weak") != "strong" and args.workload == "C2"
+    p, kw = workload(args.workload, rank if weak else 0)
     stream = torch.cuda.current_stream(dev)
     pl = S.planner_for(p, device=local, stream=stream.cuda_stream)
     arr_dev = torch.as_tensor(p.arrivals_us).to(dev)                 # HBM-resident inputs
     arr_pin = torch.as_tensor(p.arrivals_us).pin_memory()            # e2e: pinned host inputs
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
-    plan_kw = dict(kw, flags=S.FLAG_NO_PRUNE, shard=rank, n_shards=world)
+    # weak: every rank its own slice (no sharding inside); strong: the rank-0 slice split
+    shard_kw = dict(shard=0, n_shards=1) if weak else dict(shard=rank, n_shards=world)
+    plan_kw = dict(kw, flags=S.FLAG_NO_PRUNE, **shard_kw)
+    slice_size = pl.space_size(len(p.windows_us), kw["n_fixed"])
+
+    def union_index(r):
+        # index in the function-0-pinned space (function 1's digit is the rank's slice), so
+        # the lowest-index tie-break is the same for every world size
+        return None if not r.feasible else (kw["fixed_digits"][1] * slice_size + r.index if weak else r.index)
 
     def step(arrivals):
         r = pl.plan(arrivals, p.sla_us, p.windows_us, **plan_kw)
         if world > 1:
-            reduce_best(r.cost if r.feasible else None, r.index, r.max_latency_us, r.n_decided, xdev)
+            reduce_best(r.cost if r.feasible else None, union_index(r), r.max_latency_us, r.n_decided, xdev)
         return r
 
     def barrier():
@@ -605,7 +624,7 @@ def main():
     # pruned (exact plan with early exit): time-to-optimal of the same slice
     pruned = None
     if not args.no_pruned:
-        kwp = dict(kw, flags=0, shard=rank, n_shards=world)
+        kwp = dict(kw, flags=0, **shard_kw)
         pl.plan(arr_dev, p.sla_us, p.windows_us, **kwp)          # NVRTC compile of the prune-mode kernels
         barrier()
         a = torch.cuda.Event(enable_timing=True)
@@ -613,7 +632,7 @@ def main():
         a.record(stream)
         rp = pl.plan(arr_dev, p.sla_us, p.windows_us, **kwp)
         if world > 1:
-            reduce_best(rp.cost if rp.feasible else None, rp.index, rp.max_latency_us, rp.n_decided, xdev)
+            reduce_best(rp.cost if rp.feasible else None, union_index(rp), rp.max_latency_us, rp.n_decided, xdev)
         b.record(stream)
         torch.cuda.synchronize(dev)
         pruned = {"time_to_optimal_ms": a.elapsed_time(b), "index": rp.index, "cost": rp.cost,
@@ -701,8 +720,8 @@ def main():
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
-        "scaling": "strong", "vs_baseline": None, "dtype": "i32+f64", "data": "synthetic",
-        "config": config_block(p, kw, args),
+        "scaling": "weak" if weak else "strong", "vs_baseline": None, "dtype": "i32+f64", "data": "synthetic",
+        "config": config_block(p, kw, args, weak),
         "time_to_optimal_ms": ms / args.steps,
         "winner": {"index": res.index, "cost": res.cost, "max_latency_us": res.max_latency_us,
                    "config": res.config.tolist(), "window": res.window.tolist()} if world == 1 else None,

@@ -167,7 +167,7 @@ struct PlanParamsHost {
     const i64 *rrem;               // [chunks] r_{J-1} - r_{(q+1)K}
     u64 cap;                       // cost cap bits (~0: none)
     int cost_prune;
-    int pad0;
+    int no_count;                  // 1: the units were counted by an earlier pass
     u64 list_in_cap;               // list mode: entries list_in holds (clamps *list_n)
     int fixed[SMILESS_MAX_FUNCS];  // evaluator uses SM_NFIXED_ALLOC <= SMILESS_MAX_FUNCS; extra tail is ignored
 };
@@ -197,6 +197,7 @@ struct MemoParamsHost {
     int slas[8];
     u64 *cost_list;                // split cost: units holding a feasible candidate
     unsigned *cost_n;
+    int shard, n_shards;           // fused kernel: tile c belongs to shard c % n_shards
     int fixed[SMILESS_MAX_FUNCS];
 };
 
@@ -277,8 +278,9 @@ struct JitKernel {
     CUmodule mod = nullptr;
     CUfunction fn = nullptr;
     CUfunction fn_bound = nullptr, fn_bound_a = nullptr, fn_up = nullptr, fn_var = nullptr, fn_varc = nullptr;
-    size_t smem_up = 0, smem_var = 0;
-    int blocks_up = 0, blocks_var = 0;
+    CUfunction fn_fused = nullptr;
+    size_t smem_up = 0, smem_var = 0, smem_fused = 0;
+    int blocks_up = 0, blocks_var = 0, blocks_fused = 0;
     size_t smem = 0, smem_bound = 0;
     int blocks_per_sm = 0, blocks_bound = 0;
     int regs = 0;
@@ -725,6 +727,30 @@ bool split_cost() {
     return !e || atoi(e) != 0;
 }
 
+// Fused memoisation (evaluator.cuh smiless_fused_kernel): one persistent kernel whose producer
+// warp walks the upstream functions of a tile of prefixes into a shared-memory ring that its
+// consumer warps read, so the x stream never leaves the SM.  Needs the int32 path, a last
+// function that is not scaled out, and a tile of 1..32 prefixes.  SMILESS_FUSED=0: two kernels.
+constexpr int kFusedSlots = 4, kFusedSteps = 64;   // mirror SM_FSLOTS, SM_FPS
+int fused_tile(const smiless_ctx *ctx, const smiless_plan_args *a) {
+    return (vthreads_per_cta() / 32 - 1) * 32 / (ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
+}
+bool fused_on(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp) {
+    const char *e = getenv("SMILESS_FUSED");
+    if (!e || atoi(e) == 0) return false;      // off unless SMILESS_FUSED=1 (until measured)
+    if (rp.time64 || inst_of(a, ctx->N - 1) > 1) return false;
+    const int tp = fused_tile(ctx, a);
+    return tp >= 1 && tp <= 32;
+}
+size_t smem_fused(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off) {
+    const size_t padI = (size_t)((ctx->sumM + 3) & ~3), padU = (size_t)((ctx->sumM + 1) & ~1);
+    const size_t fc32 = (size_t)(vthreads_per_cta() / 32 - 1) * 32;
+    (void)rp;
+    return 3 * padI * 4 + padU * 8 + 4 * (size_t)n_off + (split_cost() ? 0 : 8 * (size_t)unit_cands(ctx, a) * fc32) +
+           4 * (size_t)kFusedSlots * kFusedSteps * (size_t)fused_tile(ctx, a) +
+           ((4 * (size_t)ctx->N * kThreads + 15) & ~(size_t)15);
+}
+
 // static cost-bound terms of every (row, window) staged in shared memory when small
 bool bound_lb_table(const smiless_ctx *ctx, int W) { return (size_t)ctx->sumM * (size_t)W <= 8192; }
 
@@ -772,6 +798,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_LBT " << (bound_lb_table(ctx, W) ? 1 : 0) << "\n";
     s << "#define SM_XPF " << xpf_groups() << "\n";
     s << "#define SM_SPLITCOST " << (split_cost() ? 1 : 0) << "\n";
+    s << "#define SM_FUSED " << (((families & FAM_MEMO) && fused_on(ctx, a, rp)) ? 1 : 0) << "\n";
     // window variants of the memoised kernel walked in the positive-time form (evaluator.cuh
     // variants_step FM: ALU busy mask + full-rate IMAD instead of the quarter-rate IMAD.HI)
     // default: every window variant (measured: 3.45e8 -> 3.81e8 candidates/s on the C2 slice,
@@ -1105,6 +1132,17 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(upstream)");
                 r = driver().occupancy(&jk.blocks_var, jk.fn_var, vthreads_per_cta(), jk.smem_var);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(variants)");
+            }
+            jk.smem_fused = smem_fused(ctx, a, rp, n_off);
+            if (fused_on(ctx, a, rp) && jk.smem_fused <= 227 * 1024) {
+                r = driver().moduleGetFunction(&jk.fn_fused, jk.mod, "smiless_fused_kernel");
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(fused)");
+                r = driver().funcSetAttribute(jk.fn_fused, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
+                                              (int)jk.smem_fused);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(fused smem)");
+                r = driver().occupancy(&jk.blocks_fused, jk.fn_fused, vthreads_per_cta(), jk.smem_fused);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(fused)");
+                if (jk.blocks_fused < 1) jk.fn_fused = nullptr;
             }
         }
         if (families & FAM_BOUND) {
@@ -1569,14 +1607,100 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         const int D = bb_depth(ctx, a);
         pp.list_upp = 1;
         const bool memo = memo_path && jk->blocks_up > 0 && jk->blocks_var > 0;
-        if (memo) {
+        if (memo && jk->fn_fused) {
+            // ---- fused memoisation: upstream walked by each CTA's producer warp into a shared-
+            // memory ring, variants by its consumer warps (evaluator.cuh smiless_fused_kernel);
+            // split cost: the units holding a feasible candidate are re-walked by the plan
+            // kernel in list mode (upstream recomputed per lane, sums of u, cost, argmin)
+            const u64 upp = (u64)(ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
+            const u64 pl0 = ub / upp, ph0 = (ue + upp - 1) / upp;
+            const bool split = split_cost();
+            // prefix batches bound the cost list; tiles of a batch are interleaved over the shards
+            const u64 batch_p = std::min<u64>((u64)1 << 20, ph0 - pl0);
+            if (split) {
+                CK(ctx->dCostList.ensure((size_t)(batch_p * upp)), "cudaMalloc cost list");
+                CK(ctx->dCostN.ensure(1), "cudaMalloc");
+            }
+            MemoParamsHost mp;
+            memset(&mp, 0, sizeof mp);
+            mp.tabNI = ctx->dNI.p;
+            mp.tabT = ctx->dT.p;
+            mp.tabW = ctx->dW.p;
+            mp.tabU = ctx->dU.p;
+            mp.off = ctx->dOff.p;
+            mp.scal = ctx->dScal.p;
+            mp.counter = ctx->dCounter.p;
+            mp.stats = ctx->dStats.p;
+            mp.cost_list = ctx->dCostList.p;
+            mp.cost_n = ctx->dCostN.p;
+            mp.dump = pp.dump;
+            mp.cand_begin = cb;
+            mp.cand_end = ce;
+            mp.n_steps = n_steps;
+            mp.n_off = n_off;
+            mp.sumM = ctx->sumM;
+            mp.sla = (int)a->sla_us;
+            mp.zero = 0;
+            mp.shard = shard;
+            mp.n_shards = n_shards;
+            for (int s_ = 0; s_ < n_sla; ++s_) mp.slas[s_] = (int)slas[s_];
+            for (int k = 0; k < a->n_fixed; ++k) mp.fixed[k] = a->fixed_digits[k];
+            const int grid_f = jk->blocks_fused * ctx->n_sms;
+            if (grid_f > grid) {     // per-CTA argmin slots of the fused kernel
+                CK(ctx->dBlk.ensure((size_t)grid_f * 2 * n_sla), "cudaMalloc");
+                CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid_f * 16 * n_sla, st), "memset");
+                pp.blk_best = ctx->dBlk.p;
+            }
+            mp.blk_best = ctx->dBlk.p;
+            // the cost re-walk: plan kernel, list mode over the fused pass's cost list
+            PlanParamsHost pc = pp;
+            pc.prune = 0;
+            pc.cost_prune = 0;
+            pc.cap = ~0ull;
+            pc.horizon = 0;
+            pc.claims_begin = 0;
+            pc.claims_end = ~0ull;
+            pc.list_in = ctx->dCostList.p;
+            pc.list_n = ctx->dCostN.p;
+            pc.list_upp = 1;
+            pc.list_base = 0;
+            pc.list_in_cap = batch_p * upp;
+            pc.no_count = 1;
+            CK(cudaEventRecord(ctx->ev[1], st), "event");
+            NvtxRange nv("memo: fused producer/consumer batches");
+            for (u64 b0 = pl0; b0 < ph0; b0 += batch_p) {
+                const u64 b1 = std::min(ph0, b0 + batch_p);
+                mp.pref_begin = b0;
+                mp.pref_end = b1;
+                mp.unit_begin = std::max(ub, b0 * upp);
+                mp.unit_end = std::min(ue, b1 * upp);
+                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                if (split) CK(cudaMemsetAsync(ctx->dCostN.p, 0, sizeof(unsigned), st), "memset cost list");
+                void *args[] = {&mp};
+                CUresult r = driver().launchKernel(jk->fn_fused, (unsigned)grid_f, 1, 1, vthreads_per_cta(), 1, 1,
+                                                   (unsigned)jk->smem_fused, (CUstream)st, args, nullptr);
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "fused launch");
+                ++launches;
+                if (split) {
+                    CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                    void *cargs[] = {&pc};
+                    r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
+                                              (CUstream)st, cargs, nullptr);
+                    if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "fused cost re-walk launch");
+                    ++launches;
+                }
+            }
+            grid_used = std::max(grid, grid_f);
+        } else if (memo) {
             // ---- prefix memoisation: upstream once per prefix, then the variants per unit ---------
             const u64 upp = (u64)(ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
             const u64 pl0 = ub / upp, ph0 = (ue + upp - 1) / upp;
             const size_t tsz2 = rp.time64 ? 8 : 4;
             // + SM_XPF + 1 groups of 4 steps of read-ahead slack for the variants kernel
             const size_t row_bytes = tsz2 * (size_t)(n_off + 4 * (xpf_groups() + 1));
-            const u64 max_batch = std::max<u64>(1, std::min<u64>((u64)1 << 16, ((u64)4 << 30) / row_bytes));
+            u64 max_batch = std::max<u64>(1, std::min<u64>((u64)1 << 16, ((u64)4 << 30) / row_bytes));
+            if (const char *mb_env = getenv("SMILESS_MEMO_BATCH"))   // tuning: prefixes per batch (<= 64 GB buffer)
+                max_batch = std::max<u64>(1, std::min<u64>((u64)atoll(mb_env), ((u64)64 << 30) / row_bytes));
             const u64 batch_p = std::min<u64>(max_batch, ph0 - pl0);
             CK(ctx->dX.ensure((size_t)batch_p * row_bytes), "cudaMalloc memo buffer");
             CK(ctx->dRecNx.ensure((size_t)batch_p), "cudaMalloc");

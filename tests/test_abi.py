@@ -185,6 +185,28 @@ def test_nvrtc_specialises_every_config_for_sm100a(name):
     assert ("#define SM_INST %d" % scale_out) in src and ("#define SM_VIRT %d" % virt) in src
 
 
+def test_fused_memo_kernel_compiles_for_the_bench_slice(monkeypatch):
+    """The bench slice (C2, throughput mode) selects the fused producer/consumer kernel
+    (SMILESS_FUSED=0 the two-kernel path); it compiles for sm_100a with no local memory and
+    its consumer loop reads x from shared memory, not global memory."""
+    import bench
+    p, kw = bench.workload("C2")
+    pl = S.planner_for(p)
+    args = (p.arrivals_us, p.sla_us, p.windows_us)
+    monkeypatch.setenv("SMILESS_FUSED", "0")
+    assert "#define SM_FUSED 0" in pl.kernel_source(*args, flags=S.FLAG_NO_PRUNE, **kw)
+    monkeypatch.setenv("SMILESS_FUSED", "1")
+    assert "#define SM_FUSED 1" in pl.kernel_source(*args, flags=S.FLAG_NO_PRUNE, **kw)
+    log, n = pl.jit_compile(*args, flags=S.FLAG_NO_PRUNE, **kw)
+    entry = log.split("Compiling entry function 'smiless_fused_kernel'")[1].split("Compiling entry")[0]
+    assert "0 bytes stack frame, 0 bytes spill stores, 0 bytes spill loads" in entry, entry
+    import sys
+    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tools"))
+    import sass_mix
+    body, _ = sass_mix.loop_body("smiless_fused_kernel")
+    assert any(t.startswith("LDS.128") for t in body) and not any(t.startswith("LDG") for t in body)
+
+
 def test_int64_path_selected_when_int32_range_fails():
     p = W.make_config("C1", n_arrivals=20)
     p = p.replace(windows_us=np.array([0, (1 << 29) - 1], np.int32), init_us=np.full_like(p.init_us, (1 << 29) - 1))

@@ -711,6 +711,65 @@ def test_memo_variants_shapes_are_exact(g, split, fmask, monkeypatch):
     assert n_checked > 10
 
 
+@pytest.mark.parametrize("g,split", [("1", "1"), ("1", "0"), ("2", "1"), ("2", "0")])
+def test_fused_memo_kernel_is_exact(g, split, monkeypatch):
+    """The fused memoisation kernel (producer warp -> shared-memory ring of x -> consumer
+    warps; split cost re-walked by the plan kernel in list mode) on random DAGs whose last
+    function has >= 7 config groups: per-candidate parity with the oracle over ragged ranges
+    (partial tiles), several ring slots and a one-step tail, and every candidate counted once."""
+    monkeypatch.setenv("SMILESS_MEMO", "1")
+    monkeypatch.setenv("SMILESS_FUSED", "1")
+    monkeypatch.setenv("SMILESS_SPLITCOST", split)
+    monkeypatch.setenv("SMILESS_G", g)
+    rng = np.random.default_rng(211 + 10 * int(g) + int(split))
+    n_checked = 0
+    for t in range(120):
+        n = int(rng.integers(2, 5))
+        p = W.random_problem(rng, n, 16, int(rng.integers(1, 4)), int(rng.choice([2, 5, 64, 65, 130, 257, 400])))
+        space = p.space_size()
+        if space > 40000 or int(p.n_configs[-1]) // int(g) < 7 or int(p.n_configs[-1]) % int(g):
+            continue
+        pl = S.planner_for(p)
+        flags = S.FLAG_NO_PRUNE
+        assert "#define SM_FUSED 1" in pl.kernel_source(p.arrivals_us, p.sla_us, p.windows_us, flags=flags)
+        b = int(rng.integers(0, space // 4 + 1))
+        out = np.empty(space - b)
+        r = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=flags, begin=b, cost_out=out)
+        o = OracleProblem(p)
+        oc, ol, of = o.evaluate(np.arange(b, space, dtype=np.uint64))
+        assert_dump_matches(out, oc, of)
+        assert_same_plan(r, o.plan(begin=b), o)
+        assert r.n_full_evals == r.n_decided == space - b
+        n_checked += 1
+        if n_checked >= 12:
+            break
+    assert n_checked >= 6
+
+
+def test_fused_memo_kernel_shards_and_matches_two_kernel_path(monkeypatch):
+    """Fused vs two-kernel memoisation on the bench slice of C2 at J = 10^4 (2^28 candidates
+    is too long here: a 2^22-candidate range around the winner), bit-identical winner; and the
+    fused kernel's tiles interleaved over 3 shards decide the range exactly once."""
+    import bench
+    p, kw = bench.workload("C2")
+    pl = S.planner_for(p)
+    full = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, flags=S.FLAG_NO_PRUNE, **kw)
+    lo = full.index - full.index % (1 << 22) if full.feasible else 0
+    rng_kw = dict(kw, begin=lo + 77, end=lo + (1 << 22) - 5, flags=S.FLAG_NO_PRUNE)
+    monkeypatch.setenv("SMILESS_FUSED", "0")
+    two = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, **rng_kw)
+    monkeypatch.setenv("SMILESS_FUSED", "1")
+    assert "#define SM_FUSED 1" in pl.kernel_source(p.arrivals_us, p.sla_us, p.windows_us, **rng_kw)
+    one = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, **rng_kw)
+    assert (one.index, one.cost, one.max_latency_us) == (two.index, two.cost, two.max_latency_us)
+    assert one.n_decided == two.n_decided == one.n_full_evals == (1 << 22) - 82
+    parts = [pl.plan(p.arrivals_us, p.sla_us, p.windows_us, shard=s, n_shards=3, **rng_kw) for s in range(3)]
+    assert sum(r.n_decided for r in parts) == one.n_decided
+    assert all(r.n_decided > 0 for r in parts)
+    best = min((r for r in parts if r.feasible), key=lambda r: (r.cost, r.index))
+    assert (best.index, best.cost) == (one.index, one.cost)
+
+
 # ---------------------------------------------------------------------------------------
 # Cost-bound pruning against an incumbent, and the caller's cost cap (DESIGN.md section 5
 # item 11): only candidates costing strictly more than a real feasible candidate (or the
