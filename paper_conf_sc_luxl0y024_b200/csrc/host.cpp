@@ -1866,9 +1866,10 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 CK(ctx->dListCntA.ensure(1), "cudaMalloc");
                 // best-first: with the cost bound on, the shallow survivors are sorted by their
                 // static cost lower bound so the first deep launch sets a good incumbent early
-                // (SMILESS_BB_SORT=0: atomic append order)
+                // (SMILESS_BB_SORT=1; off by default: measured slower on C2 with live windows and
+                // no faster elsewhere, profiles/r02k_bb_sort.md)
                 const char *sort_env = getenv("SMILESS_BB_SORT");
-                const bool bb_sort = pp.cost_prune && (!sort_env || atoi(sort_env) != 0);
+                const bool bb_sort = pp.cost_prune && sort_env && atoi(sort_env) != 0;
                 if (bb_sort) CK(ctx->dListKeyA.ensure((size_t)batch), "cudaMalloc keys");
                 std::vector<u64> h_pref, h_key;
                 std::vector<uint32_t> h_ord;
