@@ -327,15 +327,16 @@ def throughput_slice(name, S, dev, stream, local, steps=2, n_cand=1 << 24):
     torch.cuda.synchronize(dev)
     sec = a.elapsed_time(b) / 1e3
     scale_out = virtual_sink(p)
+    memo = r.eval_path in (S.PATH_MEMO, S.PATH_MEMO_FUSED)
     ops = (plan_kernel_ops_per_candidate(p) if scale_out else
-           algorithmic_ops_per_candidate(p, memo=os.environ.get("SMILESS_MEMO", "1") != "0",
-                                         split=os.environ.get("SMILESS_SPLITCOST", "1") != "0"))
+           algorithmic_ops_per_candidate(p, memo=memo, split=os.environ.get("SMILESS_SPLITCOST", "1") != "0"))
     value = steps * r.n_decided / sec
     return {"candidates_per_step": r.n_decided, "value": value, "unit": UNIT,
             "function_steps_per_s": value * p.n_funcs * (len(p.arrivals_us) - 1),
             "slice": f"first {n_cand} candidates, functions 0..{nf - 1} pinned to digits {fixed}",
             "kernel": ("smiless_plan_kernel (scaled-out last function: virtual sink)" if scale_out else
-                       "memoised upstream + variants" + (" (scale-out upstream rings)" if p.instances is not None else "")),
+                       KERNEL_LABEL.get(r.eval_path, "smiless_plan_kernel") +
+                       (" (scale-out upstream rings)" if p.instances is not None else "")),
             "int_ops_per_candidate": ops, "achieved_int_ops_per_s": ops * r.n_decided / (kms / steps / 1e3),
             "instances": None if p.instances is None else p.instances.tolist(),
             "winner": {"index": r.index, "cost": r.cost} if r.feasible else None}
@@ -365,6 +366,18 @@ PAPER_CONTEXT = {
 }
 
 
+TRAFFIC_BASIS = {
+    3: "ncu dram__bytes_read+write per plan call (profiles/ncu_memo_summary.json): the memoised x-buffer "
+       "round trip, ~5.4 GB per 65,536 prefixes",
+    4: "ncu dram__bytes_read+write per plan call (profiles/ncu_fused_summary.json): the fused kernel keeps "
+       "the x stream in a shared-memory ring; what is left is the tables, offsets and the cost re-walk",
+}
+KERNEL_LABEL = {
+    3: "smiless_variants_kernel + smiless_upstream_kernel (prefix memoisation, x stream through HBM)",
+    4: "smiless_fused_kernel (prefix memoisation: producer warp -> shared-memory ring -> consumer warps)",
+}
+
+
 def measured_peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -372,14 +385,20 @@ def measured_peaks():
         return {}
 
 
-def ncu_traffic(memo: bool, plan_launches: int, split: bool = True):
+def ncu_traffic(path: int, plan_launches: int, split: bool = True):
     """DRAM bytes of the timed kernels per plan call (the unit `achieved` uses), from the
-    committed ncu --set full summaries.  Memo path: one plan call = prep + B x (upstream,
-    variants[, variants cost]) + reduce + exact, so B = (launches - 3) / 3 batches with the
-    split cost (2 without), each moving the upstream kernel's x-buffer write and the variants
-    kernel's read of it (the cost pass re-reads the few units with a feasible candidate)."""
+    committed ncu --set full summaries.  Fused memo path (PATH_MEMO_FUSED): one plan call =
+    prep + B x (fused[, plan-kernel cost re-walk]) + reduce + exact; the x stream stays in
+    shared memory, so a batch moves only the tables, offsets and the re-walked units' inputs.
+    Two-kernel memo path: B x (upstream, variants[, variants cost]), each batch moving the
+    upstream kernel's x-buffer write and the variants kernel's read of it."""
+    PATH_MEMO, PATH_MEMO_FUSED = 3, 4
     try:
-        if memo:
+        if path == PATH_MEMO_FUSED:
+            d = json.load(open(os.path.join(ROOT, "profiles", "ncu_fused_summary.json")))
+            per = sum(k["dram_bytes_per_launch"] for k in d["launches"] if k["dram_bytes_per_launch"] == k["dram_bytes_per_launch"])
+            return per * max(1, (plan_launches - 3) // (2 if split else 1))
+        if path == PATH_MEMO:
             d = json.load(open(os.path.join(ROOT, "profiles", "ncu_memo_summary.json")))
             pair = sum(k["dram_bytes_per_launch"] for k in d["launches"])
             return pair * max(1, (plan_launches - 3) // (3 if split else 2))
@@ -711,7 +730,7 @@ def main():
     clocks = clk.summary()
     sm_mhz = clocks["sm_mhz"] or peaks.get("sm_max_mhz", 1965.0)
     peak_ops = props.multi_processor_count * ISSUE_LANES_PER_CLK_PER_SM * float(clocks["sm_max_mhz"] or 1965.0) * 1e6
-    memo = os.environ.get("SMILESS_MEMO", "1") != "0"
+    memo = res.eval_path in (S.PATH_MEMO, S.PATH_MEMO_FUSED)
     split = os.environ.get("SMILESS_SPLITCOST", "1") != "0"
     ops_per_cand = algorithmic_ops_per_candidate(p, memo=memo, split=split)
     ops = ops_per_cand * res.n_decided
@@ -736,11 +755,9 @@ def main():
                 "bytes_basis": "counted by the library per smiless_plan call (smiless_plan_result)"},
         "clocks": clocks,
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_ops, "unit": "int-ops/s",
-                     "frac": achieved / peak_ops, "traffic": ncu_traffic(memo, res.launches, split),
-                     "traffic_basis": "ncu dram__bytes_read+write per plan call (profiles/ncu_memo_summary.json): "
-                                      "the memoised x-buffer round trip, ~5.4 GB per 65,536-prefix batch",
-                     "kernel": ("smiless_variants_kernel + smiless_upstream_kernel (prefix memoisation)"
-                                if memo else "smiless_plan_kernel"),
+                     "frac": achieved / peak_ops, "traffic": ncu_traffic(res.eval_path, res.launches, split),
+                     "traffic_basis": TRAFFIC_BASIS.get(res.eval_path, "ncu dram__bytes_read+write per plan call"),
+                     "kernel": KERNEL_LABEL.get(res.eval_path, "smiless_plan_kernel"),
                      "kernel_ms_per_launch": kernel_ms_per_step,
                      "int_ops_per_candidate": ops_per_cand, "configs_per_lane": configs_per_lane(p),
                      "peak_basis": "issue peak: SMs x 4 SMSP x 32 lanes x sm_max_mhz (DESIGN.md Roofline)"},

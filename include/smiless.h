@@ -175,7 +175,20 @@ typedef struct {
                                  the device, windows / tables when changed, counts, caps)          */
     uint64_t d2h_bytes;       /* device -> host bytes this call copied (result block, counts,
                                  cost_out)                                                         */
+    int32_t eval_path;        /* which evaluator path decided the range: SMILESS_PATH_*            */
+    int32_t reserved;         /* 0                                                                 */
 } smiless_plan_result;
+
+/* smiless_plan_result.eval_path */
+enum {
+    SMILESS_PATH_NONE = 0,       /* nothing to search (empty range or every function pinned)      */
+    SMILESS_PATH_PLAN = 1,       /* smiless_plan_kernel over the range (prune mode: compaction)    */
+    SMILESS_PATH_BNB = 2,        /* branch-and-bound pre-pass + smiless_plan_kernel in list mode   */
+    SMILESS_PATH_MEMO = 3,       /* throughput mode, prefix memoisation: upstream + variants kernels
+                                    with the x stream through HBM                                 */
+    SMILESS_PATH_MEMO_FUSED = 4  /* throughput mode, prefix memoisation in one kernel: producer warp
+                                    -> shared-memory ring -> consumer warps (x stays on chip)     */
+};
 
 /* Size of the suffix candidate space prod_{k >= n_fixed} M_k * W.
  * Returns OK, ESTATE (profiles not loaded), EINVAL or ERANGE (> 2^63). */

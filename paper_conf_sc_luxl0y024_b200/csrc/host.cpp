@@ -731,23 +731,38 @@ bool split_cost() {
 // warp walks the upstream functions of a tile of prefixes into a shared-memory ring that its
 // consumer warps read, so the x stream never leaves the SM.  Needs the int32 path, a last
 // function that is not scaled out, and a tile of 1..32 prefixes.  SMILESS_FUSED=0: two kernels.
-constexpr int kFusedSlots = 4, kFusedSteps = 64;   // mirror SM_FSLOTS, SM_FPS
+constexpr int kFusedSteps = 64;                      // mirrors SM_FPS
+int fused_slots() {                                  // ring depth (SM_FSLOTS)
+    const char *e = getenv("SMILESS_FSLOTS");
+    const int v = e ? atoi(e) : 4;
+    return (v >= 2 && v <= 8) ? v : 4;
+}
+int fused_min_blocks() {                             // min CTAs/SM of the fused kernel (SM_FMINB)
+    const char *e = getenv("SMILESS_FMINB");
+    const int v = e ? atoi(e) : 2;
+    return (v >= 1 && v <= 4) ? v : 2;
+}
+int fused_producers() {                              // producer warps per CTA (SM_FPW)
+    const char *e = getenv("SMILESS_FPW");
+    const int v = e ? atoi(e) : 1;
+    return (v >= 1 && v <= 4) ? v : 1;
+}
 int fused_tile(const smiless_ctx *ctx, const smiless_plan_args *a) {
-    return (vthreads_per_cta() / 32 - 1) * 32 / (ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
+    return (vthreads_per_cta() / 32 - fused_producers()) * 32 / (ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
 }
 bool fused_on(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp) {
     const char *e = getenv("SMILESS_FUSED");
     if (!e || atoi(e) == 0) return false;      // off unless SMILESS_FUSED=1 (until measured)
     if (rp.time64 || inst_of(a, ctx->N - 1) > 1) return false;
-    const int tp = fused_tile(ctx, a);
-    return tp >= 1 && tp <= 32;
+    const int tp = fused_tile(ctx, a), fpw = fused_producers();
+    return tp >= 1 && (tp + fpw - 1) / fpw <= 32 && 32 * fpw <= kThreads;
 }
 size_t smem_fused(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off) {
     const size_t padI = (size_t)((ctx->sumM + 3) & ~3), padU = (size_t)((ctx->sumM + 1) & ~1);
-    const size_t fc32 = (size_t)(vthreads_per_cta() / 32 - 1) * 32;
+    const size_t fc32 = (size_t)(vthreads_per_cta() / 32 - fused_producers()) * 32;
     (void)rp;
     return 3 * padI * 4 + padU * 8 + 4 * (size_t)n_off + (split_cost() ? 0 : 8 * (size_t)unit_cands(ctx, a) * fc32) +
-           4 * (size_t)kFusedSlots * kFusedSteps * (size_t)fused_tile(ctx, a) +
+           4 * (size_t)fused_slots() * kFusedSteps * (size_t)fused_tile(ctx, a) +
            ((4 * (size_t)ctx->N * kThreads + 15) & ~(size_t)15);
 }
 
@@ -798,7 +813,8 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_LBT " << (bound_lb_table(ctx, W) ? 1 : 0) << "\n";
     s << "#define SM_XPF " << xpf_groups() << "\n";
     s << "#define SM_SPLITCOST " << (split_cost() ? 1 : 0) << "\n";
-    s << "#define SM_FUSED " << (((families & FAM_MEMO) && fused_on(ctx, a, rp)) ? 1 : 0) << "\n";
+    s << "#define SM_FUSED " << (((families & FAM_MEMO) && fused_on(ctx, a, rp)) ? 1 : 0) << "\n#define SM_FSLOTS "
+      << fused_slots() << "\n#define SM_FMINB " << fused_min_blocks() << "\n#define SM_FPW " << fused_producers() << "\n";
     // window variants of the memoised kernel walked in the positive-time form (evaluator.cuh
     // variants_step FM: ALU busy mask + full-rate IMAD instead of the quarter-rate IMAD.HI)
     // default: every window variant (measured: 3.45e8 -> 3.81e8 candidates/s on the C2 slice,
@@ -1504,6 +1520,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     cudaStream_t st = ctx->stream;
     CK(cudaEventRecord(ctx->ev[0], st), "event");
     int launches = 0;
+    int32_t eval_path = SMILESS_PATH_NONE;
 
     const i64 *d_arr = nullptr;
     if ((rc = stage_arrivals(ctx, a, &d_arr))) return rc;
@@ -1608,6 +1625,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         pp.list_upp = 1;
         const bool memo = memo_path && jk->blocks_up > 0 && jk->blocks_var > 0;
         if (memo && jk->fn_fused) {
+            eval_path = SMILESS_PATH_MEMO_FUSED;
             // ---- fused memoisation: upstream walked by each CTA's producer warp into a shared-
             // memory ring, variants by its consumer warps (evaluator.cuh smiless_fused_kernel);
             // split cost: the units holding a feasible candidate are re-walked by the plan
@@ -1692,6 +1710,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             }
             grid_used = std::max(grid, grid_f);
         } else if (memo) {
+            eval_path = SMILESS_PATH_MEMO;
             // ---- prefix memoisation: upstream once per prefix, then the variants per unit ---------
             const u64 upp = (u64)(ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
             const u64 pl0 = ub / upp, ph0 = (ue + upp - 1) / upp;
@@ -1776,6 +1795,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             }
             grid_used = std::max(grid, grid_var);
         } else if (bnb_path && D > 0 && jk->blocks_bound > 0) {
+            eval_path = SMILESS_PATH_BNB;
             // ---- exact branch-and-bound: prefixes of functions n_fixed..D-1, then list mode ----
             // Sharding (multi-GPU): the deep level's prefixes (one level) or the deep children of
             // every shallow survivor (two levels) are interleaved over the shards, ordinal
@@ -1999,6 +2019,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 }
             }
         } else {
+            eval_path = SMILESS_PATH_PLAN;
             // split very large ranges into several launches (bounded kernel duration).  Prune mode
             // with J - 1 > horizon runs each batch twice: pass 1 (every unit, `horizon` steps,
             // survivors compacted into a list), pass 2 (survivors only, all steps).
@@ -2134,6 +2155,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         r.launches = launches;
         r.h2d_bytes = ctx->h2d;
         r.d2h_bytes = ctx->d2h;
+        r.eval_path = eval_path;
         int32_t *co = config_out ? config_out + (size_t)s_ * ctx->N : nullptr;
         int32_t *wo = window_out ? window_out + (size_t)s_ * ctx->N : nullptr;
         if (!found) {

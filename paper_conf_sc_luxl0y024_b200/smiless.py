@@ -19,6 +19,7 @@ LIB_PATH = os.path.join(_PKG, "libsmiless.so")
 OK, INFEASIBLE = 0, 1
 EINVAL, ENOTTOPO, ERANGE, ESTATE, ECUDA, ENOMEM, EJIT = -1, -2, -3, -4, -5, -6, -7
 FLAG_NO_PRUNE, FLAG_ARRIVALS_ON_DEVICE, FLAG_FORCE_INT64, FLAG_COST_CAP = 1, 2, 4, 8
+PATH_NONE, PATH_PLAN, PATH_BNB, PATH_MEMO, PATH_MEMO_FUSED = 0, 1, 2, 3, 4   # smiless_plan_result.eval_path
 _NAMES = {0: "OK", 1: "INFEASIBLE", -1: "EINVAL", -2: "ENOTTOPO", -3: "ERANGE", -4: "ESTATE",
           -5: "ECUDA", -6: "ENOMEM", -7: "EJIT"}
 
@@ -73,6 +74,8 @@ class PlanResultC(ctypes.Structure):
         ("launches", ctypes.c_int32),
         ("h2d_bytes", ctypes.c_uint64),
         ("d2h_bytes", ctypes.c_uint64),
+        ("eval_path", ctypes.c_int32),
+        ("reserved", ctypes.c_int32),
     ]
 
 
@@ -96,6 +99,7 @@ class PlanResult:
     launches: int
     h2d_bytes: int = 0          # host -> device bytes the call copied (counted by the library)
     d2h_bytes: int = 0          # device -> host bytes the call copied
+    eval_path: int = 0          # PATH_* (which evaluator path decided the range)
 
     @property
     def feasible(self) -> bool:
@@ -302,7 +306,7 @@ class Planner:
                           window=win[:self.n_funcs], n_decided=int(r.n_decided), n_full_evals=int(r.n_full_evals),
                           eval_kernel_ms=float(r.eval_kernel_ms), total_device_ms=float(r.total_device_ms),
                           int64_path=bool(r.int64_path), launches=int(r.launches),
-                          h2d_bytes=int(r.h2d_bytes), d2h_bytes=int(r.d2h_bytes))
+                          h2d_bytes=int(r.h2d_bytes), d2h_bytes=int(r.d2h_bytes), eval_path=int(r.eval_path))
 
     def plan_sla_sweep(self, arrivals, slas_us, windows_us, **kw):
         """One pass over the space, one winner per SLA (smiless_plan_sla_sweep)."""

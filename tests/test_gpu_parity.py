@@ -740,6 +740,7 @@ def test_fused_memo_kernel_is_exact(g, split, monkeypatch):
         assert_dump_matches(out, oc, of)
         assert_same_plan(r, o.plan(begin=b), o)
         assert r.n_full_evals == r.n_decided == space - b
+        assert r.eval_path == S.PATH_MEMO_FUSED
         n_checked += 1
         if n_checked >= 12:
             break
@@ -763,6 +764,7 @@ def test_fused_memo_kernel_shards_and_matches_two_kernel_path(monkeypatch):
     one = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, **rng_kw)
     assert (one.index, one.cost, one.max_latency_us) == (two.index, two.cost, two.max_latency_us)
     assert one.n_decided == two.n_decided == one.n_full_evals == (1 << 22) - 82
+    assert (one.eval_path, two.eval_path) == (S.PATH_MEMO_FUSED, S.PATH_MEMO)
     parts = [pl.plan(p.arrivals_us, p.sla_us, p.windows_us, shard=s, n_shards=3, **rng_kw) for s in range(3)]
     assert sum(r.n_decided for r in parts) == one.n_decided
     assert all(r.n_decided > 0 for r in parts)
