@@ -1717,10 +1717,20 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             const size_t tsz2 = rp.time64 ? 8 : 4;
             // + SM_XPF + 1 groups of 4 steps of read-ahead slack for the variants kernel
             const size_t row_bytes = tsz2 * (size_t)(n_off + 4 * (xpf_groups() + 1));
-            u64 max_batch = std::max<u64>(1, std::min<u64>((u64)1 << 16, ((u64)4 << 30) / row_bytes));
-            if (const char *mb_env = getenv("SMILESS_MEMO_BATCH"))   // tuning: prefixes per batch (<= 64 GB buffer)
+            // Batches of up to 2^20 prefixes (fewer launches, fewer tails, a fuller upstream
+            // kernel: 3.80e8 -> 3.95e8 candidates/s on the C2 slice, profiles/r02l_memo_batch.md),
+            // the x buffer bounded by a quarter of the device memory; halved while the
+            // allocation fails.  SMILESS_MEMO_BATCH (tuning) sets the prefixes per batch.
+            size_t mem_free = 0, mem_total = 0;
+            CK(cudaMemGetInfo(&mem_free, &mem_total), "cudaMemGetInfo");
+            u64 max_batch = std::max<u64>(1, std::min<u64>((u64)1 << 20, (u64)(mem_total / 4) / row_bytes));
+            if (const char *mb_env = getenv("SMILESS_MEMO_BATCH"))
                 max_batch = std::max<u64>(1, std::min<u64>((u64)atoll(mb_env), ((u64)64 << 30) / row_bytes));
-            const u64 batch_p = std::min<u64>(max_batch, ph0 - pl0);
+            u64 batch_p = std::min<u64>(max_batch, ph0 - pl0);
+            while (ctx->dX.ensure((size_t)batch_p * row_bytes) != cudaSuccess && batch_p > 1) {
+                cudaGetLastError();                                  // clear the allocation failure
+                batch_p = (batch_p + 1) / 2;
+            }
             CK(ctx->dX.ensure((size_t)batch_p * row_bytes), "cudaMalloc memo buffer");
             CK(ctx->dRecNx.ensure((size_t)batch_p), "cudaMalloc");
             CK(ctx->dRecNlu.ensure((size_t)batch_p), "cudaMalloc");
