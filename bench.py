@@ -396,7 +396,8 @@ def ncu_traffic(path: int, plan_launches: int, split: bool = True):
     try:
         if path == PATH_MEMO_FUSED:
             d = json.load(open(os.path.join(ROOT, "profiles", "ncu_fused_summary.json")))
-            per = sum(k["dram_bytes_per_launch"] for k in d["launches"] if k["dram_bytes_per_launch"] == k["dram_bytes_per_launch"])
+            per = sum(k["dram_bytes_per_launch"] for k in d.get("launches", [d])
+                      if k["dram_bytes_per_launch"] == k["dram_bytes_per_launch"])      # skip NaN
             return per * max(1, (plan_launches - 3) // (2 if split else 1))
         if path == PATH_MEMO:
             d = json.load(open(os.path.join(ROOT, "profiles", "ncu_memo_summary.json")))

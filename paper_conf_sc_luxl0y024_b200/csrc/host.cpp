@@ -739,27 +739,35 @@ int fused_slots() {                                  // ring depth (SM_FSLOTS)
 }
 int fused_min_blocks() {                             // min CTAs/SM of the fused kernel (SM_FMINB)
     const char *e = getenv("SMILESS_FMINB");
-    const int v = e ? atoi(e) : 2;
-    return (v >= 1 && v <= 4) ? v : 2;
-}
-int fused_producers() {                              // producer warps per CTA (SM_FPW)
-    const char *e = getenv("SMILESS_FPW");
     const int v = e ? atoi(e) : 1;
     return (v >= 1 && v <= 4) ? v : 1;
 }
+// Default shape: one 640-thread CTA per SM, 16 consumer warps and 4 producer warps (16 lanes
+// each), so each SM sub-partition runs 4 consumers and 1 producer (profiles/r02l_memo_batch.md:
+// with the producers on one SMSP its issue rate fell to 51 %)
+int fused_producers() {                              // producer warps per CTA (SM_FPW)
+    const char *e = getenv("SMILESS_FPW");
+    const int v = e ? atoi(e) : 4;
+    return (v >= 1 && v <= 8) ? v : 4;
+}
+int fused_threads() {                                // CTA size (SM_FTHREADS)
+    const char *e = getenv("SMILESS_FTHREADS");
+    const int v = e ? atoi(e) : 640;
+    return (v >= 64 && v <= 1024 && v % 32 == 0) ? v : 640;
+}
 int fused_tile(const smiless_ctx *ctx, const smiless_plan_args *a) {
-    return (vthreads_per_cta() / 32 - fused_producers()) * 32 / (ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
+    return (fused_threads() / 32 - fused_producers()) * 32 / (ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
 }
 bool fused_on(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp) {
     const char *e = getenv("SMILESS_FUSED");
-    if (!e || atoi(e) == 0) return false;      // off unless SMILESS_FUSED=1 (until measured)
+    if (e && atoi(e) == 0) return false;
     if (rp.time64 || inst_of(a, ctx->N - 1) > 1) return false;
     const int tp = fused_tile(ctx, a), fpw = fused_producers();
     return tp >= 1 && (tp + fpw - 1) / fpw <= 32 && 32 * fpw <= kThreads;
 }
 size_t smem_fused(const smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp, i64 n_off) {
     const size_t padI = (size_t)((ctx->sumM + 3) & ~3), padU = (size_t)((ctx->sumM + 1) & ~1);
-    const size_t fc32 = (size_t)(vthreads_per_cta() / 32 - fused_producers()) * 32;
+    const size_t fc32 = (size_t)(fused_threads() / 32 - fused_producers()) * 32;
     (void)rp;
     return 3 * padI * 4 + padU * 8 + 4 * (size_t)n_off + (split_cost() ? 0 : 8 * (size_t)unit_cands(ctx, a) * fc32) +
            4 * (size_t)fused_slots() * kFusedSteps * (size_t)fused_tile(ctx, a) +
@@ -814,7 +822,8 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     s << "#define SM_XPF " << xpf_groups() << "\n";
     s << "#define SM_SPLITCOST " << (split_cost() ? 1 : 0) << "\n";
     s << "#define SM_FUSED " << (((families & FAM_MEMO) && fused_on(ctx, a, rp)) ? 1 : 0) << "\n#define SM_FSLOTS "
-      << fused_slots() << "\n#define SM_FMINB " << fused_min_blocks() << "\n#define SM_FPW " << fused_producers() << "\n";
+      << fused_slots() << "\n#define SM_FMINB " << fused_min_blocks() << "\n#define SM_FPW " << fused_producers()
+      << "\n#define SM_FTHREADS " << fused_threads() << "\n";
     // window variants of the memoised kernel walked in the positive-time form (evaluator.cuh
     // variants_step FM: ALU busy mask + full-rate IMAD instead of the quarter-rate IMAD.HI)
     // default: every window variant (measured: 3.45e8 -> 3.81e8 candidates/s on the C2 slice,
@@ -1156,7 +1165,7 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
                 r = driver().funcSetAttribute(jk.fn_fused, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
                                               (int)jk.smem_fused);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(fused smem)");
-                r = driver().occupancy(&jk.blocks_fused, jk.fn_fused, vthreads_per_cta(), jk.smem_fused);
+                r = driver().occupancy(&jk.blocks_fused, jk.fn_fused, fused_threads(), jk.smem_fused);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(fused)");
                 if (jk.blocks_fused < 1) jk.fn_fused = nullptr;
             }
@@ -1695,7 +1704,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
                 if (split) CK(cudaMemsetAsync(ctx->dCostN.p, 0, sizeof(unsigned), st), "memset cost list");
                 void *args[] = {&mp};
-                CUresult r = driver().launchKernel(jk->fn_fused, (unsigned)grid_f, 1, 1, vthreads_per_cta(), 1, 1,
+                CUresult r = driver().launchKernel(jk->fn_fused, (unsigned)grid_f, 1, 1, fused_threads(), 1, 1,
                                                    (unsigned)jk->smem_fused, (CUstream)st, args, nullptr);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "fused launch");
                 ++launches;

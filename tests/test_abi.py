@@ -193,10 +193,10 @@ def test_fused_memo_kernel_compiles_for_the_bench_slice(monkeypatch):
     p, kw = bench.workload("C2")
     pl = S.planner_for(p)
     args = (p.arrivals_us, p.sla_us, p.windows_us)
+    assert "#define SM_FUSED 1" in pl.kernel_source(*args, flags=S.FLAG_NO_PRUNE, **kw)
     monkeypatch.setenv("SMILESS_FUSED", "0")
     assert "#define SM_FUSED 0" in pl.kernel_source(*args, flags=S.FLAG_NO_PRUNE, **kw)
-    monkeypatch.setenv("SMILESS_FUSED", "1")
-    assert "#define SM_FUSED 1" in pl.kernel_source(*args, flags=S.FLAG_NO_PRUNE, **kw)
+    monkeypatch.delenv("SMILESS_FUSED")
     log, n = pl.jit_compile(*args, flags=S.FLAG_NO_PRUNE, **kw)
     entry = log.split("Compiling entry function 'smiless_fused_kernel'")[1].split("Compiling entry")[0]
     assert "0 bytes stack frame, 0 bytes spill stores, 0 bytes spill loads" in entry, entry

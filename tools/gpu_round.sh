@@ -14,7 +14,7 @@ timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > $O/${TAG}_be
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $O/${TAG}_launches.csv \
     python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-full-space --no-c4 --no-pruned --no-extra > $O/${TAG}_ncu_launch_bench.log 2>&1
 echo "ncu launches exit $?"
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:"smiless_(variants|upstream)_kernel" -c 2 \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"smiless_(fused|plan|variants|upstream)_kernel" -c 2 \
     -o $O/${TAG}_prof_eval -f python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-full-space --no-c4 --no-pruned --no-extra \
     > $O/${TAG}_ncu_full.log 2>&1
 echo "ncu full exit $?"
