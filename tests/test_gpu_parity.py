@@ -752,6 +752,39 @@ def test_fused_memo_kernel_is_exact(g, split, monkeypatch):
     assert n_checked >= 6
 
 
+def test_fused_memo_kernel_with_scaled_out_upstream(monkeypatch):
+    """The fused kernel's producers with instance rings and the scale-out prologue (upstream
+    functions with 2-4 round-robin instances, the last one with 1, as C3): per-candidate
+    parity with the oracle."""
+    monkeypatch.setenv("SMILESS_FUSED", "1")
+    rng = np.random.default_rng(577)
+    n_checked = 0
+    for t in range(200):
+        n = int(rng.integers(2, 5))
+        p = W.random_problem(rng, n, 16, int(rng.integers(1, 4)), int(rng.choice([3, 9, 17, 70, 131])))
+        space = p.space_size()
+        if space > 40000:
+            continue
+        inst = [int(rng.integers(1, 5)) for _ in range(n - 1)] + [1]
+        if max(inst) == 1:
+            continue
+        pl = S.planner_for(p)
+        kw = dict(flags=S.FLAG_NO_PRUNE, instances=inst)
+        if "#define SM_FUSED 1" not in pl.kernel_source(p.arrivals_us, p.sla_us, p.windows_us, **kw):
+            continue
+        o = OracleProblem(p, instances=inst)
+        oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
+        out = np.empty(space)
+        r = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, cost_out=out, **kw)
+        assert r.eval_path == S.PATH_MEMO_FUSED
+        assert_dump_matches(out, oc, of)
+        assert_same_plan(r, o.plan(), o)
+        n_checked += 1
+        if n_checked >= 10:
+            break
+    assert n_checked >= 5
+
+
 def test_fused_memo_kernel_shards_and_matches_two_kernel_path(monkeypatch):
     """Fused vs two-kernel memoisation on the bench slice of C2 at J = 10^4 (2^28 candidates
     is too long here: a 2^22-candidate range around the winner), bit-identical winner; and the
