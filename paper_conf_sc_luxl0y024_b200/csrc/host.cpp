@@ -278,7 +278,7 @@ struct JitKernel {
     CUmodule mod = nullptr;
     CUfunction fn = nullptr;
     CUfunction fn_bound = nullptr, fn_bound_a = nullptr, fn_up = nullptr, fn_var = nullptr, fn_varc = nullptr;
-    CUfunction fn_fused = nullptr;
+    CUfunction fn_fused = nullptr, fn_bound_m = nullptr;
     size_t smem_up = 0, smem_var = 0, smem_fused = 0;
     int blocks_up = 0, blocks_var = 0, blocks_fused = 0;
     size_t smem = 0, smem_bound = 0;
@@ -344,9 +344,9 @@ struct smiless_ctx {
     DevBuf<i64> dLat;
     DevBuf<unsigned char> dFeas;
     DevBuf<double> dDump;
-    DevBuf<u64> dList, dListA, dCostList, dListKeyA;
+    DevBuf<u64> dList, dListA, dListM, dCostList, dListKeyA;
     DevBuf<unsigned> dCostN;
-    DevBuf<unsigned> dListCnt, dListCntA, dChunkCnt;
+    DevBuf<unsigned> dListCnt, dListCntA, dListCntM, dChunkCnt, dChunkCntM;
     DevBuf<int> dW;                          // per-row windows of the current plan (padded)
     DevBuf<unsigned char> dX;                // memoised last-function inputs [n_off/4][prefix][4]
     DevBuf<i64> dRecNx, dRecNlu;             // per-prefix records (int32 or int64 time)
@@ -710,6 +710,24 @@ int bb_depth_a(const smiless_ctx *ctx, const smiless_plan_args *a, int D) {
     return best;
 }
 
+// Middle B&B level (three-level scheme): when every shallow survivor has more than 2^16 deep
+// children, a level at DM = DA + ceil((D - DA) / 2) prunes them first, so the deep level only
+// enumerates the children of middle survivors (C5: 2^28 deep children per shallow survivor
+// become 2 x 2^14).  0: none.  SMILESS_BB_DEPTH_M overrides (0 disables).
+int bb_depth_m(const smiless_ctx *ctx, const smiless_plan_args *a, int D, int DA) {
+    if (D <= 0 || DA <= 0) return 0;
+    const char *env = getenv("SMILESS_BB_DEPTH_M");
+    if (env) {
+        const int d = atoi(env);
+        return (d > DA && d < D) ? d : 0;
+    }
+    if (D - DA < 2) return 0;
+    unsigned __int128 r = 1;
+    for (int k = DA; k < D; ++k) r *= (u64)ctx->M[k] * (u64)a->n_windows;
+    if (r <= ((unsigned __int128)1 << 16)) return 0;
+    return DA + (D - DA + 1) / 2;
+}
+
 u64 cands_per_prefix(const smiless_ctx *ctx, const smiless_plan_args *a, int d) {
     u64 s = 1;
     for (int k = d; k < ctx->N; ++k) s *= (u64)ctx->M[k] * (u64)a->n_windows;
@@ -815,7 +833,7 @@ std::string dag_spec_source(const smiless_ctx *ctx, const smiless_plan_args *a, 
     const int D = bb_depth(ctx, a);
     const int DA = bb_depth_a(ctx, a, D);
     s << "#define SM_D " << (D > 0 ? D : N - 1) << "\n#define SM_DA " << (DA > 0 ? DA : (D > 0 ? D : N - 1))
-      << "\n#define SMILESS_MAXF " << SMILESS_MAX_FUNCS << "\n";
+      << "\n#define SM_DM " << bb_depth_m(ctx, a, D, DA) << "\n#define SMILESS_MAXF " << SMILESS_MAX_FUNCS << "\n";
     s << "#define SM_NSLA " << ctx->nsla << "\n";
     s << "#define SM_ROWWIN " << (a->row_windows_us ? 1 : 0) << "\n";
     s << "#define SM_LBT " << (bound_lb_table(ctx, W) ? 1 : 0) << "\n";
@@ -1124,6 +1142,11 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
             if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound)");
             r = driver().moduleGetFunction(&jk.fn_bound_a, jk.mod, "smiless_bound_kernel_a");
             if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound_a)");
+            const int D = bb_depth(ctx, a);
+            if (bb_depth_m(ctx, a, D, bb_depth_a(ctx, a, D)) > 0) {
+                r = driver().moduleGetFunction(&jk.fn_bound_m, jk.mod, "smiless_bound_kernel_m");
+                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuModuleGetFunction(bound_m)");
+            }
         }
         if (families & FAM_MEMO) {
             r = driver().moduleGetFunction(&jk.fn_up, jk.mod, "smiless_upstream_kernel");
@@ -1179,6 +1202,11 @@ int get_kernel(smiless_ctx *ctx, const smiless_plan_args *a, const RangePlan &rp
                 r = driver().funcSetAttribute(jk.fn_bound_a, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
                                               (int)jk.smem_bound);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(bound_a smem)");
+                if (jk.fn_bound_m) {
+                    r = driver().funcSetAttribute(jk.fn_bound_m, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
+                                                  (int)jk.smem_bound);
+                    if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "cuFuncSetAttribute(bound_m smem)");
+                }
                 r = driver().occupancy(&jk.blocks_bound, jk.fn_bound, kThreads, jk.smem_bound);
                 if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "occupancy(bound)");
             }
@@ -1287,6 +1315,7 @@ void smiless_destroy(smiless_ctx *ctx) {
         ctx->dCost.release(); ctx->dLat.release(); ctx->dFeas.release(); ctx->dRes.release(); ctx->dDump.release();
         ctx->dList.release(); ctx->dListCnt.release(); ctx->dW.release();
         ctx->dListA.release(); ctx->dListCntA.release(); ctx->dChunkCnt.release(); ctx->dListKeyA.release();
+        ctx->dListM.release(); ctx->dListCntM.release(); ctx->dChunkCntM.release();
         ctx->dCostList.release(); ctx->dCostN.release();
         ctx->dX.release(); ctx->dRecNx.release(); ctx->dRecNlu.release(); ctx->dRecPre.release();
         if (ctx->hRes) cudaFreeHost(ctx->hRes);
@@ -1966,54 +1995,103 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                         ctx->h2d += (u64)n_a * sizeof(u64);
                         hp.mark("sort_a");
                     }
-                    // deep launches (first survivor entry, entries, first child, children per entry):
-                    // at most list_cap ordinals each.  With the cost bound on, the first launch is small:
-                    // its evaluation sets the incumbent the static prefix bound of every later launch
-                    // prunes against.
+                    // Launches over a survivor list (first entry, entries, first child, children per
+                    // entry): at most list_cap ordinals each.  With the cost bound on, the first launch
+                    // is small: its evaluation sets the incumbent the static prefix bound of every later
+                    // launch prunes against.  A survivor with more than list_cap children spans several.
                     struct DeepLaunch { u64 e0; unsigned ne; u64 r0, span; };
-                    std::vector<DeepLaunch> L;
-                    if (R <= list_cap) {
-                        const u64 per_chunk = list_cap / R;
-                        const char *first_env = getenv("SMILESS_BB_FIRST");
-                        const u64 first = std::max<u64>(
-                            1, std::min<u64>(per_chunk, pp.cost_prune ? (first_env ? (u64)atoll(first_env) : 64) : per_chunk));
-                        for (u64 c0 = 0; c0 < n_a;) {
-                            const u64 len = std::min<u64>(c0 == 0 ? first : per_chunk, n_a - c0);
-                            L.push_back({c0, (unsigned)len, 0, R});
-                            c0 += len;
+                    auto make_chunks = [&](u64 n_entries, u64 Rc) {
+                        std::vector<DeepLaunch> L;
+                        if (Rc <= list_cap) {
+                            const u64 per_chunk = list_cap / Rc;
+                            const char *first_env = getenv("SMILESS_BB_FIRST");
+                            const u64 first = std::max<u64>(
+                                1, std::min<u64>(per_chunk,
+                                                 pp.cost_prune ? (first_env ? (u64)atoll(first_env) : 64) : per_chunk));
+                            for (u64 c0 = 0; c0 < n_entries;) {
+                                const u64 len = std::min<u64>(c0 == 0 ? first : per_chunk, n_entries - c0);
+                                L.push_back({c0, (unsigned)len, 0, Rc});
+                                c0 += len;
+                            }
+                        } else {
+                            for (u64 e = 0; e < n_entries; ++e)
+                                for (u64 r0 = 0; r0 < Rc; r0 += list_cap)
+                                    L.push_back({e, 1u, r0, std::min(list_cap, Rc - r0)});
                         }
-                    } else {                                      // a survivor's children over several launches
-                        for (u64 e = 0; e < n_a; ++e)
-                            for (u64 r0 = 0; r0 < R; r0 += list_cap) L.push_back({e, 1u, r0, std::min(list_cap, R - r0)});
-                    }
-                    std::vector<unsigned> cnts(std::max<size_t>(L.size(), 1), 0u);
-                    for (size_t i = 0; i < L.size(); ++i) cnts[i] = L[i].ne;
-                    CK(ctx->dChunkCnt.ensure(cnts.size()), "cudaMalloc counts");
-                    ctx->h2d += cnts.size() * sizeof(unsigned);
-                    CK(cudaMemcpyAsync(ctx->dChunkCnt.p, cnts.data(), cnts.size() * sizeof(unsigned),
-                                       cudaMemcpyHostToDevice, st),
-                       "H2D counts");
-                    bp.list_cap = list_cap;
-                    bp.shard = shard;
-                    bp.n_shards = n_shards;
-                    bp.attr_shard = 0;
-                    bp.attr_n = 1;
-                    NvtxRange nv("bnb deep level + evaluate");
-                    for (size_t i = 0; i < L.size(); ++i) {
-                        CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                        CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
-                        bp.list_in = ctx->dListA.p + L[i].e0;
-                        bp.list_n = ctx->dChunkCnt.p + i;
-                        bp.list_upp = L[i].span;
-                        bp.list_stride = R;
-                        bp.list_r0 = L[i].r0;
-                        bp.prefix_begin = 0;
-                        bp.prefix_end = 0;
-                        bp.cands_per_prefix = S;
-                        bp.list_out = ctx->dList.p;
-                        bp.list_cnt = ctx->dListCnt.p;
-                        if ((rc = run_bound(jk->fn_bound))) return rc;
-                        if ((rc = run_eval())) return rc;
+                        return L;
+                    };
+                    auto upload_counts = [&](const std::vector<DeepLaunch> &L, DevBuf<unsigned> &buf) -> int {
+                        std::vector<unsigned> cnts(std::max<size_t>(L.size(), 1), 0u);
+                        for (size_t i = 0; i < L.size(); ++i) cnts[i] = L[i].ne;
+                        CK(buf.ensure(cnts.size()), "cudaMalloc counts");
+                        ctx->h2d += cnts.size() * sizeof(unsigned);
+                        CK(cudaMemcpyAsync(buf.p, cnts.data(), cnts.size() * sizeof(unsigned), cudaMemcpyHostToDevice, st),
+                           "H2D counts");
+                        return SMILESS_OK;
+                    };
+                    // one level over the children of a survivor list: bound kernel `fn` at depth with
+                    // `Sc` candidates per prefix writes its survivors to out / out_cnt; then `after`
+                    auto run_level = [&](CUfunction fn, const u64 *list, const std::vector<DeepLaunch> &L,
+                                         DevBuf<unsigned> &cnt_buf, u64 Rc, u64 Sc, u64 *out, unsigned *out_cnt,
+                                         int shard_, int n_shards_, const std::function<int(size_t)> &after) -> int {
+                        for (size_t i = 0; i < L.size(); ++i) {
+                            CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                            CK(cudaMemsetAsync(out_cnt, 0, sizeof(unsigned), st), "memset list");
+                            bp.list_in = list + L[i].e0;
+                            bp.list_n = cnt_buf.p + i;
+                            bp.list_upp = L[i].span;
+                            bp.list_stride = Rc;
+                            bp.list_r0 = L[i].r0;
+                            bp.prefix_begin = 0;
+                            bp.prefix_end = 0;
+                            bp.cands_per_prefix = Sc;
+                            bp.list_out = out;
+                            bp.list_cnt = out_cnt;
+                            bp.list_cap = list_cap;
+                            bp.shard = shard_;
+                            bp.n_shards = n_shards_;
+                            bp.attr_shard = 0;
+                            bp.attr_n = 1;
+                            if ((rc = run_bound(fn))) return rc;
+                            if ((rc = after(i))) return rc;
+                        }
+                        return SMILESS_OK;
+                    };
+                    const int DM = jk->fn_bound_m ? bb_depth_m(ctx, a, D, DA) : 0;
+                    if (DM == 0) {
+                        // two levels: the deep children of the shallow survivors, interleaved over shards
+                        const std::vector<DeepLaunch> L = make_chunks(n_a, R);
+                        if ((rc = upload_counts(L, ctx->dChunkCnt))) return rc;
+                        NvtxRange nv("bnb deep level + evaluate");
+                        if ((rc = run_level(jk->fn_bound, ctx->dListA.p, L, ctx->dChunkCnt, R, S, ctx->dList.p,
+                                            ctx->dListCnt.p, shard, n_shards, [&](size_t) { return run_eval(); })))
+                            return rc;
+                    } else {
+                        // three levels: the middle children of the shallow survivors (interleaved over
+                        // shards), then the deep children of each middle launch's survivors (this
+                        // rank's own, not split again) and the evaluator over those
+                        const u64 SMd = cands_per_prefix(ctx, a, DM);
+                        const u64 R1 = SA / SMd, R2 = SMd / S;
+                        CK(ctx->dListM.ensure((size_t)list_cap), "cudaMalloc list");
+                        CK(ctx->dListCntM.ensure(1), "cudaMalloc");
+                        const std::vector<DeepLaunch> Lm = make_chunks(n_a, R1);
+                        if ((rc = upload_counts(Lm, ctx->dChunkCntM))) return rc;
+                        NvtxRange nv("bnb middle + deep level + evaluate");
+                        auto deep = [&](size_t) -> int {
+                            unsigned n_m = 0;
+                            CK(cudaMemcpyAsync(&n_m, ctx->dListCntM.p, sizeof n_m, cudaMemcpyDeviceToHost, st), "D2H count");
+                            ctx->d2h += sizeof n_m;
+                            CK(cudaStreamSynchronize(st), "count");
+                            hp.note("n_m", n_m);
+                            if (n_m == 0) return SMILESS_OK;
+                            const std::vector<DeepLaunch> L = make_chunks(n_m, R2);
+                            if ((rc = upload_counts(L, ctx->dChunkCnt))) return rc;
+                            return run_level(jk->fn_bound, ctx->dListM.p, L, ctx->dChunkCnt, R2, S, ctx->dList.p,
+                                             ctx->dListCnt.p, 0, 1, [&](size_t) { return run_eval(); });
+                        };
+                        if ((rc = run_level(jk->fn_bound_m, ctx->dListA.p, Lm, ctx->dChunkCntM, R1, SMd, ctx->dListM.p,
+                                            ctx->dListCntM.p, shard, n_shards, deep)))
+                            return rc;
                     }
                     hp.mark("chunks_launched");
                     CK(cudaStreamSynchronize(st), "chunks");      // the next batch reuses dListA

@@ -619,10 +619,11 @@ def test_branch_and_bound_with_pinned_digits(monkeypatch):
             continue
         oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
         ref = o.plan()
-        for d in range(nf + 1, n):
-            for da in [0] + list(range(nf + 1, d)):
+        for d, da, dm in [(d, da, dm) for d in range(nf + 1, n) for da in [0] + list(range(nf + 1, d))
+                          for dm in [0] + ([da + 1] if 0 < da and da + 1 < d else [])]:
                 monkeypatch.setenv("SMILESS_BB_DEPTH", str(d))
                 monkeypatch.setenv("SMILESS_BB_DEPTH_A", str(da))
+                monkeypatch.setenv("SMILESS_BB_DEPTH_M", str(dm))          # three levels when dm > 0 (C5)
                 pl = S.planner_for(p)
                 out = np.empty(space)
                 g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, n_fixed=nf, fixed_digits=fixed, cost_out=out)
@@ -949,8 +950,9 @@ def test_bench_full_space_seed_cap_same_opt(monkeypatch, name):
 
 @pytest.mark.parametrize("listcap", ["0", "1", "5"])
 def test_branch_and_bound_shards_and_list_splits_are_exact(listcap, monkeypatch):
-    """Every (D, DA) pair, 2 and 3 shards, and a forced small survivor-list capacity (a
-    shallow survivor's children then span several deep launches): the shards' merged
+    """Every (D, DA) pair, with and without a middle level DM (three-level B&B), 2 and 3
+    shards, and a forced small survivor-list capacity (a survivor's children then span
+    several launches): the shards' merged
     per-candidate costs equal the oracle's, each candidate is decided by exactly one shard,
     and the best shard winner is the oracle's OPT."""
     if listcap != "0":
@@ -969,11 +971,13 @@ def test_branch_and_bound_shards_and_list_splits_are_exact(listcap, monkeypatch)
         o = OracleProblem(p)
         oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
         ref = o.plan()
-        for d in range(2, n):
-            for da in [0] + list(range(1, d)):
+        for d, da, dm in [(d, da, dm) for d in range(2, n) for da in [0] + list(range(1, d))
+                          for dm in [0] + ([da + 1] if 0 < da and da + 1 < d else [])]:
                 monkeypatch.setenv("SMILESS_BB_DEPTH", str(d))
                 monkeypatch.setenv("SMILESS_BB_DEPTH_A", str(da))
+                monkeypatch.setenv("SMILESS_BB_DEPTH_M", str(dm))
                 pl = S.planner_for(p)
+                assert ("#define SM_DM %d" % dm) in pl.kernel_source(p.arrivals_us, p.sla_us, p.windows_us)
                 for world in (2, 3):
                     merged = np.full(space, np.nan)
                     parts = []
@@ -1194,11 +1198,12 @@ def test_scale_out_branch_and_bound_and_shards(lring, monkeypatch):
         oc, ol, of = o.evaluate(np.arange(space, dtype=np.uint64))
         ref = o.plan()
         for d in range(2, n):
-            for da in (0, 1):
-                if da >= d:
+            for da, dm in ((0, 0), (1, 0), (1, 2)):
+                if da >= d or dm >= d:
                     continue
                 monkeypatch.setenv("SMILESS_BB_DEPTH", str(d))
                 monkeypatch.setenv("SMILESS_BB_DEPTH_A", str(da))
+                monkeypatch.setenv("SMILESS_BB_DEPTH_M", str(dm))
                 pl = S.planner_for(p)
                 out = np.empty(space)
                 g = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, cost_out=out, instances=inst)
