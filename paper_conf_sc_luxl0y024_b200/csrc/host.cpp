@@ -710,10 +710,11 @@ int bb_depth_a(const smiless_ctx *ctx, const smiless_plan_args *a, int D) {
     return best;
 }
 
-// Middle B&B level (three-level scheme): when every shallow survivor has more than 2^16 deep
+// Middle B&B level (three-level scheme): when every shallow survivor has more than 2^20 deep
 // children, a level at DM = DA + ceil((D - DA) / 2) prunes them first, so the deep level only
 // enumerates the children of middle survivors (C5: 2^28 deep children per shallow survivor
-// become 2 x 2^14).  0: none.  SMILESS_BB_DEPTH_M overrides (0 disables).
+// become 2 x 2^14; C5 437 -> 57 ms, C5s 232 -> 51 ms; C3's 2^19.8 measured 12 -> 14 ms with it,
+// so it stays at two levels; profiles/r02n_bb3.md).  0: none.  SMILESS_BB_DEPTH_M overrides.
 int bb_depth_m(const smiless_ctx *ctx, const smiless_plan_args *a, int D, int DA) {
     if (D <= 0 || DA <= 0) return 0;
     const char *env = getenv("SMILESS_BB_DEPTH_M");
@@ -724,7 +725,7 @@ int bb_depth_m(const smiless_ctx *ctx, const smiless_plan_args *a, int D, int DA
     if (D - DA < 2) return 0;
     unsigned __int128 r = 1;
     for (int k = DA; k < D; ++k) r *= (u64)ctx->M[k] * (u64)a->n_windows;
-    if (r <= ((unsigned __int128)1 << 16)) return 0;
+    if (r <= ((unsigned __int128)1 << 20)) return 0;
     return DA + (D - DA + 1) / 2;
 }
 
