@@ -539,7 +539,7 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_sc_luxl0y024_b200 import smiless as S
-    from paper_conf_sc_luxl0y024_b200.dist import reduce_best
+    from paper_conf_sc_luxl0y024_b200.dist import reduce_best, union_index as dist_union_index
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -573,7 +573,9 @@ def main():
     def union_index(r):
         # index in the function-0-pinned space (function 1's digit is the rank's slice), so
         # the lowest-index tie-break is the same for every world size
-        return None if not r.feasible else (kw["fixed_digits"][1] * slice_size + r.index if weak else r.index)
+        if not (weak and r.feasible):
+            return r.index
+        return dist_union_index(kw["fixed_digits"][1], slice_size, r.index)
 
     def step(arrivals):
         r = pl.plan(arrivals, p.sla_us, p.windows_us, **plan_kw)

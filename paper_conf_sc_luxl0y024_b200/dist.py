@@ -57,6 +57,14 @@ def reduce_best(local_cost: Optional[float], local_index: Optional[int], local_l
     return bits_cost(best_bits), best_index, lat, dec
 
 
+def union_index(pinned_digit: int, slice_size: int, index: Optional[int]) -> Optional[int]:
+    """Index of a slice's candidate in the space with one digit fewer pinned: weak scaling gives
+    every rank its own slice (the last pinned digit differs per rank), and the winner of the
+    union is the lexicographic (cost, union index) minimum, the same tie-break as one plan over
+    the union."""
+    return None if index is None else int(pinned_digit) * int(slice_size) + int(index)
+
+
 def plan_distributed(planner, arrivals, sla_us, windows_us, group=None, device=None, **kw):
     """Plan this rank's shard through the C ABI and reduce across ranks.
 

@@ -336,3 +336,59 @@ def test_digits_sharded_with_global_cost_cap(world, zero_prices):
         assert dec >= 4096 // (2 * world)
         assert bits_cost(keys[0]) == ref_cost and keys[1] * 256 + keys[2] == ref_idx and pay[0] == ref_lat
         assert all(cp is None or cp >= ref_cost for cp in caps)
+
+
+def _weak_worker(rank, world, port, zero_prices, out_q):
+    """Weak scaling as bench.py runs it: rank r plans its own slice of C1 (function 0 pinned to
+    digit 5, function 1 to digit 15 - r); the winners are reduced with their indices in the
+    function-0-pinned space (dist.union_index)."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import workloads as W
+    from oracle import OracleProblem
+    from paper_conf_sc_luxl0y024_b200.dist import union_index
+    p = W.make_config("C1", n_arrivals=40)
+    if zero_prices:                       # every feasible candidate ties: the lowest union index wins
+        p = p.replace(price_per_us=np.zeros_like(p.price_per_us))
+    o = OracleProblem(p, n_fixed=2, fixed_digits=[5, 15 - rank])
+    ref = o.plan()
+    gi = union_index(15 - rank, o.space_size(), ref[0] if ref else None)
+    r = reduce_best(ref[1] if ref else None, gi, ref[2] if ref else -1, o.space_size(), "cpu")
+    out_q.put((rank, r))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,zero_prices", [(2, False), (3, False), (3, True)])
+def test_weak_scaling_union_of_slices(world, zero_prices):
+    """The bench's weak-scaled step: the reduced winner of the per-rank slices equals one oracle
+    plan over the union of the slices (function 0 pinned, function 1 on the ranks' digits),
+    with the lowest-index tie-break, and the decided counts sum to the union's size."""
+    import workloads as W
+    from oracle import OracleProblem
+    p = W.make_config("C1", n_arrivals=40)
+    if zero_prices:
+        p = p.replace(price_per_us=np.zeros_like(p.price_per_us))
+    o1 = OracleProblem(p, n_fixed=1, fixed_digits=[5])
+    S = OracleProblem(p, n_fixed=2, fixed_digits=[5, 15]).space_size()
+    best = None
+    for r in range(world):                # the union: function 1's digits 15, 14, ...
+        d1 = 15 - r
+        ref = o1.plan(begin=d1 * S, end=(d1 + 1) * S)
+        if ref and (best is None or (ref[1], ref[0]) < (best[1], best[0])):
+            best = ref
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_weak_worker, args=(r, world, port, zero_prices, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    out = dict(q.get(timeout=180) for _ in range(world))
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    for r in range(world):
+        cost, idx, lat, dec = out[r]
+        assert (idx, cost, lat) == (best if best else (None, None, -1))
+        assert dec == world * S
