@@ -207,6 +207,24 @@ def test_fused_memo_kernel_compiles_for_the_bench_slice(monkeypatch):
     assert any(t.startswith("LDS.128") for t in body) and not any(t.startswith("LDG") for t in body)
 
 
+def test_branch_and_bound_levels_per_config():
+    """B&B depths the library picks for the exact full-space plans: three levels (a middle
+    level) only where a shallow survivor would have more than 2^20 deep children (C5 with
+    function 0 pinned: D = 8, DA = 4, DM = 6), two levels on C2 and C3."""
+    expect = {"C2": (4, 3, 0), "C3": (6, 3, 0), "C5": (8, 4, 6)}
+    for name, (d, da, dm) in expect.items():
+        p = W.make_config(name, n_arrivals=100)
+        pl = S.planner_for(p)
+        nf = 1 if name == "C5" else 0
+        kw = dict(n_fixed=nf, fixed_digits=[96] * nf)
+        if p.instances is not None:
+            kw["instances"] = list(p.instances)
+        src = pl.kernel_source(p.arrivals_us, p.sla_us, p.windows_us, **kw)
+        got = tuple(int(re.search(r"#define %s (\d+)" % m, src).group(1)) for m in ("SM_D", "SM_DA", "SM_DM"))
+        assert got == (d, da, dm), (name, got)
+        assert ("smiless_bound_kernel_m" in src) and (dm == 0 or "#define SM_DM 6" in src)
+
+
 def test_int64_path_selected_when_int32_range_fails():
     p = W.make_config("C1", n_arrivals=20)
     p = p.replace(windows_us=np.array([0, (1 << 29) - 1], np.int32), init_us=np.full_like(p.init_us, (1 << 29) - 1))
