@@ -153,14 +153,16 @@ class ClockSampler:
 
 
 def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier, sla=None):
-    """Exact OPT of a whole BASELINE config space with pruning + two-level B&B, sharded over
+    """Exact OPT of a whole BASELINE config space with pruning + multi-level B&B, sharded over
     the ranks (C2 / C3: interleaved prefix batches of one plan; C5, 2^70 candidates: the 128
-    values of function 0's digit, each a 2^63-candidate plan, round-robin over the ranks),
-    reduced lexicographically on (cost bits, digit, index) across ranks."""
+    values of function 0's digit, each a 2^63-candidate plan, planned in blocks of digits per
+    smiless_plan_digits call on every rank's interleaved shard), reduced lexicographically on
+    (cost bits, digit, index) across ranks."""
     import torch
     import torch.distributed as dist
     from paper_conf_sc_luxl0y024_b200.dist import (cost_bits, bits_cost, reduce_lex, plan_pinned_rounds,
-                                                   plan_range_rounds, plan_digits_sharded, INF_BITS)
+                                                   plan_range_rounds, plan_digits_sharded,
+                                                   plan_digit_blocks_sharded, INF_BITS)
     rounds = int(os.environ.get("SMILESS_BENCH_ROUNDS", "1" if world == 1 else "2"))
     p = W.make_config(name)
     if sla is not None:
@@ -193,10 +195,20 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier, sla=
         cap0 = bits_cost(int(cb.item())) if int(cb.item()) != INF_BITS else None
         seed_ms = (time.perf_counter() - ts) * 1e3
     if pinned:
-        # every rank plans every function-0 digit on its interleaved shard, incumbent exchanged
-        # after each digit (a heavy digit is split across the GPUs); SMILESS_BENCH_DIGITS=rr
-        # deals whole digits round-robin instead (dist.plan_pinned_rounds)
-        if os.environ.get("SMILESS_BENCH_DIGITS", "sharded") == "rr":
+        # every rank plans every function-0 digit on its interleaved shard (a heavy digit is split
+        # across the GPUs), a block of digits per smiless_plan_digits call (incumbent carried on
+        # the device inside a block, exchanged across ranks after each block: one block on one
+        # GPU, 16 digits with N > 1); SMILESS_BENCH_DIGITS=sharded plans one digit per call,
+        # =rr deals whole digits round-robin (dist.plan_pinned_rounds)
+        scheme = os.environ.get("SMILESS_BENCH_DIGITS", "blocks")
+        if scheme == "blocks":
+            block = int(os.environ.get("SMILESS_BENCH_DIGIT_BLOCK", "0")) or (len(digits) if world == 1 else 16)
+            best, decided, full_evals, _ = plan_digit_blocks_sharded(
+                lambda d_lo, d_hi, cap: pl.plan_digits(arr, p.sla_us, p.windows_us, d_lo, d_hi, n_fixed=1,
+                                                       fixed_digits=[0], shard=rank, n_shards=world,
+                                                       **({"cost_cap": cap} if cap is not None else {})),
+                digits[0], digits[-1] + 1, block, rank, world, xdev, initial_cap=cap0)
+        elif scheme == "rr":
             best, decided, full_evals, _ = plan_pinned_rounds(
                 lambda d0, cap: pl.plan(arr, p.sla_us, p.windows_us, n_fixed=1, fixed_digits=[d0],
                                         **({"cost_cap": cap} if cap is not None else {})),
@@ -245,7 +257,7 @@ def full_space_opt(name, S, rank, world, dev, xdev, stream, local, barrier, sla=
     cost = bits_cost(keys[0])
     out = {"candidates": decided, "time_to_optimal_s": sec, "wall_s": wall, "decided_per_s": decided / sec,
            "sla_us": p.sla_us, "instances": None if p.instances is None else p.instances.tolist(),
-           "full_evals_local": full_evals, "digits": ("rr" if os.environ.get("SMILESS_BENCH_DIGITS") == "rr" else "sharded") if pinned else None, "decided_per_rank": per_rank, "full_evals_per_rank": per_rank_full,
+           "full_evals_local": full_evals, "digits": os.environ.get("SMILESS_BENCH_DIGITS", "blocks") if pinned else None, "decided_per_rank": per_rank, "full_evals_per_rank": per_rank_full,
            "rounds": 1 if pinned else rounds,
            "cost": cost, "max_latency_us": lat if cost is not None else -1,
            "seed_cap": {"enabled": seed, "cap": cap0, "wall_ms": seed_ms}}

@@ -176,7 +176,8 @@ typedef struct {
     uint64_t d2h_bytes;       /* device -> host bytes this call copied (result block, counts,
                                  cost_out)                                                         */
     int32_t eval_path;        /* which evaluator path decided the range: SMILESS_PATH_*            */
-    int32_t reserved;         /* 0                                                                 */
+    uint32_t n_decided_hi;    /* bits 64..95 of the decided count (smiless_plan_digits: a range of
+                                 digits can hold more than 2^64 candidates, C5: 2^70); else 0     */
 } smiless_plan_result;
 
 /* smiless_plan_result.eval_path */
@@ -202,6 +203,21 @@ SMILESS_API int smiless_space_size(const smiless_ctx *ctx, int32_t n_windows, in
  * max_latency = -1, outputs set to -1), or an error. */
 SMILESS_API int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_result *res,
                  int32_t *config_out, int32_t *window_out);
+
+/* Exhaustive search over several sub-spaces in one call: every value d in [d_begin, d_end) of
+ * the LAST pinned digit (a->fixed_digits[a->n_fixed - 1] is ignored), each over [begin, end) of
+ * its suffix space, one after the other on the device with the running incumbent carried from
+ * one digit to the next (its cost bound prunes the later digits), and one exact re-check of the
+ * winner.  This is how spaces above 2^63 are planned (C5: 2^70 = 128 digits x 2^63) without a
+ * host round trip per digit.  Result: the lexicographic (cost, digit, index) minimum: res->index
+ * is its index in digit *digit_out's suffix space; n_decided + 2^64 n_decided_hi sums every
+ * digit.  Requires 1 <= n_fixed < n_funcs, fixed_digits, 0 <= d_begin < d_end <= M * W of
+ * function n_fixed - 1, and no cost_out.  Sharding (shard, n_shards) and FLAG_COST_CAP apply
+ * to every digit as in smiless_plan.  digit_out (or NULL) gets -1 when nothing is feasible.
+ * Returns OK, INFEASIBLE or an error. */
+SMILESS_API int smiless_plan_digits(smiless_ctx *ctx, const smiless_plan_args *a, int32_t d_begin, int32_t d_end,
+                                    smiless_plan_result *res, int32_t *digit_out, int32_t *config_out,
+                                    int32_t *window_out);
 
 /* The paper's adaptive pre-warming window per (function, config) row for a predicted
  * inter-arrival time it_us: Case I (T + I < IT): IT - T - I, the unloaded gap

@@ -347,6 +347,7 @@ struct smiless_ctx {
     DevBuf<u64> dList, dListA, dListM, dCostList, dListKeyA;
     DevBuf<unsigned> dCostN;
     DevBuf<unsigned> dListCnt, dListCntA, dListCntM, dChunkCnt, dChunkCntM;
+    DevBuf<ResBlock> dDig;                   // smiless_plan_digits: each digit's winner
     DevBuf<int> dW;                          // per-row windows of the current plan (padded)
     DevBuf<unsigned char> dX;                // memoised last-function inputs [n_off/4][prefix][4]
     DevBuf<i64> dRecNx, dRecNlu;             // per-prefix records (int32 or int64 time)
@@ -1316,7 +1317,7 @@ void smiless_destroy(smiless_ctx *ctx) {
         ctx->dCost.release(); ctx->dLat.release(); ctx->dFeas.release(); ctx->dRes.release(); ctx->dDump.release();
         ctx->dList.release(); ctx->dListCnt.release(); ctx->dW.release();
         ctx->dListA.release(); ctx->dListCntA.release(); ctx->dChunkCnt.release(); ctx->dListKeyA.release();
-        ctx->dListM.release(); ctx->dListCntM.release(); ctx->dChunkCntM.release();
+        ctx->dListM.release(); ctx->dListCntM.release(); ctx->dChunkCntM.release(); ctx->dDig.release();
         ctx->dCostList.release(); ctx->dCostN.release();
         ctx->dX.release(); ctx->dRecNx.release(); ctx->dRecNlu.release(); ctx->dRecPre.release();
         if (ctx->hRes) cudaFreeHost(ctx->hRes);
@@ -1526,8 +1527,13 @@ struct HostProf {
 
 // The hot path.  n_sla = 1: an ordinary plan with a->sla_us.  n_sla > 1: one evaluation of the
 // space, one argmin key per SLA in slas[] (pruning against their maximum); a->sla_us is ignored.
+// d_end > d_begin (smiless_plan_digits): plan the sub-spaces of every value d in [d_begin, d_end) of
+// the last pinned digit one after the other inside this call -- arrivals, tables and the kernel
+// staged once, the incumbent kept on the device from one digit to the next, each digit's winner
+// reduced into its own slot, one exact re-check of the overall (cost, digit, index) minimum.
 int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, int n_sla, smiless_plan_result *res,
-              int32_t *config_out, int32_t *window_out) {
+              int32_t *config_out, int32_t *window_out, int32_t d_begin = 0, int32_t d_end = 0,
+              int32_t *digit_out = nullptr) {
     if (!a_in) return fail(ctx, SMILESS_EINVAL, "args is NULL");
     HostProf hp;
     NvtxRange nv_plan("smiless_plan");
@@ -1537,6 +1543,20 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     for (int s_ = 1; s_ < n_sla; ++s_) sla_max = std::max<i64>(sla_max, slas[s_]);
     a_copy.sla_us = sla_max;
     const smiless_plan_args *a = &a_copy;
+    const bool digit_mode = d_end > d_begin;
+    int32_t fixed_local[SMILESS_MAX_FUNCS] = {0};
+    if (digit_mode) {
+        if (n_sla != 1) return fail(ctx, SMILESS_EINVAL, "digit ranges take one SLA");
+        if (a->n_fixed < 1 || a->n_fixed >= ctx->N || !a->fixed_digits)
+            return fail(ctx, SMILESS_EINVAL, "digit ranges need 1 <= n_fixed < n_funcs and fixed_digits");
+        if (a->cost_out) return fail(ctx, SMILESS_EINVAL, "cost_out is not supported with digit ranges");
+        const int32_t radix = ctx->M[a->n_fixed - 1] * a->n_windows;
+        if (d_begin < 0 || d_end > radix)
+            return fail(ctx, SMILESS_EINVAL, "digit range [%d, %d) outside [0, %d)", d_begin, d_end, radix);
+        for (int k = 0; k < a->n_fixed; ++k) fixed_local[k] = a->fixed_digits[k];
+        fixed_local[a->n_fixed - 1] = d_begin;
+        a_copy.fixed_digits = fixed_local;
+    }
     int rc = validate_args(ctx, a, true);
     if (rc) return rc;
     for (int s_ = 0; s_ < n_sla; ++s_)
@@ -1583,6 +1603,8 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     }
 
     const bool single = a->n_fixed == ctx->N;    // nothing left to search: one candidate
+    u64 digit_dec_lo = 0, digit_dec_hi = 0, digit_full = 0;
+    int32_t digit_best = -1;
     double eval_ms = 0.0;
     u64 n_decided = 0, n_full = 0;
     if (!single && ce > cb) {
@@ -1602,6 +1624,10 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             if ((rc = get_kernel(ctx, a, rp, n_off, families, &jk))) return rc;
         }
         hp.mark("get_kernel");
+        // one evaluation of [cb, ce) for the current pinned digits, its winner reduced into dst;
+        // `first`: the first (or only) digit uploads the caller's cap as the incumbent and starts
+        // the evaluator's event
+        auto run_once = [&](ResBlock *dst, const bool first) -> int {
         const u64 V = unit_cands(ctx, a);   // candidates per unit
         const u64 ub = cb / V, ue = (ce + V - 1) / V;
         const u64 U = ue - ub;
@@ -1648,8 +1674,10 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 double c = a->cost_cap + 0.0;               // -0.0 -> +0.0: bits order like the costs
                 memcpy(&pp.cap, &c, 8);
             }
-            CK(cudaMemcpyAsync(ctx->dInc.p, &pp.cap, 8, cudaMemcpyHostToDevice, st), "H2D incumbent");
-            ctx->h2d += 8;
+            if (first) {                                   // later digits keep the running incumbent
+                CK(cudaMemcpyAsync(ctx->dInc.p, &pp.cap, 8, cudaMemcpyHostToDevice, st), "H2D incumbent");
+                ctx->h2d += 8;
+            }
         }
         pp.shard = shard;
         pp.n_shards = n_shards;
@@ -1723,7 +1751,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             pc.list_base = 0;
             pc.list_in_cap = batch_p * upp;
             pc.no_count = 1;
-            CK(cudaEventRecord(ctx->ev[1], st), "event");
+            if (first) CK(cudaEventRecord(ctx->ev[1], st), "event");
             NvtxRange nv("memo: fused producer/consumer batches");
             for (u64 b0 = pl0; b0 < ph0; b0 += batch_p) {
                 const u64 b1 = std::min(ph0, b0 + batch_p);
@@ -1812,7 +1840,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid_var * 16 * n_sla, st), "memset");
                 mp.blk_best = ctx->dBlk.p;
             }
-            CK(cudaEventRecord(ctx->ev[1], st), "event");
+            if (first) CK(cudaEventRecord(ctx->ev[1], st), "event");
             NvtxRange nv("memo: upstream + variants batches");
             u64 bi = 0;
             for (u64 b0 = pl0; b0 < ph0; b0 += batch_p, ++bi) {
@@ -1899,7 +1927,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             }
             for (int k = 0; k < a->n_fixed; ++k) bp.fixed[k] = a->fixed_digits[k];
             const int grid_b = jk->blocks_bound * ctx->n_sms;
-            CK(cudaEventRecord(ctx->ev[1], st), "event");
+            if (first) CK(cudaEventRecord(ctx->ev[1], st), "event");
             // evaluator over the deep survivors in dList (absolute depth-D prefix ids)
             auto run_eval = [&]() -> int {
                 CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
@@ -2130,7 +2158,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 CK(ctx->dList.ensure((size_t)claims_per_launch), "cudaMalloc list");
                 CK(ctx->dListCnt.ensure(1), "cudaMalloc");
             }
-            CK(cudaEventRecord(ctx->ev[1], st), "event");
+            if (first) CK(cudaEventRecord(ctx->ev[1], st), "event");
             NvtxRange nv("evaluate");
             for (u64 q0 = 0; q0 < claims_total; q0 += claims_per_launch) {
                 const u64 q1 = std::min(claims_total, q0 + claims_per_launch);
@@ -2171,19 +2199,55 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                 }
             }
         }
-        CK(cudaEventRecord(ctx->ev[2], st), "event");
         NvtxRange nv("argmin reduce");
         for (int s_ = 0; s_ < n_sla; ++s_) {
-            e = smiless_dev_reduce_best(ctx->dBlk.p + 2 * s_, grid_used, n_sla, ctx->dRes.p + s_, st);
-            if (e) return cuda_fail(ctx, (cudaError_t)e, "reduce launch");
+            int e2 = smiless_dev_reduce_best(ctx->dBlk.p + 2 * s_, grid_used, n_sla, dst + s_, st);
+            if (e2) return cuda_fail(ctx, (cudaError_t)e2, "reduce launch");
             ++launches;
         }
-        CK(cudaMemcpyAsync(&ctx->dRes.p->stats[0], ctx->dStats.p, 16, cudaMemcpyDeviceToDevice, st), "D2D stats");
+        CK(cudaMemcpyAsync(&dst->stats[0], ctx->dStats.p, 16, cudaMemcpyDeviceToDevice, st), "D2D stats");
         if (a->cost_out) {
             ctx->d2h += (size_t)(ce - cb) * sizeof(double);
             CK(cudaMemcpyAsync(a->cost_out, ctx->dDump.p, (size_t)(ce - cb) * sizeof(double), cudaMemcpyDeviceToHost, st),
                "D2H dump");
         }
+        return SMILESS_OK;
+        };
+        if (!digit_mode) {
+            if ((rc = run_once(ctx->dRes.p, true))) return rc;
+        } else {
+            const int n_dig = d_end - d_begin;
+            CK(ctx->dDig.ensure((size_t)n_dig), "cudaMalloc digit results");
+            for (int d = d_begin; d < d_end; ++d) {
+                fixed_local[a->n_fixed - 1] = d;
+                if ((rc = run_once(ctx->dDig.p + (d - d_begin), d == d_begin))) return rc;
+            }
+            // the lexicographic (cost bits, digit, index) minimum over the digits' winners; the
+            // decided counts summed in 128 bits (C5: 128 digits x 2^63 candidates)
+            std::vector<ResBlock> hd((size_t)n_dig);
+            CK(cudaMemcpyAsync(hd.data(), ctx->dDig.p, sizeof(ResBlock) * (size_t)n_dig, cudaMemcpyDeviceToHost, st),
+               "D2H digit results");
+            ctx->d2h += sizeof(ResBlock) * (size_t)n_dig;
+            CK(cudaStreamSynchronize(st), "digits");
+            int best_d = -1;
+            unsigned __int128 dec = 0;
+            u64 full = 0;
+            for (int i = 0; i < n_dig; ++i) {
+                dec += hd[i].stats[0];
+                full += hd[i].stats[1];
+                if (hd[i].best_i == ~0ull) continue;
+                if (best_d < 0 || hd[i].best_c < hd[best_d].best_c) best_d = i;   // ties: the lower digit
+            }
+            digit_dec_lo = (u64)dec;
+            digit_dec_hi = (u64)(dec >> 64);
+            digit_full = full;
+            digit_best = best_d < 0 ? -1 : d_begin + best_d;
+            fixed_local[a->n_fixed - 1] = best_d < 0 ? d_begin : d_begin + best_d;
+            const u64 win[2] = {best_d < 0 ? ~0ull : hd[best_d].best_c, best_d < 0 ? ~0ull : hd[best_d].best_i};
+            CK(cudaMemcpyAsync(&ctx->dRes.p->best_c, win, 16, cudaMemcpyHostToDevice, st), "H2D winner");
+            ctx->h2d += 16;
+        }
+        CK(cudaEventRecord(ctx->ev[2], st), "event");
     } else if (single && ce > cb) {
         // the space is the single candidate of the pinned digits: index 0
         for (int s_ = 0; s_ < n_sla; ++s_) CK(cudaMemsetAsync(&ctx->dRes.p[s_].best_c, 0, 16, st), "memset");
@@ -2223,8 +2287,8 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
     if (h0.err & 2) return fail(ctx, SMILESS_EINVAL, "arrival times out of range (|r| >= 2^62)");
     if (h0.err & 4) return fail(ctx, SMILESS_ECUDA, "internal: branch-and-bound survivor list overflow");
     if (!single && ce > cb) {
-        n_decided = h0.stats[0];
-        n_full = h0.stats[1];
+        n_decided = digit_mode ? digit_dec_lo : h0.stats[0];
+        n_full = digit_mode ? digit_full : h0.stats[1];
     } else if (single && ce > cb) {
         n_decided = n_full = 1;
     }
@@ -2254,6 +2318,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         r.h2d_bytes = ctx->h2d;
         r.d2h_bytes = ctx->d2h;
         r.eval_path = eval_path;
+        r.n_decided_hi = digit_mode ? (uint32_t)digit_dec_hi : 0u;
         int32_t *co = config_out ? config_out + (size_t)s_ * ctx->N : nullptr;
         int32_t *wo = window_out ? window_out + (size_t)s_ * ctx->N : nullptr;
         if (!found) {
@@ -2267,6 +2332,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
             continue;
         }
         if (s_ == 0) status = SMILESS_OK;
+        if (digit_out) *digit_out = digit_mode ? digit_best : -1;
         r.index = h.best_i;
         r.cost = h.cost;
         r.max_latency_us = h.maxlat;
@@ -2290,6 +2356,18 @@ int smiless_plan(smiless_ctx *ctx, const smiless_plan_args *a, smiless_plan_resu
     if (!a) return fail(ctx, SMILESS_EINVAL, "args is NULL");
     const i64 sla = a->sla_us;
     return plan_impl(ctx, a, &sla, 1, res, config_out, window_out);
+}
+
+int smiless_plan_digits(smiless_ctx *ctx, const smiless_plan_args *a, int32_t d_begin, int32_t d_end,
+                        smiless_plan_result *res, int32_t *digit_out, int32_t *config_out, int32_t *window_out) {
+    if (!ctx) return SMILESS_EINVAL;
+    ctx->err.clear();
+    if (!res) return fail(ctx, SMILESS_EINVAL, "res is NULL");
+    if (!a) return fail(ctx, SMILESS_EINVAL, "args is NULL");
+    if (d_end <= d_begin) return fail(ctx, SMILESS_EINVAL, "empty digit range [%d, %d)", d_begin, d_end);
+    if (digit_out) *digit_out = -1;
+    const i64 sla = a->sla_us;
+    return plan_impl(ctx, a, &sla, 1, res, config_out, window_out, d_begin, d_end, digit_out);
 }
 
 int smiless_derive_windows(const smiless_ctx *ctx, int64_t it_us, int32_t *row_windows_out) {

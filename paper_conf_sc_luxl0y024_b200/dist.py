@@ -201,6 +201,34 @@ def plan_digits_sharded(plan_digit, digits, rank, world, device, group=None, ini
     return best, decided, full_evals, caps
 
 
+def plan_digit_blocks_sharded(plan_block, d_begin, d_end, block, rank, world, device, group=None, initial_cap=None):
+    """plan_digits_sharded with blocks of consecutive digits per library call:
+    plan_block(d_lo, d_hi, cap) plans digits d_lo .. d_hi - 1 on this rank's interleaved shard in
+    one smiless_plan_digits call (the incumbent carried on the device inside the block) and
+    returns a result with .digit; the ranks MIN-all-reduce their cheapest feasible cost after
+    every block.  One GPU: one block of all digits, no host round trip per digit.
+
+    Returns (best, decided, full_evals, caps) like plan_digits_sharded."""
+    best, decided, full_evals, caps = None, 0, 0, []
+    cap_bits = cost_bits(initial_cap) if initial_cap is not None else INF_BITS
+    for lo in range(d_begin, d_end, block):
+        hi = min(d_end, lo + block)
+        cap = bits_cost(cap_bits) if cap_bits != INF_BITS else None
+        caps.append(cap)
+        r = plan_block(lo, hi, cap)
+        decided += r.n_decided
+        full_evals += r.n_full_evals
+        if r.feasible and (best is None or (r.cost, r.digit, r.index) < best[:3]):
+            best = (r.cost, r.digit, r.index, r.max_latency_us)
+        if best is not None:
+            cap_bits = min(cap_bits, cost_bits(best[0]))
+        if world > 1 and hi < d_end:
+            t = torch.tensor([cap_bits], dtype=torch.int64, device=device)
+            dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+            cap_bits = int(t.item())
+    return best, decided, full_evals, caps
+
+
 def decompose_plan_distributed(planner, arrivals, sla_us, windows_us, group=None, device=None, **kw):
     """NEXT-3 with model M on N GPUs: every rank plans its interleaved share of each source-to-
     sink path (smiless_decompose_plan_sharded) and the path winners are reduced with the same

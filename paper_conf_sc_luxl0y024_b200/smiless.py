@@ -25,7 +25,7 @@ _NAMES = {0: "OK", 1: "INFEASIBLE", -1: "EINVAL", -2: "ENOTTOPO", -3: "ERANGE", 
 
 # every symbol include/smiless.h declares (checked by tests/test_abi.py)
 EXPORTS = ("smiless_create", "smiless_set_stream", "smiless_destroy", "smiless_last_error",
-           "smiless_load_dag", "smiless_load_profiles", "smiless_space_size", "smiless_plan",
+           "smiless_load_dag", "smiless_load_profiles", "smiless_space_size", "smiless_plan", "smiless_plan_digits",
            "smiless_plan_sla_sweep", "smiless_derive_windows", "smiless_top1_search", "smiless_decompose_search", "smiless_decompose_plan",
            "smiless_decompose_plan_sharded",
            "smiless_autoscale", "smiless_autoscale_rows",
@@ -75,7 +75,7 @@ class PlanResultC(ctypes.Structure):
         ("h2d_bytes", ctypes.c_uint64),
         ("d2h_bytes", ctypes.c_uint64),
         ("eval_path", ctypes.c_int32),
-        ("reserved", ctypes.c_int32),
+        ("n_decided_hi", ctypes.c_uint32),
     ]
 
 
@@ -100,6 +100,7 @@ class PlanResult:
     h2d_bytes: int = 0          # host -> device bytes the call copied (counted by the library)
     d2h_bytes: int = 0          # device -> host bytes the call copied
     eval_path: int = 0          # PATH_* (which evaluator path decided the range)
+    digit: Optional[int] = None  # plan_digits: the winner's value of the last pinned digit
 
     @property
     def feasible(self) -> bool:
@@ -130,6 +131,8 @@ def load_library(build_if_missing: bool = True):
     lib.smiless_load_profiles.argtypes = [vp, vp, vp, vp, vp]
     lib.smiless_space_size.argtypes = [vp, i32, i32, ctypes.POINTER(u64)]
     lib.smiless_plan.argtypes = [vp, ctypes.POINTER(PlanArgs), ctypes.POINTER(PlanResultC), vp, vp]
+    lib.smiless_plan_digits.argtypes = [vp, ctypes.POINTER(PlanArgs), i32, i32, ctypes.POINTER(PlanResultC),
+                                        ctypes.POINTER(ctypes.c_int32), vp, vp]
     lib.smiless_plan_sla_sweep.argtypes = [vp, ctypes.POINTER(PlanArgs), vp, i32, ctypes.POINTER(PlanResultC),
                                            vp, vp]
     lib.smiless_derive_windows.argtypes = [vp, i64, vp]
@@ -307,6 +310,28 @@ class Planner:
                           eval_kernel_ms=float(r.eval_kernel_ms), total_device_ms=float(r.total_device_ms),
                           int64_path=bool(r.int64_path), launches=int(r.launches),
                           h2d_bytes=int(r.h2d_bytes), d2h_bytes=int(r.d2h_bytes), eval_path=int(r.eval_path))
+
+    def plan_digits(self, arrivals, sla_us, windows_us, d_begin: int, d_end: int, **kw) -> PlanResult:
+        """Every value of the last pinned digit in [d_begin, d_end), one after the other in one
+        call with the incumbent carried on the device (smiless_plan_digits).  kw as plan();
+        n_fixed >= 1 and fixed_digits required (the last one is ignored).  n_decided sums all
+        digits (it may exceed 2^64); .digit is the winner's digit."""
+        a, keep = self._args(arrivals, sla_us, windows_us, **kw)
+        r = PlanResultC()
+        dg = ctypes.c_int32(-1)
+        cfg = np.zeros(max(self.n_funcs, 1), np.int32)
+        win = np.zeros(max(self.n_funcs, 1), np.int32)
+        rc = self._check(self._lib.smiless_plan_digits(self._ctx, ctypes.byref(a), int(d_begin), int(d_end),
+                                                       ctypes.byref(r), ctypes.byref(dg), cfg.ctypes.data,
+                                                       win.ctypes.data), allow=(OK, INFEASIBLE))
+        del keep
+        return PlanResult(status=rc, index=None if rc == INFEASIBLE else int(r.index), cost=float(r.cost),
+                          max_latency_us=int(r.max_latency_us), config=cfg[:self.n_funcs],
+                          window=win[:self.n_funcs], n_decided=int(r.n_decided) + (int(r.n_decided_hi) << 64),
+                          n_full_evals=int(r.n_full_evals), eval_kernel_ms=float(r.eval_kernel_ms),
+                          total_device_ms=float(r.total_device_ms), int64_path=bool(r.int64_path),
+                          launches=int(r.launches), h2d_bytes=int(r.h2d_bytes), d2h_bytes=int(r.d2h_bytes),
+                          eval_path=int(r.eval_path), digit=None if rc == INFEASIBLE else int(dg.value))
 
     def plan_sla_sweep(self, arrivals, slas_us, windows_us, **kw):
         """One pass over the space, one winner per SLA (smiless_plan_sla_sweep)."""

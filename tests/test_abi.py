@@ -130,6 +130,28 @@ def test_plan_argument_validation_before_any_gpu_work():
         assert e.value.code == code, over
 
 
+def test_plan_digits_argument_validation_before_any_gpu_work():
+    """smiless_plan_digits rejects bad digit ranges and unsupported options before touching the
+    device (works without a GPU)."""
+    p = W.make_config("C1", n_arrivals=20)
+    pl = S.planner_for(p)
+    args = (p.arrivals_us, p.sla_us, p.windows_us)
+    Wn = len(p.windows_us)
+    bad = [
+        ((0, 0), dict(n_fixed=1, fixed_digits=[0])),                          # empty range
+        ((3, 2), dict(n_fixed=1, fixed_digits=[0])),
+        ((0, 4), dict(n_fixed=0)),                                             # no pinned digit
+        ((0, 4 * Wn + 1), dict(n_fixed=1, fixed_digits=[0])),                  # beyond the radix
+        ((-1, 2), dict(n_fixed=1, fixed_digits=[0])),
+        ((0, 2), dict(n_fixed=3, fixed_digits=[0, 0, 0])),                     # nothing left to search
+        ((0, 2), dict(n_fixed=1, fixed_digits=[0], cost_out=np.empty(256))),   # no per-candidate dump
+    ]
+    for (d0, d1), kw in bad:
+        with pytest.raises(S.SmilessError) as e:
+            pl.plan_digits(*args, d0, d1, **kw)
+        assert e.value.code == S.EINVAL, (d0, d1, kw)
+
+
 def test_negative_zero_price_rejected():
     """-0.0 would give cost bits with the sign set: rejected like a negative price."""
     pl = S.Planner(device=0)

@@ -276,7 +276,7 @@ def test_range_rounds_with_in_plan_incumbent_exchange(world, rounds, zero_prices
             assert caps[-1] is not None       # the global incumbent reached every rank's last round
 
 
-def _digits_sharded_worker(rank, world, port, zero_prices, out_q):
+def _digits_sharded_worker(rank, world, port, zero_prices, out_q, block=0):
     """C1 as 16 function-0 digits, EVERY rank planning every digit on its interleaved shard
     (emulated on the oracle's per-candidate costs with the library's semantics), the
     incumbent exchanged after each digit."""
@@ -285,7 +285,7 @@ def _digits_sharded_worker(rank, world, port, zero_prices, out_q):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     import workloads as W
     from oracle import OracleProblem
-    from paper_conf_sc_luxl0y024_b200.dist import plan_digits_sharded, reduce_lex
+    from paper_conf_sc_luxl0y024_b200.dist import plan_digits_sharded, plan_digit_blocks_sharded, reduce_lex
     p = W.make_config("C1", n_arrivals=40)
     if zero_prices:
         p = p.replace(price_per_us=np.zeros_like(p.price_per_us))
@@ -301,7 +301,23 @@ def _digits_sharded_worker(rank, world, port, zero_prices, out_q):
         k = s_[ok][np.lexsort((s_[ok], c[g][ok]))[0]]
         return _Res(True, float(c[d * 256 + k]), int(k), int(l[d * 256 + k]), len(s_))
 
-    best, dec, _, caps = plan_digits_sharded(plan_digit, list(range(16)), rank, world, "cpu")
+    def plan_block(lo, hi, cap):          # smiless_plan_digits: the (cost, digit, index) minimum of the block
+        rs = [(plan_digit(d, cap), d) for d in range(lo, hi)]
+        ok = [(r.cost, d, r.index, r) for r, d in rs if r.feasible]
+        n = sum(r.n_decided for r, _ in rs)
+        if not ok:
+            out = _Res(False, float("inf"), None, -1, n)
+            out.digit = None
+            return out
+        c_, d_, i_, r_ = min(ok, key=lambda t: t[:3])
+        out = _Res(True, c_, i_, r_.max_latency_us, n)
+        out.digit = d_
+        return out
+
+    if block:
+        best, dec, _, caps = plan_digit_blocks_sharded(plan_block, 0, 16, block, rank, world, "cpu")
+    else:
+        best, dec, _, caps = plan_digits_sharded(plan_digit, list(range(16)), rank, world, "cpu")
     keys = [cost_bits(best[0]) if best else INF_BITS, best[1] if best else 0, best[2] if best else 0]
     keys, pay = reduce_lex(keys, [best[3] if best else -1], "cpu")
     out_q.put((rank, (keys, pay, dec, caps)))
@@ -309,11 +325,13 @@ def _digits_sharded_worker(rank, world, port, zero_prices, out_q):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,zero_prices", [(2, False), (3, False), (2, True)])
-def test_digits_sharded_with_global_cost_cap(world, zero_prices):
-    """bench.py's C5 driver (dist.plan_digits_sharded): every rank decides its share of every
-    digit, the caps are real feasible costs, and the reduced (cost, digit, index) is the
-    oracle's OPT with the lowest-index tie-break."""
+@pytest.mark.parametrize("world,zero_prices,block", [(2, False, 0), (3, False, 0), (2, True, 0), (2, False, 4),
+                                                     (3, False, 5), (2, True, 4)])
+def test_digits_sharded_with_global_cost_cap(world, zero_prices, block):
+    """bench.py's C5 driver (dist.plan_digits_sharded, or with block > 0
+    dist.plan_digit_blocks_sharded: several digits per library call, exchange per block): every
+    rank decides its share of every digit, the caps are real feasible costs, and the reduced
+    (cost, digit, index) is the oracle's OPT with the lowest-index tie-break."""
     import workloads as W
     from oracle import OracleProblem
     p = W.make_config("C1", n_arrivals=40)
@@ -323,7 +341,8 @@ def test_digits_sharded_with_global_cost_cap(world, zero_prices):
     port = _free_port()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_digits_sharded_worker, args=(r, world, port, zero_prices, q)) for r in range(world)]
+    procs = [ctx.Process(target=_digits_sharded_worker, args=(r, world, port, zero_prices, q, block))
+             for r in range(world)]
     for pr in procs:
         pr.start()
     out = dict(q.get(timeout=180) for _ in range(world))

@@ -1391,3 +1391,76 @@ def test_arrivals_device_view_at_8_byte_offset():
     assert_same_plan(g, o.plan(), o)
     idx = np.arange(0, 4096, 13, dtype=np.uint64)
     assert_same_eval(*pl.evaluate(idx, view, p.sla_us, p.windows_us), *o.evaluate(idx))
+
+
+# ---------------------------------------------------------------------------------------
+# smiless_plan_digits: a range of values of the last pinned digit in one call
+# ---------------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("flags", [0, S.FLAG_NO_PRUNE])
+def test_plan_digits_matches_oracle_over_the_union(flags):
+    """Every value of the last pinned digit in [d0, d1), one call, the incumbent carried on the
+    device: the (cost, digit, index) minimum equals one oracle plan over the union of the digits'
+    sub-spaces (ties to the lowest digit, then index), every candidate is counted once, and the
+    shards of the call together decide the union; also with a cost cap at OPT."""
+    rng = np.random.default_rng(909 + flags)
+    n_checked = 0
+    for t in range(60):
+        n = int(rng.integers(3, 6))
+        p = W.random_problem(rng, n, 4, int(rng.integers(2, 4)), int(rng.integers(20, 150)),
+                             sla_us=int(rng.integers(15_000, 60_000)))
+        Wn = len(p.windows_us)
+        nf = int(rng.integers(1, 3))
+        fixed = [int(rng.integers(0, p.n_configs[k] * Wn)) for k in range(nf)]
+        radix = int(p.n_configs[nf - 1]) * Wn
+        o_pre = OracleProblem(p, n_fixed=nf - 1, fixed_digits=fixed[:-1])
+        S_ = OracleProblem(p, n_fixed=nf, fixed_digits=fixed).space_size()
+        if S_ * radix > 40000 or radix < 3:
+            continue
+        d0 = int(rng.integers(0, radix - 1))
+        d1 = int(rng.integers(d0 + 1, radix + 1))
+        ref = o_pre.plan(begin=d0 * S_, end=d1 * S_)
+        pl = S.planner_for(p)
+        kw = dict(n_fixed=nf, fixed_digits=fixed, flags=flags)
+        r = pl.plan_digits(p.arrivals_us, p.sla_us, p.windows_us, d0, d1, **kw)
+        assert r.n_decided == (d1 - d0) * S_
+        if ref is None:
+            assert not r.feasible and r.digit is None
+        else:
+            assert r.feasible and (r.digit * S_ + r.index, r.cost, r.max_latency_us) == ref
+            assert r.config.tolist() == o_pre.decode(ref[0])[0].tolist()
+            rc = pl.plan_digits(p.arrivals_us, p.sla_us, p.windows_us, d0, d1, cost_cap=ref[1], **dict(kw, flags=0))
+            assert (rc.digit * S_ + rc.index, rc.cost) == ref[:2]
+        parts = [pl.plan_digits(p.arrivals_us, p.sla_us, p.windows_us, d0, d1, shard=s_, n_shards=3, **kw)
+                 for s_ in range(3)]
+        assert sum(q.n_decided for q in parts) == (d1 - d0) * S_
+        win = [(q.cost, q.digit, q.index) for q in parts if q.feasible]
+        assert (min(win) if win else None) == (None if ref is None else (ref[1], ref[0] // S_, ref[0] % S_))
+        n_checked += 1
+        if n_checked == 10:
+            break
+    assert n_checked >= 6
+
+
+def test_plan_digits_c5_equals_the_per_digit_loop():
+    """C5 (2^70 candidates, scale-out) in one smiless_plan_digits call over function 0's 128
+    digits: the same OPT as planning the digits one call each with the running best as cost
+    cap, 2^70 candidates decided (beyond 2^64: n_decided_hi), and the winner re-checks on the
+    oracle."""
+    p = W.make_config("C5")
+    pl = S.planner_for(p)
+    Wn = len(p.windows_us)
+    radix = int(p.n_configs[0]) * Wn
+    r = pl.plan_digits(p.arrivals_us, p.sla_us, p.windows_us, 0, radix, n_fixed=1, fixed_digits=[0])
+    assert r.n_decided == 1 << 70
+    best = None
+    for d in range(radix):
+        kw = dict(n_fixed=1, fixed_digits=[d])
+        if best is not None:
+            kw["cost_cap"] = best[0]
+        q = pl.plan(p.arrivals_us, p.sla_us, p.windows_us, **kw)
+        if q.feasible and (best is None or (q.cost, d, q.index) < best[:3]):
+            best = (q.cost, d, q.index, q.max_latency_us)
+    assert best is not None and (r.cost, r.digit, r.index, r.max_latency_us) == best
+    c, l, f = OracleProblem(p, n_fixed=1, fixed_digits=[r.digit]).evaluate([r.index])
+    assert f[0] and c[0] == r.cost and l[0] == r.max_latency_us

@@ -23,6 +23,8 @@ def main():
     ap.add_argument("name")
     ap.add_argument("--sla", type=int, default=None)
     ap.add_argument("--limit-digits", type=int, default=0)
+    ap.add_argument("--per-digit", action="store_true",
+                    help="one smiless_plan call per function-0 digit (default: one smiless_plan_digits call)")
     args = ap.parse_args()
     import torch
     from paper_conf_sc_luxl0y024_b200 import smiless as S
@@ -48,6 +50,12 @@ def main():
         digits = list(range(int(p.n_configs[0]) * Wn))
         if args.limit_digits:
             digits = digits[:args.limit_digits]
+        if not args.per_digit:
+            r = pl.plan_digits(arr, p.sla_us, p.windows_us, digits[0], digits[-1] + 1, n_fixed=1, fixed_digits=[0])
+            decided, full, launches = r.n_decided, r.n_full_evals, r.launches
+            if r.feasible:
+                best = (r.cost, r.digit, r.index, r.max_latency_us)
+            digits = []
         for d in digits:
             td = time.perf_counter()
             kw = dict(n_fixed=1, fixed_digits=[d])
