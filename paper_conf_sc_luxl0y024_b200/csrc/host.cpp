@@ -689,8 +689,11 @@ int bb_depth(const smiless_ctx *ctx, const smiless_plan_args *a) {
     return best;
 }
 
-// Shallow B&B level (two-level scheme): the deepest depth < D with at most 2^22 prefixes, if
-// the deep level has more than 2^24 prefixes (else 0: single level).  SMILESS_BB_DEPTH_A overrides.
+// Shallow B&B level (two-level scheme): the deepest depth < D with at most 2^22 prefixes (2^16
+// for a sub-plan with pinned digits: C5's 128 function-0 digits are mostly pruned at this level,
+// and a 2^21-prefix level took 0.13 ms per digit against ~0.02 ms for 2^14; C5 44 -> 39 ms,
+// C5s 35 -> 30 ms, profiles/r02n_bb3.md), if the deep level has more than 2^24 prefixes (else 0:
+// single level).  SMILESS_BB_DEPTH_A overrides.
 int bb_depth_a(const smiless_ctx *ctx, const smiless_plan_args *a, int D) {
     if (D <= 0) return 0;
     const int nf = a->n_fixed, W = a->n_windows;
@@ -704,9 +707,10 @@ int bb_depth_a(const smiless_ctx *ctx, const smiless_plan_args *a, int D) {
     if (prefD <= ((unsigned __int128)1 << 24)) return 0;
     int best = 0;
     unsigned __int128 pref = 1;
+    const unsigned __int128 cap = (unsigned __int128)1 << (nf > 0 ? 16 : 22);
     for (int d = nf + 1; d < D; ++d) {
         pref *= (u64)ctx->M[d - 1] * (u64)W;
-        if (pref <= ((unsigned __int128)1 << 22)) best = d;
+        if (pref <= cap) best = d;
     }
     return best;
 }

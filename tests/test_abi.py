@@ -232,8 +232,9 @@ def test_fused_memo_kernel_compiles_for_the_bench_slice(monkeypatch):
 def test_branch_and_bound_levels_per_config():
     """B&B depths the library picks for the exact full-space plans: three levels (a middle
     level) only where a shallow survivor would have more than 2^20 deep children (C5 with
-    function 0 pinned: D = 8, DA = 4, DM = 6), two levels on C2 and C3."""
-    expect = {"C2": (4, 3, 0), "C3": (6, 3, 0), "C5": (8, 4, 6)}
+    function 0 pinned: D = 8, DA = 3 -- sub-plans keep the shallow level at <= 2^16 prefixes --
+    and DM = 6), two levels on C2 and C3."""
+    expect = {"C2": (4, 3, 0), "C3": (6, 3, 0), "C5": (8, 3, 6)}
     for name, (d, da, dm) in expect.items():
         p = W.make_config(name, n_arrivals=100)
         pl = S.planner_for(p)
