@@ -1028,11 +1028,16 @@ def test_full_space_plan_shards_split_the_work(name, world):
     assert min((r.cost, r.index) for r in parts if r.feasible) == (one.cost, one.index)
 
 
-def test_c5_heavy_subplan_children_split_over_launches():
-    """C5s's sub-plan of function 0's digit 112 (2^63 candidates): its shallow survivors have
-    2^28 deep children each, more than one survivor list holds, so their children run over
-    several deep launches.  Single rank and 2 shards agree; the oracle re-checks the winner."""
+@pytest.mark.parametrize("levels", ["two", "auto"])
+def test_c5_heavy_subplan_children_split_over_launches(levels, monkeypatch):
+    """C5s's sub-plan of function 0's digit 112 (2^63 candidates).  levels = two (DA = 4, no
+    middle level): its shallow survivors have 2^28 deep children each, more than one survivor
+    list holds, so their children run over several deep launches.  auto: the default three
+    levels.  Single rank and 2 shards agree; the oracle re-checks the winner."""
     import torch
+    if levels == "two":
+        monkeypatch.setenv("SMILESS_BB_DEPTH_A", "4")
+        monkeypatch.setenv("SMILESS_BB_DEPTH_M", "0")
     p = W.make_config("C5s")
     pl = S.planner_for(p)
     arr = torch.as_tensor(p.arrivals_us).cuda()
