@@ -46,6 +46,29 @@ for s_ in range(2):
 for k in ("SMILESS_BB_DEPTH", "SMILESS_BB_DEPTH_A", "SMILESS_BB_LISTCAP"):
     os.environ.pop(k)
 plq.decompose_plan(q.arrivals_us, q.sla_us, q.windows_us)
+# round 2 (later): the fused producer/consumer memo kernel (mbarrier ring; plain and with a
+# scaled-out upstream), the three-level B&B, smiless_plan_digits
+rng2 = np.random.default_rng(11)
+while True:
+    f = W.random_problem(rng2, 4, 16, 2, 200, sla_us=60_000)
+    if int(f.n_configs[-1]) >= 12:
+        break
+plf = S.planner_for(f)
+os.environ["SMILESS_G"] = "1"
+plf.plan(f.arrivals_us, f.sla_us, f.windows_us, flags=S.FLAG_NO_PRUNE)
+plf.plan(f.arrivals_us, f.sla_us, f.windows_us, flags=S.FLAG_NO_PRUNE, instances=[2, 3, 1, 1])
+os.environ["SMILESS_SPLITCOST"] = "0"
+plf.plan(f.arrivals_us, f.sla_us, f.windows_us, flags=S.FLAG_NO_PRUNE, shard=1, n_shards=2)
+os.environ.pop("SMILESS_SPLITCOST")
+os.environ.pop("SMILESS_G")
+os.environ.update(SMILESS_BB_DEPTH="4", SMILESS_BB_DEPTH_A="1", SMILESS_BB_DEPTH_M="2", SMILESS_BB_LISTCAP="5")
+q6 = W.random_problem(rng2, 6, 3, 2, 200, sla_us=40_000)
+pl6 = S.planner_for(q6)
+pl6.plan(q6.arrivals_us, q6.sla_us, q6.windows_us)
+pl6.plan(q6.arrivals_us, q6.sla_us, q6.windows_us, shard=0, n_shards=2)
+for k in ("SMILESS_BB_DEPTH", "SMILESS_BB_DEPTH_A", "SMILESS_BB_DEPTH_M", "SMILESS_BB_LISTCAP"):
+    os.environ.pop(k)
+pl6.plan_digits(q6.arrivals_us, q6.sla_us, q6.windows_us, 0, int(q6.n_configs[0]) * 2, n_fixed=1, fixed_digits=[0])
 print("sanitize workload done")
 PY
 for tool in memcheck racecheck synccheck initcheck; do
