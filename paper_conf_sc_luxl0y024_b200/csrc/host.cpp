@@ -2030,11 +2030,13 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                     }
                     // Launches over a survivor list (first entry, entries, first child, children per
                     // entry): at most list_cap ordinals each.  With the cost bound on, the first launch
-                    // is small and each next one SMILESS_BB_GROW (4) times larger: every launch's
+                    // is small and each next one SMILESS_BB_GROW (256) times larger: every launch's
                     // static prefix bound prunes against the incumbent the evaluations before it set,
-                    // so the incumbent is refined early instead of once (C2 at SLA 8 s: 131,072-entry
-                    // chunks after a 64-entry first one took 95-406 ms depending on which survivors
-                    // came first).  A survivor with more than list_cap children spans several.
+                    // so the incumbent is refined before the bulk of the list (C2 at SLA 8 s:
+                    // 131,072-entry chunks right after the 64-entry first one took 95-406 ms depending
+                    // on which survivors came first, 113-137 ms with a 16,384-entry step between;
+                    // profiles/r02p_bb_grow.md).  A survivor with more than list_cap children spans
+                    // several.
                     struct DeepLaunch { u64 e0; unsigned ne; u64 r0, span; };
                     auto make_chunks = [&](u64 n_entries, u64 Rc) {
                         std::vector<DeepLaunch> L;
@@ -2045,7 +2047,7 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
                                 1, std::min<u64>(per_chunk,
                                                  pp.cost_prune ? (first_env ? (u64)atoll(first_env) : 64) : per_chunk));
                             const char *grow_env = getenv("SMILESS_BB_GROW");
-                            const u64 grow = std::max<u64>(1, grow_env ? (u64)atoll(grow_env) : 4);
+                            const u64 grow = std::max<u64>(1, grow_env ? (u64)atoll(grow_env) : 256);
                             u64 cur = first;
                             for (u64 c0 = 0; c0 < n_entries;) {
                                 const u64 len = std::min<u64>(cur, n_entries - c0);
