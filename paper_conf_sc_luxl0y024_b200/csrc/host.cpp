@@ -1632,599 +1632,599 @@ int plan_impl(smiless_ctx *ctx, const smiless_plan_args *a_in, const i64 *slas, 
         // `first`: the first (or only) digit uploads the caller's cap as the incumbent and starts
         // the evaluator's event
         auto run_once = [&](ResBlock *dst, const bool first) -> int {
-        const u64 V = unit_cands(ctx, a);   // candidates per unit
-        const u64 ub = cb / V, ue = (ce + V - 1) / V;
-        const u64 U = ue - ub;
-        const u64 n_chunks = (U + kChunkUnits - 1) / kChunkUnits;
-        const u64 my_chunks = n_chunks > (u64)shard ? (n_chunks - 1 - (u64)shard) / (u64)n_shards + 1 : 0;
-        const u64 claims_total = my_chunks * (u64)kChunkUnits;
-        const int grid = jk->blocks_per_sm * ctx->n_sms;
-        int grid_used = grid;                        // CTAs whose argmin slots the reduce reads
-        CK(ctx->dBlk.ensure((size_t)grid * 2 * n_sla), "cudaMalloc");
-        CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid * 16 * n_sla, st), "memset");
-        CK(cudaMemsetAsync(ctx->dStats.p, 0, 16, st), "memset");
-        PlanParamsHost pp;
-        memset(&pp, 0, sizeof pp);
-        pp.tabI = ctx->dI.p;
-        pp.tabNI = ctx->dNI.p;
-        pp.tabW = ctx->dW.p;
-        pp.zero = 0;
-        pp.tabT = ctx->dT.p;
-        pp.tabU = ctx->dU.p;
-        pp.off = ctx->dOff.p;
-        pp.scal = ctx->dScal.p;
-        pp.counter = ctx->dCounter.p;
-        pp.stats = ctx->dStats.p;
-        pp.blk_best = ctx->dBlk.p;
-        pp.unit_begin = ub;
-        pp.unit_end = ue;
-        pp.cand_begin = cb;
-        pp.cand_end = ce;
-        pp.n_steps = n_steps;
-        pp.n_off = n_off;
-        pp.sumM = kernel_rows(ctx, a);
-        pp.sla = (int)a->sla_us;
-        for (int s_ = 0; s_ < n_sla; ++s_) pp.slas[s_] = (int)slas[s_];
-        pp.prune = (a->flags & SMILESS_FLAG_NO_PRUNE) ? 0 : 1;
-        // cost-bound pruning against a running incumbent (one SLA, no per-candidate dump);
-        // SMILESS_COST_PRUNE=0 disables it
-        {
-            const char *cp_env = getenv("SMILESS_COST_PRUNE");
-            pp.cost_prune = (pp.prune && n_sla == 1 && !a->cost_out && (!cp_env || atoi(cp_env) != 0)) ? 1 : 0;
-            pp.inc = ctx->dInc.p;
-            pp.rrem = ctx->dRrem.p;
-            pp.cap = ~0ull;
-            if (a->flags & SMILESS_FLAG_COST_CAP) {
-                double c = a->cost_cap + 0.0;               // -0.0 -> +0.0: bits order like the costs
-                memcpy(&pp.cap, &c, 8);
+            const u64 V = unit_cands(ctx, a);   // candidates per unit
+            const u64 ub = cb / V, ue = (ce + V - 1) / V;
+            const u64 U = ue - ub;
+            const u64 n_chunks = (U + kChunkUnits - 1) / kChunkUnits;
+            const u64 my_chunks = n_chunks > (u64)shard ? (n_chunks - 1 - (u64)shard) / (u64)n_shards + 1 : 0;
+            const u64 claims_total = my_chunks * (u64)kChunkUnits;
+            const int grid = jk->blocks_per_sm * ctx->n_sms;
+            int grid_used = grid;                        // CTAs whose argmin slots the reduce reads
+            CK(ctx->dBlk.ensure((size_t)grid * 2 * n_sla), "cudaMalloc");
+            CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid * 16 * n_sla, st), "memset");
+            CK(cudaMemsetAsync(ctx->dStats.p, 0, 16, st), "memset");
+            PlanParamsHost pp;
+            memset(&pp, 0, sizeof pp);
+            pp.tabI = ctx->dI.p;
+            pp.tabNI = ctx->dNI.p;
+            pp.tabW = ctx->dW.p;
+            pp.zero = 0;
+            pp.tabT = ctx->dT.p;
+            pp.tabU = ctx->dU.p;
+            pp.off = ctx->dOff.p;
+            pp.scal = ctx->dScal.p;
+            pp.counter = ctx->dCounter.p;
+            pp.stats = ctx->dStats.p;
+            pp.blk_best = ctx->dBlk.p;
+            pp.unit_begin = ub;
+            pp.unit_end = ue;
+            pp.cand_begin = cb;
+            pp.cand_end = ce;
+            pp.n_steps = n_steps;
+            pp.n_off = n_off;
+            pp.sumM = kernel_rows(ctx, a);
+            pp.sla = (int)a->sla_us;
+            for (int s_ = 0; s_ < n_sla; ++s_) pp.slas[s_] = (int)slas[s_];
+            pp.prune = (a->flags & SMILESS_FLAG_NO_PRUNE) ? 0 : 1;
+            // cost-bound pruning against a running incumbent (one SLA, no per-candidate dump);
+            // SMILESS_COST_PRUNE=0 disables it
+            {
+                const char *cp_env = getenv("SMILESS_COST_PRUNE");
+                pp.cost_prune = (pp.prune && n_sla == 1 && !a->cost_out && (!cp_env || atoi(cp_env) != 0)) ? 1 : 0;
+                pp.inc = ctx->dInc.p;
+                pp.rrem = ctx->dRrem.p;
+                pp.cap = ~0ull;
+                if (a->flags & SMILESS_FLAG_COST_CAP) {
+                    double c = a->cost_cap + 0.0;               // -0.0 -> +0.0: bits order like the costs
+                    memcpy(&pp.cap, &c, 8);
+                }
+                if (first) {                                   // later digits keep the running incumbent
+                    CK(cudaMemcpyAsync(ctx->dInc.p, &pp.cap, 8, cudaMemcpyHostToDevice, st), "H2D incumbent");
+                    ctx->h2d += 8;
+                }
             }
-            if (first) {                                   // later digits keep the running incumbent
-                CK(cudaMemcpyAsync(ctx->dInc.p, &pp.cap, 8, cudaMemcpyHostToDevice, st), "H2D incumbent");
-                ctx->h2d += 8;
+            pp.shard = shard;
+            pp.n_shards = n_shards;
+            pp.chunk_units = kChunkUnits;
+            for (int k = 0; k < a->n_fixed; ++k) pp.fixed[k] = a->fixed_digits[k];
+            if (a->cost_out) {
+                CK(ctx->dDump.ensure((size_t)(ce - cb)), "cudaMalloc dump");
+                CK(cudaMemsetAsync(ctx->dDump.p, 0xff, (size_t)(ce - cb) * sizeof(double), st), "memset dump");  // NaN
+                pp.dump = ctx->dDump.p;
             }
-        }
-        pp.shard = shard;
-        pp.n_shards = n_shards;
-        pp.chunk_units = kChunkUnits;
-        for (int k = 0; k < a->n_fixed; ++k) pp.fixed[k] = a->fixed_digits[k];
-        if (a->cost_out) {
-            CK(ctx->dDump.ensure((size_t)(ce - cb)), "cudaMalloc dump");
-            CK(cudaMemsetAsync(ctx->dDump.p, 0xff, (size_t)(ce - cb) * sizeof(double), st), "memset dump");  // NaN
-            pp.dump = ctx->dDump.p;
-        }
-        const int D = bb_depth(ctx, a);
-        pp.list_upp = 1;
-        const bool memo = memo_path && jk->blocks_up > 0 && jk->blocks_var > 0;
-        if (memo && jk->fn_fused) {
-            eval_path = SMILESS_PATH_MEMO_FUSED;
-            // ---- fused memoisation: upstream walked by each CTA's producer warp into a shared-
-            // memory ring, variants by its consumer warps (evaluator.cuh smiless_fused_kernel);
-            // split cost: the units holding a feasible candidate are re-walked by the plan
-            // kernel in list mode (upstream recomputed per lane, sums of u, cost, argmin)
-            const u64 upp = (u64)(ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
-            const u64 pl0 = ub / upp, ph0 = (ue + upp - 1) / upp;
-            const bool split = split_cost();
-            // prefix batches bound the cost list; tiles of a batch are interleaved over the shards
-            const u64 batch_p = std::min<u64>((u64)1 << 20, ph0 - pl0);
-            if (split) {
-                CK(ctx->dCostList.ensure((size_t)(batch_p * upp)), "cudaMalloc cost list");
-                CK(ctx->dCostN.ensure(1), "cudaMalloc");
-            }
-            MemoParamsHost mp;
-            memset(&mp, 0, sizeof mp);
-            mp.tabNI = ctx->dNI.p;
-            mp.tabT = ctx->dT.p;
-            mp.tabW = ctx->dW.p;
-            mp.tabU = ctx->dU.p;
-            mp.off = ctx->dOff.p;
-            mp.scal = ctx->dScal.p;
-            mp.counter = ctx->dCounter.p;
-            mp.stats = ctx->dStats.p;
-            mp.cost_list = ctx->dCostList.p;
-            mp.cost_n = ctx->dCostN.p;
-            mp.dump = pp.dump;
-            mp.cand_begin = cb;
-            mp.cand_end = ce;
-            mp.n_steps = n_steps;
-            mp.n_off = n_off;
-            mp.sumM = ctx->sumM;
-            mp.sla = (int)a->sla_us;
-            mp.zero = 0;
-            mp.shard = shard;
-            mp.n_shards = n_shards;
-            for (int s_ = 0; s_ < n_sla; ++s_) mp.slas[s_] = (int)slas[s_];
-            for (int k = 0; k < a->n_fixed; ++k) mp.fixed[k] = a->fixed_digits[k];
-            const int grid_f = jk->blocks_fused * ctx->n_sms;
-            if (grid_f > grid) {     // per-CTA argmin slots of the fused kernel
-                CK(ctx->dBlk.ensure((size_t)grid_f * 2 * n_sla), "cudaMalloc");
-                CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid_f * 16 * n_sla, st), "memset");
-                pp.blk_best = ctx->dBlk.p;
-            }
-            mp.blk_best = ctx->dBlk.p;
-            // the cost re-walk: plan kernel, list mode over the fused pass's cost list
-            PlanParamsHost pc = pp;
-            pc.prune = 0;
-            pc.cost_prune = 0;
-            pc.cap = ~0ull;
-            pc.horizon = 0;
-            pc.claims_begin = 0;
-            pc.claims_end = ~0ull;
-            pc.list_in = ctx->dCostList.p;
-            pc.list_n = ctx->dCostN.p;
-            pc.list_upp = 1;
-            pc.list_base = 0;
-            pc.list_in_cap = batch_p * upp;
-            pc.no_count = 1;
-            if (first) CK(cudaEventRecord(ctx->ev[1], st), "event");
-            NvtxRange nv("memo: fused producer/consumer batches");
-            for (u64 b0 = pl0; b0 < ph0; b0 += batch_p) {
-                const u64 b1 = std::min(ph0, b0 + batch_p);
-                mp.pref_begin = b0;
-                mp.pref_end = b1;
-                mp.unit_begin = std::max(ub, b0 * upp);
-                mp.unit_end = std::min(ue, b1 * upp);
-                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                if (split) CK(cudaMemsetAsync(ctx->dCostN.p, 0, sizeof(unsigned), st), "memset cost list");
-                void *args[] = {&mp};
-                CUresult r = driver().launchKernel(jk->fn_fused, (unsigned)grid_f, 1, 1, fused_threads(), 1, 1,
-                                                   (unsigned)jk->smem_fused, (CUstream)st, args, nullptr);
-                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "fused launch");
-                ++launches;
+            const int D = bb_depth(ctx, a);
+            pp.list_upp = 1;
+            const bool memo = memo_path && jk->blocks_up > 0 && jk->blocks_var > 0;
+            if (memo && jk->fn_fused) {
+                eval_path = SMILESS_PATH_MEMO_FUSED;
+                // ---- fused memoisation: upstream walked by each CTA's producer warp into a shared-
+                // memory ring, variants by its consumer warps (evaluator.cuh smiless_fused_kernel);
+                // split cost: the units holding a feasible candidate are re-walked by the plan
+                // kernel in list mode (upstream recomputed per lane, sums of u, cost, argmin)
+                const u64 upp = (u64)(ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
+                const u64 pl0 = ub / upp, ph0 = (ue + upp - 1) / upp;
+                const bool split = split_cost();
+                // prefix batches bound the cost list; tiles of a batch are interleaved over the shards
+                const u64 batch_p = std::min<u64>((u64)1 << 20, ph0 - pl0);
                 if (split) {
-                    CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                    void *cargs[] = {&pc};
-                    r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
-                                              (CUstream)st, cargs, nullptr);
-                    if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "fused cost re-walk launch");
-                    ++launches;
+                    CK(ctx->dCostList.ensure((size_t)(batch_p * upp)), "cudaMalloc cost list");
+                    CK(ctx->dCostN.ensure(1), "cudaMalloc");
                 }
-            }
-            grid_used = std::max(grid, grid_f);
-        } else if (memo) {
-            eval_path = SMILESS_PATH_MEMO;
-            // ---- prefix memoisation: upstream once per prefix, then the variants per unit ---------
-            const u64 upp = (u64)(ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
-            const u64 pl0 = ub / upp, ph0 = (ue + upp - 1) / upp;
-            const size_t tsz2 = rp.time64 ? 8 : 4;
-            // + SM_XPF + 1 groups of 4 steps of read-ahead slack for the variants kernel
-            const size_t row_bytes = tsz2 * (size_t)(n_off + 4 * (xpf_groups() + 1));
-            // Batches of up to 2^20 prefixes (fewer launches, fewer tails, a fuller upstream
-            // kernel: 3.80e8 -> 3.95e8 candidates/s on the C2 slice, profiles/r02l_memo_batch.md),
-            // the x buffer bounded by a quarter of the device memory; halved while the
-            // allocation fails.  SMILESS_MEMO_BATCH (tuning) sets the prefixes per batch.
-            size_t mem_free = 0, mem_total = 0;
-            CK(cudaMemGetInfo(&mem_free, &mem_total), "cudaMemGetInfo");
-            u64 max_batch = std::max<u64>(1, std::min<u64>((u64)1 << 20, (u64)(mem_total / 4) / row_bytes));
-            if (const char *mb_env = getenv("SMILESS_MEMO_BATCH"))
-                max_batch = std::max<u64>(1, std::min<u64>((u64)atoll(mb_env), ((u64)64 << 30) / row_bytes));
-            u64 batch_p = std::min<u64>(max_batch, ph0 - pl0);
-            while (ctx->dX.ensure((size_t)batch_p * row_bytes) != cudaSuccess && batch_p > 1) {
-                cudaGetLastError();                                  // clear the allocation failure
-                batch_p = (batch_p + 1) / 2;
-            }
-            CK(ctx->dX.ensure((size_t)batch_p * row_bytes), "cudaMalloc memo buffer");
-            CK(ctx->dRecNx.ensure((size_t)batch_p), "cudaMalloc");
-            CK(ctx->dRecNlu.ensure((size_t)batch_p), "cudaMalloc");
-            CK(ctx->dRecPre.ensure((size_t)batch_p), "cudaMalloc");
-            if (jk->fn_varc) {
-                CK(ctx->dCostList.ensure((size_t)(batch_p * upp)), "cudaMalloc cost list");
-                CK(ctx->dCostN.ensure(1), "cudaMalloc");
-            }
-            MemoParamsHost mp;
-            memset(&mp, 0, sizeof mp);
-            mp.tabNI = ctx->dNI.p;
-            mp.tabT = ctx->dT.p;
-            mp.tabW = ctx->dW.p;
-            mp.tabU = ctx->dU.p;
-            mp.off = ctx->dOff.p;
-            mp.scal = ctx->dScal.p;
-            mp.counter = ctx->dCounter.p;
-            mp.stats = ctx->dStats.p;
-            mp.blk_best = ctx->dBlk.p;
-            mp.xbuf = ctx->dX.p;
-            mp.rec_nx = ctx->dRecNx.p;
-            mp.rec_pre = ctx->dRecPre.p;
-            mp.rec_nlu = ctx->dRecNlu.p;
-            mp.cost_list = ctx->dCostList.p;
-            mp.cost_n = ctx->dCostN.p;
-            mp.dump = pp.dump;
-            mp.cand_begin = cb;
-            mp.cand_end = ce;
-            mp.n_steps = n_steps;
-            mp.n_off = n_off;
-            mp.sumM = ctx->sumM;
-            mp.sla = (int)a->sla_us;
-            mp.zero = 0;
-            for (int s_ = 0; s_ < n_sla; ++s_) mp.slas[s_] = (int)slas[s_];
-            for (int k = 0; k < a->n_fixed; ++k) mp.fixed[k] = a->fixed_digits[k];
-            const int grid_up = jk->blocks_up * ctx->n_sms;
-            const int grid_var = jk->blocks_var * ctx->n_sms;
-            if (grid_var > grid) {     // per-CTA argmin slots of the variants kernel
-                CK(ctx->dBlk.ensure((size_t)grid_var * 2 * n_sla), "cudaMalloc");
-                CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid_var * 16 * n_sla, st), "memset");
+                MemoParamsHost mp;
+                memset(&mp, 0, sizeof mp);
+                mp.tabNI = ctx->dNI.p;
+                mp.tabT = ctx->dT.p;
+                mp.tabW = ctx->dW.p;
+                mp.tabU = ctx->dU.p;
+                mp.off = ctx->dOff.p;
+                mp.scal = ctx->dScal.p;
+                mp.counter = ctx->dCounter.p;
+                mp.stats = ctx->dStats.p;
+                mp.cost_list = ctx->dCostList.p;
+                mp.cost_n = ctx->dCostN.p;
+                mp.dump = pp.dump;
+                mp.cand_begin = cb;
+                mp.cand_end = ce;
+                mp.n_steps = n_steps;
+                mp.n_off = n_off;
+                mp.sumM = ctx->sumM;
+                mp.sla = (int)a->sla_us;
+                mp.zero = 0;
+                mp.shard = shard;
+                mp.n_shards = n_shards;
+                for (int s_ = 0; s_ < n_sla; ++s_) mp.slas[s_] = (int)slas[s_];
+                for (int k = 0; k < a->n_fixed; ++k) mp.fixed[k] = a->fixed_digits[k];
+                const int grid_f = jk->blocks_fused * ctx->n_sms;
+                if (grid_f > grid) {     // per-CTA argmin slots of the fused kernel
+                    CK(ctx->dBlk.ensure((size_t)grid_f * 2 * n_sla), "cudaMalloc");
+                    CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid_f * 16 * n_sla, st), "memset");
+                    pp.blk_best = ctx->dBlk.p;
+                }
                 mp.blk_best = ctx->dBlk.p;
-            }
-            if (first) CK(cudaEventRecord(ctx->ev[1], st), "event");
-            NvtxRange nv("memo: upstream + variants batches");
-            u64 bi = 0;
-            for (u64 b0 = pl0; b0 < ph0; b0 += batch_p, ++bi) {
-                if (bi % (u64)n_shards != (u64)shard) continue;
-                const u64 b1 = std::min(ph0, b0 + batch_p);
-                mp.pref_begin = b0;
-                mp.pref_end = b1;
-                mp.unit_begin = std::max(ub, b0 * upp);
-                mp.unit_end = std::min(ue, b1 * upp);
-                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                void *args[] = {&mp};
-                CUresult r = driver().launchKernel(jk->fn_up, (unsigned)grid_up, 1, 1, kThreads, 1, 1,
-                                                   (unsigned)jk->smem_up, (CUstream)st, args, nullptr);
-                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "upstream launch");
-                ++launches;
-                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                if (jk->fn_varc) CK(cudaMemsetAsync(ctx->dCostN.p, 0, sizeof(unsigned), st), "memset cost list");
-                r = driver().launchKernel(jk->fn_var, (unsigned)grid_var, 1, 1, vthreads_per_cta(), 1, 1,
-                                          (unsigned)jk->smem_var, (CUstream)st, args, nullptr);
-                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "variants launch");
-                ++launches;
-                if (jk->fn_varc) {                 // split cost: re-walk the units with a feasible candidate
+                // the cost re-walk: plan kernel, list mode over the fused pass's cost list
+                PlanParamsHost pc = pp;
+                pc.prune = 0;
+                pc.cost_prune = 0;
+                pc.cap = ~0ull;
+                pc.horizon = 0;
+                pc.claims_begin = 0;
+                pc.claims_end = ~0ull;
+                pc.list_in = ctx->dCostList.p;
+                pc.list_n = ctx->dCostN.p;
+                pc.list_upp = 1;
+                pc.list_base = 0;
+                pc.list_in_cap = batch_p * upp;
+                pc.no_count = 1;
+                if (first) CK(cudaEventRecord(ctx->ev[1], st), "event");
+                NvtxRange nv("memo: fused producer/consumer batches");
+                for (u64 b0 = pl0; b0 < ph0; b0 += batch_p) {
+                    const u64 b1 = std::min(ph0, b0 + batch_p);
+                    mp.pref_begin = b0;
+                    mp.pref_end = b1;
+                    mp.unit_begin = std::max(ub, b0 * upp);
+                    mp.unit_end = std::min(ue, b1 * upp);
                     CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                    r = driver().launchKernel(jk->fn_varc, (unsigned)grid_var, 1, 1, vthreads_per_cta(), 1, 1,
-                                              (unsigned)jk->smem_var, (CUstream)st, args, nullptr);
-                    if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "variants cost launch");
+                    if (split) CK(cudaMemsetAsync(ctx->dCostN.p, 0, sizeof(unsigned), st), "memset cost list");
+                    void *args[] = {&mp};
+                    CUresult r = driver().launchKernel(jk->fn_fused, (unsigned)grid_f, 1, 1, fused_threads(), 1, 1,
+                                                       (unsigned)jk->smem_fused, (CUstream)st, args, nullptr);
+                    if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "fused launch");
                     ++launches;
+                    if (split) {
+                        CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                        void *cargs[] = {&pc};
+                        r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
+                                                  (CUstream)st, cargs, nullptr);
+                        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "fused cost re-walk launch");
+                        ++launches;
+                    }
                 }
-            }
-            grid_used = std::max(grid, grid_var);
-        } else if (bnb_path && D > 0 && jk->blocks_bound > 0) {
-            eval_path = SMILESS_PATH_BNB;
-            // ---- exact branch-and-bound: prefixes of functions n_fixed..D-1, then list mode ----
-            // Sharding (multi-GPU): the deep level's prefixes (one level) or the deep children of
-            // every shallow survivor (two levels) are interleaved over the shards, ordinal
-            // c = c' * n_shards + shard, so every rank decides an equal share of every survivor's
-            // subtree; the shallow level (<= 2^22 prefixes) is replicated on every rank.
-            const u64 S = cands_per_prefix(ctx, a, D);
-            const u64 upp = S / V;                            // evaluator units per prefix
-            const u64 p_lo = cb / S, p_hi = (ce + S - 1) / S;
-            const u64 batch = (u64)1 << 22;                   // prefixes per range-mode bound launch
-            const int DA = bb_depth_a(ctx, a, D);
-            const u64 R = DA > 0 ? cands_per_prefix(ctx, a, DA) / S : 1;   // deep children per shallow prefix
-            // deep survivor list: no launch enumerates more than list_cap ordinals, so it cannot
-            // overflow (the kernel still checks, and a violation fails the call)
-            u64 list_cap = R > ((u64)1 << 24) ? ((u64)1 << 26) : ((u64)1 << 24);
-            if (const char *lc_env = getenv("SMILESS_BB_LISTCAP"))   // testing: force the split paths
-                list_cap = std::max<u64>(1, std::min<u64>(list_cap, (u64)atoll(lc_env)));
-            CK(ctx->dList.ensure((size_t)list_cap), "cudaMalloc list");
-            CK(ctx->dListCnt.ensure(1), "cudaMalloc");
-            pp.list_in_cap = list_cap;
-            BoundParamsHost bp;
-            memset(&bp, 0, sizeof bp);
-            bp.tabNI = ctx->dNI.p;
-            bp.tabW = ctx->dW.p;
-            bp.tabT = ctx->dT.p;
-            bp.tabU = ctx->dU.p;
-            bp.scal = ctx->dScal.p;
-            bp.inc = ctx->dInc.p;
-            bp.cost_prune = pp.cost_prune;
-            bp.off = ctx->dOff.p;
-            bp.counter = ctx->dCounter.p;
-            bp.stats = ctx->dStats.p;
-            bp.list_out = ctx->dList.p;
-            bp.list_cnt = ctx->dListCnt.p;
-            bp.list_cap = list_cap;
-            bp.overflow = (unsigned *)ctx->dErr.p;            // bit 2 (value 4): list overflow
-            bp.cands_per_prefix = S;
-            bp.cand_begin = cb;
-            bp.cand_end = ce;
-            bp.n_steps = n_steps;
-            bp.n_off = n_off;
-            bp.sumM = kernel_rows(ctx, a);
-            bp.sla = (int)a->sla_us;
-            bp.zero = 0;
-            bp.shard = shard;
-            bp.n_shards = n_shards;
-            bp.attr_shard = 0;
-            bp.attr_n = 1;
-            for (int k = 0; k < ctx->N; ++k) {
-                int m = ctx->I[ctx->row0[k]];
-                for (int c = 1; c < ctx->M[k]; ++c) m = std::min(m, ctx->I[ctx->row0[k] + c]);
-                bp.nimin[k] = -m;
-            }
-            for (int k = 0; k < a->n_fixed; ++k) bp.fixed[k] = a->fixed_digits[k];
-            const int grid_b = jk->blocks_bound * ctx->n_sms;
-            if (first) CK(cudaEventRecord(ctx->ev[1], st), "event");
-            // evaluator over the deep survivors in dList (absolute depth-D prefix ids)
-            auto run_eval = [&]() -> int {
-                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                pp.claims_begin = 0;
-                pp.claims_end = ~0ull;
-                pp.list_in = ctx->dList.p;
-                pp.list_n = ctx->dListCnt.p;
-                pp.list_upp = upp;
-                pp.list_base = 0;
-                pp.list_out = nullptr;
-                pp.list_cnt = nullptr;
-                pp.horizon = 0;
-                void *args[] = {&pp};
-                CUresult r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
-                                                   (CUstream)st, args, nullptr);
-                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
-                ++launches;
-                return SMILESS_OK;
-            };
-            auto run_bound = [&](CUfunction fn) -> int {
-                void *bargs[] = {&bp};
-                CUresult r = driver().launchKernel(fn, (unsigned)grid_b, 1, 1, kThreads, 1, 1,
-                                                   (unsigned)jk->smem_bound, (CUstream)st, bargs, nullptr);
-                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "bound launch");
-                ++launches;
-                return SMILESS_OK;
-            };
-            if (DA > 0) {
-                // ---- two levels: depth DA over every prefix, depth D over the DA survivors' children --
-                const u64 SA = cands_per_prefix(ctx, a, DA);
-                const u64 a_lo = cb / SA, a_hi = (ce + SA - 1) / SA;
-                CK(ctx->dListA.ensure((size_t)batch), "cudaMalloc list");
-                CK(ctx->dListCntA.ensure(1), "cudaMalloc");
-                // best-first: with the cost bound on, the shallow survivors are sorted by their
-                // static cost lower bound so the first deep launch sets a good incumbent early
-                // (SMILESS_BB_SORT=1; off by default: measured slower on C2 with live windows and
-                // no faster elsewhere, profiles/r02k_bb_sort.md)
-                const char *sort_env = getenv("SMILESS_BB_SORT");
-                const bool bb_sort = pp.cost_prune && sort_env && atoi(sort_env) != 0;
-                if (bb_sort) CK(ctx->dListKeyA.ensure((size_t)batch), "cudaMalloc keys");
-                std::vector<u64> h_pref, h_key;
-                std::vector<uint32_t> h_ord;
-                for (u64 b0 = a_lo; b0 < a_hi; b0 += batch) {
-                    const u64 b1 = std::min(a_hi, b0 + batch);
+                grid_used = std::max(grid, grid_f);
+            } else if (memo) {
+                eval_path = SMILESS_PATH_MEMO;
+                // ---- prefix memoisation: upstream once per prefix, then the variants per unit ---------
+                const u64 upp = (u64)(ctx->M[ctx->N - 1] / configs_per_lane(ctx, a));
+                const u64 pl0 = ub / upp, ph0 = (ue + upp - 1) / upp;
+                const size_t tsz2 = rp.time64 ? 8 : 4;
+                // + SM_XPF + 1 groups of 4 steps of read-ahead slack for the variants kernel
+                const size_t row_bytes = tsz2 * (size_t)(n_off + 4 * (xpf_groups() + 1));
+                // Batches of up to 2^20 prefixes (fewer launches, fewer tails, a fuller upstream
+                // kernel: 3.80e8 -> 3.95e8 candidates/s on the C2 slice, profiles/r02l_memo_batch.md),
+                // the x buffer bounded by a quarter of the device memory; halved while the
+                // allocation fails.  SMILESS_MEMO_BATCH (tuning) sets the prefixes per batch.
+                size_t mem_free = 0, mem_total = 0;
+                CK(cudaMemGetInfo(&mem_free, &mem_total), "cudaMemGetInfo");
+                u64 max_batch = std::max<u64>(1, std::min<u64>((u64)1 << 20, (u64)(mem_total / 4) / row_bytes));
+                if (const char *mb_env = getenv("SMILESS_MEMO_BATCH"))
+                    max_batch = std::max<u64>(1, std::min<u64>((u64)atoll(mb_env), ((u64)64 << 30) / row_bytes));
+                u64 batch_p = std::min<u64>(max_batch, ph0 - pl0);
+                while (ctx->dX.ensure((size_t)batch_p * row_bytes) != cudaSuccess && batch_p > 1) {
+                    cudaGetLastError();                                  // clear the allocation failure
+                    batch_p = (batch_p + 1) / 2;
+                }
+                CK(ctx->dX.ensure((size_t)batch_p * row_bytes), "cudaMalloc memo buffer");
+                CK(ctx->dRecNx.ensure((size_t)batch_p), "cudaMalloc");
+                CK(ctx->dRecNlu.ensure((size_t)batch_p), "cudaMalloc");
+                CK(ctx->dRecPre.ensure((size_t)batch_p), "cudaMalloc");
+                if (jk->fn_varc) {
+                    CK(ctx->dCostList.ensure((size_t)(batch_p * upp)), "cudaMalloc cost list");
+                    CK(ctx->dCostN.ensure(1), "cudaMalloc");
+                }
+                MemoParamsHost mp;
+                memset(&mp, 0, sizeof mp);
+                mp.tabNI = ctx->dNI.p;
+                mp.tabT = ctx->dT.p;
+                mp.tabW = ctx->dW.p;
+                mp.tabU = ctx->dU.p;
+                mp.off = ctx->dOff.p;
+                mp.scal = ctx->dScal.p;
+                mp.counter = ctx->dCounter.p;
+                mp.stats = ctx->dStats.p;
+                mp.blk_best = ctx->dBlk.p;
+                mp.xbuf = ctx->dX.p;
+                mp.rec_nx = ctx->dRecNx.p;
+                mp.rec_pre = ctx->dRecPre.p;
+                mp.rec_nlu = ctx->dRecNlu.p;
+                mp.cost_list = ctx->dCostList.p;
+                mp.cost_n = ctx->dCostN.p;
+                mp.dump = pp.dump;
+                mp.cand_begin = cb;
+                mp.cand_end = ce;
+                mp.n_steps = n_steps;
+                mp.n_off = n_off;
+                mp.sumM = ctx->sumM;
+                mp.sla = (int)a->sla_us;
+                mp.zero = 0;
+                for (int s_ = 0; s_ < n_sla; ++s_) mp.slas[s_] = (int)slas[s_];
+                for (int k = 0; k < a->n_fixed; ++k) mp.fixed[k] = a->fixed_digits[k];
+                const int grid_up = jk->blocks_up * ctx->n_sms;
+                const int grid_var = jk->blocks_var * ctx->n_sms;
+                if (grid_var > grid) {     // per-CTA argmin slots of the variants kernel
+                    CK(ctx->dBlk.ensure((size_t)grid_var * 2 * n_sla), "cudaMalloc");
+                    CK(cudaMemsetAsync(ctx->dBlk.p, 0xff, (size_t)grid_var * 16 * n_sla, st), "memset");
+                    mp.blk_best = ctx->dBlk.p;
+                }
+                if (first) CK(cudaEventRecord(ctx->ev[1], st), "event");
+                NvtxRange nv("memo: upstream + variants batches");
+                u64 bi = 0;
+                for (u64 b0 = pl0; b0 < ph0; b0 += batch_p, ++bi) {
+                    if (bi % (u64)n_shards != (u64)shard) continue;
+                    const u64 b1 = std::min(ph0, b0 + batch_p);
+                    mp.pref_begin = b0;
+                    mp.pref_end = b1;
+                    mp.unit_begin = std::max(ub, b0 * upp);
+                    mp.unit_end = std::min(ue, b1 * upp);
                     CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                    CK(cudaMemsetAsync(ctx->dListCntA.p, 0, sizeof(unsigned), st), "memset list");
-                    bp.list_in = nullptr;
-                    bp.list_n = nullptr;
-                    bp.list_upp = 1;
-                    bp.list_stride = 1;
-                    bp.list_r0 = 0;
-                    bp.prefix_begin = b0;
-                    bp.prefix_end = b1;
-                    bp.cands_per_prefix = SA;
-                    bp.list_out = ctx->dListA.p;
-                    bp.list_cnt = ctx->dListCntA.p;
-                    bp.list_cap = batch;
-                    bp.shard = 0;                                 // replicated on every shard ...
-                    bp.n_shards = 1;
-                    bp.attr_shard = shard;                        // ... its pruned prefixes counted once
-                    bp.attr_n = n_shards;
-                    bp.list_key = bb_sort ? ctx->dListKeyA.p : nullptr;
-                    {
-                        NvtxRange nv("bnb shallow level");
-                        if ((rc = run_bound(jk->fn_bound_a))) return rc;
-                    }
-                    unsigned n_a = 0;
-                    hp.mark("launch_a");
-                    CK(cudaMemcpyAsync(&n_a, ctx->dListCntA.p, sizeof n_a, cudaMemcpyDeviceToHost, st), "D2H count");
-                    ctx->d2h += sizeof n_a;
-                    CK(cudaStreamSynchronize(st), "count");
-                    hp.mark("sync_a");
-                    hp.note("n_a", n_a);
-                    bp.list_key = nullptr;
-                    if (bb_sort && n_a > 1 && n_a <= (1u << 18)) {
-                        // (key, prefix) ascending; ties by prefix: a deterministic order on every rank
-                        h_pref.resize(n_a);
-                        h_key.resize(n_a);
-                        CK(cudaMemcpyAsync(h_pref.data(), ctx->dListA.p, n_a * sizeof(u64), cudaMemcpyDeviceToHost, st),
-                           "D2H survivors");
-                        CK(cudaMemcpyAsync(h_key.data(), ctx->dListKeyA.p, n_a * sizeof(u64), cudaMemcpyDeviceToHost, st),
-                           "D2H keys");
-                        CK(cudaStreamSynchronize(st), "survivors");
-                        h_ord.resize(n_a);
-                        for (uint32_t q = 0; q < n_a; ++q) h_ord[q] = q;
-                        std::sort(h_ord.begin(), h_ord.end(), [&](uint32_t x, uint32_t y) {
-                            return h_key[x] != h_key[y] ? h_key[x] < h_key[y] : h_pref[x] < h_pref[y];
-                        });
-                        std::vector<u64> sorted(n_a);
-                        for (uint32_t q = 0; q < n_a; ++q) sorted[q] = h_pref[h_ord[q]];
-                        CK(cudaMemcpyAsync(ctx->dListA.p, sorted.data(), n_a * sizeof(u64), cudaMemcpyHostToDevice, st),
-                           "H2D survivors");
-                        ctx->d2h += 2 * (u64)n_a * sizeof(u64);
-                        ctx->h2d += (u64)n_a * sizeof(u64);
-                        hp.mark("sort_a");
-                    }
-                    // Launches over a survivor list (first entry, entries, first child, children per
-                    // entry): at most list_cap ordinals each.  With the cost bound on, the first launch
-                    // is small and each next one SMILESS_BB_GROW (256) times larger: every launch's
-                    // static prefix bound prunes against the incumbent the evaluations before it set,
-                    // so the incumbent is refined before the bulk of the list (C2 at SLA 8 s:
-                    // 131,072-entry chunks right after the 64-entry first one took 95-406 ms depending
-                    // on which survivors came first, 113-137 ms with a 16,384-entry step between;
-                    // profiles/r02p_bb_grow.md).  A survivor with more than list_cap children spans
-                    // several.
-                    struct DeepLaunch { u64 e0; unsigned ne; u64 r0, span; };
-                    auto make_chunks = [&](u64 n_entries, u64 Rc) {
-                        std::vector<DeepLaunch> L;
-                        if (Rc <= list_cap) {
-                            const u64 per_chunk = list_cap / Rc;
-                            const char *first_env = getenv("SMILESS_BB_FIRST");
-                            const u64 first = std::max<u64>(
-                                1, std::min<u64>(per_chunk,
-                                                 pp.cost_prune ? (first_env ? (u64)atoll(first_env) : 64) : per_chunk));
-                            const char *grow_env = getenv("SMILESS_BB_GROW");
-                            const u64 grow = std::max<u64>(1, grow_env ? (u64)atoll(grow_env) : 256);
-                            u64 cur = first;
-                            for (u64 c0 = 0; c0 < n_entries;) {
-                                const u64 len = std::min<u64>(cur, n_entries - c0);
-                                L.push_back({c0, (unsigned)len, 0, Rc});
-                                c0 += len;
-                                cur = std::min<u64>(per_chunk, cur * grow);
-                            }
-                        } else {
-                            for (u64 e = 0; e < n_entries; ++e)
-                                for (u64 r0 = 0; r0 < Rc; r0 += list_cap)
-                                    L.push_back({e, 1u, r0, std::min(list_cap, Rc - r0)});
-                        }
-                        return L;
-                    };
-                    auto upload_counts = [&](const std::vector<DeepLaunch> &L, DevBuf<unsigned> &buf) -> int {
-                        std::vector<unsigned> cnts(std::max<size_t>(L.size(), 1), 0u);
-                        for (size_t i = 0; i < L.size(); ++i) cnts[i] = L[i].ne;
-                        CK(buf.ensure(cnts.size()), "cudaMalloc counts");
-                        ctx->h2d += cnts.size() * sizeof(unsigned);
-                        CK(cudaMemcpyAsync(buf.p, cnts.data(), cnts.size() * sizeof(unsigned), cudaMemcpyHostToDevice, st),
-                           "H2D counts");
-                        return SMILESS_OK;
-                    };
-                    // one level over the children of a survivor list: bound kernel `fn` at depth with
-                    // `Sc` candidates per prefix writes its survivors to out / out_cnt; then `after`
-                    auto run_level = [&](CUfunction fn, const u64 *list, const std::vector<DeepLaunch> &L,
-                                         DevBuf<unsigned> &cnt_buf, u64 Rc, u64 Sc, u64 *out, unsigned *out_cnt,
-                                         int shard_, int n_shards_, const std::function<int(size_t)> &after) -> int {
-                        for (size_t i = 0; i < L.size(); ++i) {
-                            CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                            CK(cudaMemsetAsync(out_cnt, 0, sizeof(unsigned), st), "memset list");
-                            bp.list_in = list + L[i].e0;
-                            bp.list_n = cnt_buf.p + i;
-                            bp.list_upp = L[i].span;
-                            bp.list_stride = Rc;
-                            bp.list_r0 = L[i].r0;
-                            bp.prefix_begin = 0;
-                            bp.prefix_end = 0;
-                            bp.cands_per_prefix = Sc;
-                            bp.list_out = out;
-                            bp.list_cnt = out_cnt;
-                            bp.list_cap = list_cap;
-                            bp.shard = shard_;
-                            bp.n_shards = n_shards_;
-                            bp.attr_shard = 0;
-                            bp.attr_n = 1;
-                            if ((rc = run_bound(fn))) return rc;
-                            if ((rc = after(i))) return rc;
-                        }
-                        return SMILESS_OK;
-                    };
-                    const int DM = jk->fn_bound_m ? bb_depth_m(ctx, a, D, DA) : 0;
-                    if (DM == 0) {
-                        // two levels: the deep children of the shallow survivors, interleaved over shards
-                        const std::vector<DeepLaunch> L = make_chunks(n_a, R);
-                        if ((rc = upload_counts(L, ctx->dChunkCnt))) return rc;
-                        NvtxRange nv("bnb deep level + evaluate");
-                        if ((rc = run_level(jk->fn_bound, ctx->dListA.p, L, ctx->dChunkCnt, R, S, ctx->dList.p,
-                                            ctx->dListCnt.p, shard, n_shards, [&](size_t) { return run_eval(); })))
-                            return rc;
-                    } else {
-                        // three levels: the middle children of the shallow survivors (interleaved over
-                        // shards), then the deep children of each middle launch's survivors (this
-                        // rank's own, not split again) and the evaluator over those
-                        const u64 SMd = cands_per_prefix(ctx, a, DM);
-                        const u64 R1 = SA / SMd, R2 = SMd / S;
-                        CK(ctx->dListM.ensure((size_t)list_cap), "cudaMalloc list");
-                        CK(ctx->dListCntM.ensure(1), "cudaMalloc");
-                        const std::vector<DeepLaunch> Lm = make_chunks(n_a, R1);
-                        if ((rc = upload_counts(Lm, ctx->dChunkCntM))) return rc;
-                        NvtxRange nv("bnb middle + deep level + evaluate");
-                        auto deep = [&](size_t) -> int {
-                            unsigned n_m = 0;
-                            CK(cudaMemcpyAsync(&n_m, ctx->dListCntM.p, sizeof n_m, cudaMemcpyDeviceToHost, st), "D2H count");
-                            ctx->d2h += sizeof n_m;
-                            CK(cudaStreamSynchronize(st), "count");
-                            hp.note("n_m", n_m);
-                            if (n_m == 0) return SMILESS_OK;
-                            const std::vector<DeepLaunch> L = make_chunks(n_m, R2);
-                            if ((rc = upload_counts(L, ctx->dChunkCnt))) return rc;
-                            return run_level(jk->fn_bound, ctx->dListM.p, L, ctx->dChunkCnt, R2, S, ctx->dList.p,
-                                             ctx->dListCnt.p, 0, 1, [&](size_t) { return run_eval(); });
-                        };
-                        if ((rc = run_level(jk->fn_bound_m, ctx->dListA.p, Lm, ctx->dChunkCntM, R1, SMd, ctx->dListM.p,
-                                            ctx->dListCntM.p, shard, n_shards, deep)))
-                            return rc;
-                    }
-                    hp.mark("chunks_launched");
-                    CK(cudaStreamSynchronize(st), "chunks");      // the next batch reuses dListA
-                    hp.mark("sync_chunks");
-                }
-            } else {
-                NvtxRange nv("bnb level + evaluate");
-                const u64 rbatch = std::min(batch, list_cap);     // a launch's survivors fit the list
-                for (u64 b0 = p_lo; b0 < p_hi; b0 += rbatch) {
-                    const u64 b1 = std::min(p_hi, b0 + rbatch);
+                    void *args[] = {&mp};
+                    CUresult r = driver().launchKernel(jk->fn_up, (unsigned)grid_up, 1, 1, kThreads, 1, 1,
+                                                       (unsigned)jk->smem_up, (CUstream)st, args, nullptr);
+                    if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "upstream launch");
+                    ++launches;
                     CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                    CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
-                    bp.list_in = nullptr;
-                    bp.list_n = nullptr;
-                    bp.list_upp = 1;
-                    bp.list_stride = 1;
-                    bp.list_r0 = 0;
-                    bp.prefix_begin = b0;
-                    bp.prefix_end = b1;
-                    if ((rc = run_bound(jk->fn_bound))) return rc;
-                    if ((rc = run_eval())) return rc;
+                    if (jk->fn_varc) CK(cudaMemsetAsync(ctx->dCostN.p, 0, sizeof(unsigned), st), "memset cost list");
+                    r = driver().launchKernel(jk->fn_var, (unsigned)grid_var, 1, 1, vthreads_per_cta(), 1, 1,
+                                              (unsigned)jk->smem_var, (CUstream)st, args, nullptr);
+                    if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "variants launch");
+                    ++launches;
+                    if (jk->fn_varc) {                 // split cost: re-walk the units with a feasible candidate
+                        CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                        r = driver().launchKernel(jk->fn_varc, (unsigned)grid_var, 1, 1, vthreads_per_cta(), 1, 1,
+                                                  (unsigned)jk->smem_var, (CUstream)st, args, nullptr);
+                        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "variants cost launch");
+                        ++launches;
+                    }
                 }
-            }
-        } else {
-            eval_path = SMILESS_PATH_PLAN;
-            // split very large ranges into several launches (bounded kernel duration).  Prune mode
-            // with J - 1 > horizon runs each batch twice: pass 1 (every unit, `horizon` steps,
-            // survivors compacted into a list), pass 2 (survivors only, all steps).
-            const char *hz_env = getenv("SMILESS_HORIZON");
-            i64 horizon = hz_env ? atoll(hz_env) : 128;
-            horizon = horizon / rp.K * rp.K;
-            const bool compact = pp.prune && horizon > 0 && horizon < n_steps;
-            const u64 claims_per_launch = compact ? ((u64)1 << 24) : ((u64)1 << 28);   // units
-            if (compact) {
-                CK(ctx->dList.ensure((size_t)claims_per_launch), "cudaMalloc list");
+                grid_used = std::max(grid, grid_var);
+            } else if (bnb_path && D > 0 && jk->blocks_bound > 0) {
+                eval_path = SMILESS_PATH_BNB;
+                // ---- exact branch-and-bound: prefixes of functions n_fixed..D-1, then list mode ----
+                // Sharding (multi-GPU): the deep level's prefixes (one level) or the deep children of
+                // every shallow survivor (two levels) are interleaved over the shards, ordinal
+                // c = c' * n_shards + shard, so every rank decides an equal share of every survivor's
+                // subtree; the shallow level (<= 2^22 prefixes) is replicated on every rank.
+                const u64 S = cands_per_prefix(ctx, a, D);
+                const u64 upp = S / V;                            // evaluator units per prefix
+                const u64 p_lo = cb / S, p_hi = (ce + S - 1) / S;
+                const u64 batch = (u64)1 << 22;                   // prefixes per range-mode bound launch
+                const int DA = bb_depth_a(ctx, a, D);
+                const u64 R = DA > 0 ? cands_per_prefix(ctx, a, DA) / S : 1;   // deep children per shallow prefix
+                // deep survivor list: no launch enumerates more than list_cap ordinals, so it cannot
+                // overflow (the kernel still checks, and a violation fails the call)
+                u64 list_cap = R > ((u64)1 << 24) ? ((u64)1 << 26) : ((u64)1 << 24);
+                if (const char *lc_env = getenv("SMILESS_BB_LISTCAP"))   // testing: force the split paths
+                    list_cap = std::max<u64>(1, std::min<u64>(list_cap, (u64)atoll(lc_env)));
+                CK(ctx->dList.ensure((size_t)list_cap), "cudaMalloc list");
                 CK(ctx->dListCnt.ensure(1), "cudaMalloc");
-            }
-            if (first) CK(cudaEventRecord(ctx->ev[1], st), "event");
-            NvtxRange nv("evaluate");
-            for (u64 q0 = 0; q0 < claims_total; q0 += claims_per_launch) {
-                const u64 q1 = std::min(claims_total, q0 + claims_per_launch);
-                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
-                pp.claims_begin = q0;
-                pp.claims_end = q1;
-                pp.list_in = nullptr;
-                pp.list_n = nullptr;
-                pp.list_out = nullptr;
-                pp.list_cnt = nullptr;
-                pp.horizon = 0;
-                if (compact) {
-                    CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
-                    pp.list_out = ctx->dList.p;
-                    pp.list_cnt = ctx->dListCnt.p;
-                    pp.list_base = ub + (q0 / kChunkUnits * (u64)n_shards + (u64)shard) * kChunkUnits;
-                    pp.list_in_cap = claims_per_launch;
-                    pp.horizon = horizon;
+                pp.list_in_cap = list_cap;
+                BoundParamsHost bp;
+                memset(&bp, 0, sizeof bp);
+                bp.tabNI = ctx->dNI.p;
+                bp.tabW = ctx->dW.p;
+                bp.tabT = ctx->dT.p;
+                bp.tabU = ctx->dU.p;
+                bp.scal = ctx->dScal.p;
+                bp.inc = ctx->dInc.p;
+                bp.cost_prune = pp.cost_prune;
+                bp.off = ctx->dOff.p;
+                bp.counter = ctx->dCounter.p;
+                bp.stats = ctx->dStats.p;
+                bp.list_out = ctx->dList.p;
+                bp.list_cnt = ctx->dListCnt.p;
+                bp.list_cap = list_cap;
+                bp.overflow = (unsigned *)ctx->dErr.p;            // bit 2 (value 4): list overflow
+                bp.cands_per_prefix = S;
+                bp.cand_begin = cb;
+                bp.cand_end = ce;
+                bp.n_steps = n_steps;
+                bp.n_off = n_off;
+                bp.sumM = kernel_rows(ctx, a);
+                bp.sla = (int)a->sla_us;
+                bp.zero = 0;
+                bp.shard = shard;
+                bp.n_shards = n_shards;
+                bp.attr_shard = 0;
+                bp.attr_n = 1;
+                for (int k = 0; k < ctx->N; ++k) {
+                    int m = ctx->I[ctx->row0[k]];
+                    for (int c = 1; c < ctx->M[k]; ++c) m = std::min(m, ctx->I[ctx->row0[k] + c]);
+                    bp.nimin[k] = -m;
                 }
-                void *args[] = {&pp};
-                CUresult r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
-                                                   (CUstream)st, args, nullptr);
-                if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
-                ++launches;
-                if (compact) {                                    // pass 2 over the survivors
+                for (int k = 0; k < a->n_fixed; ++k) bp.fixed[k] = a->fixed_digits[k];
+                const int grid_b = jk->blocks_bound * ctx->n_sms;
+                if (first) CK(cudaEventRecord(ctx->ev[1], st), "event");
+                // evaluator over the deep survivors in dList (absolute depth-D prefix ids)
+                auto run_eval = [&]() -> int {
                     CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
                     pp.claims_begin = 0;
                     pp.claims_end = ~0ull;
                     pp.list_in = ctx->dList.p;
                     pp.list_n = ctx->dListCnt.p;
+                    pp.list_upp = upp;
+                    pp.list_base = 0;
                     pp.list_out = nullptr;
                     pp.list_cnt = nullptr;
                     pp.horizon = 0;
-                    r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
-                                              (CUstream)st, args, nullptr);
+                    void *args[] = {&pp};
+                    CUresult r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
+                                                       (CUstream)st, args, nullptr);
                     if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
                     ++launches;
+                    return SMILESS_OK;
+                };
+                auto run_bound = [&](CUfunction fn) -> int {
+                    void *bargs[] = {&bp};
+                    CUresult r = driver().launchKernel(fn, (unsigned)grid_b, 1, 1, kThreads, 1, 1,
+                                                       (unsigned)jk->smem_bound, (CUstream)st, bargs, nullptr);
+                    if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "bound launch");
+                    ++launches;
+                    return SMILESS_OK;
+                };
+                if (DA > 0) {
+                    // ---- two levels: depth DA over every prefix, depth D over the DA survivors' children --
+                    const u64 SA = cands_per_prefix(ctx, a, DA);
+                    const u64 a_lo = cb / SA, a_hi = (ce + SA - 1) / SA;
+                    CK(ctx->dListA.ensure((size_t)batch), "cudaMalloc list");
+                    CK(ctx->dListCntA.ensure(1), "cudaMalloc");
+                    // best-first: with the cost bound on, the shallow survivors are sorted by their
+                    // static cost lower bound so the first deep launch sets a good incumbent early
+                    // (SMILESS_BB_SORT=1; off by default: measured slower on C2 with live windows and
+                    // no faster elsewhere, profiles/r02k_bb_sort.md)
+                    const char *sort_env = getenv("SMILESS_BB_SORT");
+                    const bool bb_sort = pp.cost_prune && sort_env && atoi(sort_env) != 0;
+                    if (bb_sort) CK(ctx->dListKeyA.ensure((size_t)batch), "cudaMalloc keys");
+                    std::vector<u64> h_pref, h_key;
+                    std::vector<uint32_t> h_ord;
+                    for (u64 b0 = a_lo; b0 < a_hi; b0 += batch) {
+                        const u64 b1 = std::min(a_hi, b0 + batch);
+                        CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                        CK(cudaMemsetAsync(ctx->dListCntA.p, 0, sizeof(unsigned), st), "memset list");
+                        bp.list_in = nullptr;
+                        bp.list_n = nullptr;
+                        bp.list_upp = 1;
+                        bp.list_stride = 1;
+                        bp.list_r0 = 0;
+                        bp.prefix_begin = b0;
+                        bp.prefix_end = b1;
+                        bp.cands_per_prefix = SA;
+                        bp.list_out = ctx->dListA.p;
+                        bp.list_cnt = ctx->dListCntA.p;
+                        bp.list_cap = batch;
+                        bp.shard = 0;                                 // replicated on every shard ...
+                        bp.n_shards = 1;
+                        bp.attr_shard = shard;                        // ... its pruned prefixes counted once
+                        bp.attr_n = n_shards;
+                        bp.list_key = bb_sort ? ctx->dListKeyA.p : nullptr;
+                        {
+                            NvtxRange nv("bnb shallow level");
+                            if ((rc = run_bound(jk->fn_bound_a))) return rc;
+                        }
+                        unsigned n_a = 0;
+                        hp.mark("launch_a");
+                        CK(cudaMemcpyAsync(&n_a, ctx->dListCntA.p, sizeof n_a, cudaMemcpyDeviceToHost, st), "D2H count");
+                        ctx->d2h += sizeof n_a;
+                        CK(cudaStreamSynchronize(st), "count");
+                        hp.mark("sync_a");
+                        hp.note("n_a", n_a);
+                        bp.list_key = nullptr;
+                        if (bb_sort && n_a > 1 && n_a <= (1u << 18)) {
+                            // (key, prefix) ascending; ties by prefix: a deterministic order on every rank
+                            h_pref.resize(n_a);
+                            h_key.resize(n_a);
+                            CK(cudaMemcpyAsync(h_pref.data(), ctx->dListA.p, n_a * sizeof(u64), cudaMemcpyDeviceToHost, st),
+                               "D2H survivors");
+                            CK(cudaMemcpyAsync(h_key.data(), ctx->dListKeyA.p, n_a * sizeof(u64), cudaMemcpyDeviceToHost, st),
+                               "D2H keys");
+                            CK(cudaStreamSynchronize(st), "survivors");
+                            h_ord.resize(n_a);
+                            for (uint32_t q = 0; q < n_a; ++q) h_ord[q] = q;
+                            std::sort(h_ord.begin(), h_ord.end(), [&](uint32_t x, uint32_t y) {
+                                return h_key[x] != h_key[y] ? h_key[x] < h_key[y] : h_pref[x] < h_pref[y];
+                            });
+                            std::vector<u64> sorted(n_a);
+                            for (uint32_t q = 0; q < n_a; ++q) sorted[q] = h_pref[h_ord[q]];
+                            CK(cudaMemcpyAsync(ctx->dListA.p, sorted.data(), n_a * sizeof(u64), cudaMemcpyHostToDevice, st),
+                               "H2D survivors");
+                            ctx->d2h += 2 * (u64)n_a * sizeof(u64);
+                            ctx->h2d += (u64)n_a * sizeof(u64);
+                            hp.mark("sort_a");
+                        }
+                        // Launches over a survivor list (first entry, entries, first child, children per
+                        // entry): at most list_cap ordinals each.  With the cost bound on, the first launch
+                        // is small and each next one SMILESS_BB_GROW (256) times larger: every launch's
+                        // static prefix bound prunes against the incumbent the evaluations before it set,
+                        // so the incumbent is refined before the bulk of the list (C2 at SLA 8 s:
+                        // 131,072-entry chunks right after the 64-entry first one took 95-406 ms depending
+                        // on which survivors came first, 113-137 ms with a 16,384-entry step between;
+                        // profiles/r02p_bb_grow.md).  A survivor with more than list_cap children spans
+                        // several.
+                        struct DeepLaunch { u64 e0; unsigned ne; u64 r0, span; };
+                        auto make_chunks = [&](u64 n_entries, u64 Rc) {
+                            std::vector<DeepLaunch> L;
+                            if (Rc <= list_cap) {
+                                const u64 per_chunk = list_cap / Rc;
+                                const char *first_env = getenv("SMILESS_BB_FIRST");
+                                const u64 first = std::max<u64>(
+                                    1, std::min<u64>(per_chunk,
+                                                     pp.cost_prune ? (first_env ? (u64)atoll(first_env) : 64) : per_chunk));
+                                const char *grow_env = getenv("SMILESS_BB_GROW");
+                                const u64 grow = std::max<u64>(1, grow_env ? (u64)atoll(grow_env) : 256);
+                                u64 cur = first;
+                                for (u64 c0 = 0; c0 < n_entries;) {
+                                    const u64 len = std::min<u64>(cur, n_entries - c0);
+                                    L.push_back({c0, (unsigned)len, 0, Rc});
+                                    c0 += len;
+                                    cur = std::min<u64>(per_chunk, cur * grow);
+                                }
+                            } else {
+                                for (u64 e = 0; e < n_entries; ++e)
+                                    for (u64 r0 = 0; r0 < Rc; r0 += list_cap)
+                                        L.push_back({e, 1u, r0, std::min(list_cap, Rc - r0)});
+                            }
+                            return L;
+                        };
+                        auto upload_counts = [&](const std::vector<DeepLaunch> &L, DevBuf<unsigned> &buf) -> int {
+                            std::vector<unsigned> cnts(std::max<size_t>(L.size(), 1), 0u);
+                            for (size_t i = 0; i < L.size(); ++i) cnts[i] = L[i].ne;
+                            CK(buf.ensure(cnts.size()), "cudaMalloc counts");
+                            ctx->h2d += cnts.size() * sizeof(unsigned);
+                            CK(cudaMemcpyAsync(buf.p, cnts.data(), cnts.size() * sizeof(unsigned), cudaMemcpyHostToDevice, st),
+                               "H2D counts");
+                            return SMILESS_OK;
+                        };
+                        // one level over the children of a survivor list: bound kernel `fn` at depth with
+                        // `Sc` candidates per prefix writes its survivors to out / out_cnt; then `after`
+                        auto run_level = [&](CUfunction fn, const u64 *list, const std::vector<DeepLaunch> &L,
+                                             DevBuf<unsigned> &cnt_buf, u64 Rc, u64 Sc, u64 *out, unsigned *out_cnt,
+                                             int shard_, int n_shards_, const std::function<int(size_t)> &after) -> int {
+                            for (size_t i = 0; i < L.size(); ++i) {
+                                CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                                CK(cudaMemsetAsync(out_cnt, 0, sizeof(unsigned), st), "memset list");
+                                bp.list_in = list + L[i].e0;
+                                bp.list_n = cnt_buf.p + i;
+                                bp.list_upp = L[i].span;
+                                bp.list_stride = Rc;
+                                bp.list_r0 = L[i].r0;
+                                bp.prefix_begin = 0;
+                                bp.prefix_end = 0;
+                                bp.cands_per_prefix = Sc;
+                                bp.list_out = out;
+                                bp.list_cnt = out_cnt;
+                                bp.list_cap = list_cap;
+                                bp.shard = shard_;
+                                bp.n_shards = n_shards_;
+                                bp.attr_shard = 0;
+                                bp.attr_n = 1;
+                                if ((rc = run_bound(fn))) return rc;
+                                if ((rc = after(i))) return rc;
+                            }
+                            return SMILESS_OK;
+                        };
+                        const int DM = jk->fn_bound_m ? bb_depth_m(ctx, a, D, DA) : 0;
+                        if (DM == 0) {
+                            // two levels: the deep children of the shallow survivors, interleaved over shards
+                            const std::vector<DeepLaunch> L = make_chunks(n_a, R);
+                            if ((rc = upload_counts(L, ctx->dChunkCnt))) return rc;
+                            NvtxRange nv("bnb deep level + evaluate");
+                            if ((rc = run_level(jk->fn_bound, ctx->dListA.p, L, ctx->dChunkCnt, R, S, ctx->dList.p,
+                                                ctx->dListCnt.p, shard, n_shards, [&](size_t) { return run_eval(); })))
+                                return rc;
+                        } else {
+                            // three levels: the middle children of the shallow survivors (interleaved over
+                            // shards), then the deep children of each middle launch's survivors (this
+                            // rank's own, not split again) and the evaluator over those
+                            const u64 SMd = cands_per_prefix(ctx, a, DM);
+                            const u64 R1 = SA / SMd, R2 = SMd / S;
+                            CK(ctx->dListM.ensure((size_t)list_cap), "cudaMalloc list");
+                            CK(ctx->dListCntM.ensure(1), "cudaMalloc");
+                            const std::vector<DeepLaunch> Lm = make_chunks(n_a, R1);
+                            if ((rc = upload_counts(Lm, ctx->dChunkCntM))) return rc;
+                            NvtxRange nv("bnb middle + deep level + evaluate");
+                            auto deep = [&](size_t) -> int {
+                                unsigned n_m = 0;
+                                CK(cudaMemcpyAsync(&n_m, ctx->dListCntM.p, sizeof n_m, cudaMemcpyDeviceToHost, st), "D2H count");
+                                ctx->d2h += sizeof n_m;
+                                CK(cudaStreamSynchronize(st), "count");
+                                hp.note("n_m", n_m);
+                                if (n_m == 0) return SMILESS_OK;
+                                const std::vector<DeepLaunch> L = make_chunks(n_m, R2);
+                                if ((rc = upload_counts(L, ctx->dChunkCnt))) return rc;
+                                return run_level(jk->fn_bound, ctx->dListM.p, L, ctx->dChunkCnt, R2, S, ctx->dList.p,
+                                                 ctx->dListCnt.p, 0, 1, [&](size_t) { return run_eval(); });
+                            };
+                            if ((rc = run_level(jk->fn_bound_m, ctx->dListA.p, Lm, ctx->dChunkCntM, R1, SMd, ctx->dListM.p,
+                                                ctx->dListCntM.p, shard, n_shards, deep)))
+                                return rc;
+                        }
+                        hp.mark("chunks_launched");
+                        CK(cudaStreamSynchronize(st), "chunks");      // the next batch reuses dListA
+                        hp.mark("sync_chunks");
+                    }
+                } else {
+                    NvtxRange nv("bnb level + evaluate");
+                    const u64 rbatch = std::min(batch, list_cap);     // a launch's survivors fit the list
+                    for (u64 b0 = p_lo; b0 < p_hi; b0 += rbatch) {
+                        const u64 b1 = std::min(p_hi, b0 + rbatch);
+                        CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                        CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
+                        bp.list_in = nullptr;
+                        bp.list_n = nullptr;
+                        bp.list_upp = 1;
+                        bp.list_stride = 1;
+                        bp.list_r0 = 0;
+                        bp.prefix_begin = b0;
+                        bp.prefix_end = b1;
+                        if ((rc = run_bound(jk->fn_bound))) return rc;
+                        if ((rc = run_eval())) return rc;
+                    }
+                }
+            } else {
+                eval_path = SMILESS_PATH_PLAN;
+                // split very large ranges into several launches (bounded kernel duration).  Prune mode
+                // with J - 1 > horizon runs each batch twice: pass 1 (every unit, `horizon` steps,
+                // survivors compacted into a list), pass 2 (survivors only, all steps).
+                const char *hz_env = getenv("SMILESS_HORIZON");
+                i64 horizon = hz_env ? atoll(hz_env) : 128;
+                horizon = horizon / rp.K * rp.K;
+                const bool compact = pp.prune && horizon > 0 && horizon < n_steps;
+                const u64 claims_per_launch = compact ? ((u64)1 << 24) : ((u64)1 << 28);   // units
+                if (compact) {
+                    CK(ctx->dList.ensure((size_t)claims_per_launch), "cudaMalloc list");
+                    CK(ctx->dListCnt.ensure(1), "cudaMalloc");
+                }
+                if (first) CK(cudaEventRecord(ctx->ev[1], st), "event");
+                NvtxRange nv("evaluate");
+                for (u64 q0 = 0; q0 < claims_total; q0 += claims_per_launch) {
+                    const u64 q1 = std::min(claims_total, q0 + claims_per_launch);
+                    CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                    pp.claims_begin = q0;
+                    pp.claims_end = q1;
+                    pp.list_in = nullptr;
+                    pp.list_n = nullptr;
+                    pp.list_out = nullptr;
+                    pp.list_cnt = nullptr;
+                    pp.horizon = 0;
+                    if (compact) {
+                        CK(cudaMemsetAsync(ctx->dListCnt.p, 0, sizeof(unsigned), st), "memset list");
+                        pp.list_out = ctx->dList.p;
+                        pp.list_cnt = ctx->dListCnt.p;
+                        pp.list_base = ub + (q0 / kChunkUnits * (u64)n_shards + (u64)shard) * kChunkUnits;
+                        pp.list_in_cap = claims_per_launch;
+                        pp.horizon = horizon;
+                    }
+                    void *args[] = {&pp};
+                    CUresult r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
+                                                       (CUstream)st, args, nullptr);
+                    if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
+                    ++launches;
+                    if (compact) {                                    // pass 2 over the survivors
+                        CK(cudaMemsetAsync(ctx->dCounter.p, 0, 8, st), "memset counter");
+                        pp.claims_begin = 0;
+                        pp.claims_end = ~0ull;
+                        pp.list_in = ctx->dList.p;
+                        pp.list_n = ctx->dListCnt.p;
+                        pp.list_out = nullptr;
+                        pp.list_cnt = nullptr;
+                        pp.horizon = 0;
+                        r = driver().launchKernel(jk->fn, (unsigned)grid, 1, 1, kThreads, 1, 1, (unsigned)jk->smem,
+                                                  (CUstream)st, args, nullptr);
+                        if (r != CUDA_SUCCESS) return drv_fail(ctx, r, "evaluator launch");
+                        ++launches;
+                    }
                 }
             }
-        }
-        NvtxRange nv("argmin reduce");
-        for (int s_ = 0; s_ < n_sla; ++s_) {
-            int e2 = smiless_dev_reduce_best(ctx->dBlk.p + 2 * s_, grid_used, n_sla, dst + s_, st);
-            if (e2) return cuda_fail(ctx, (cudaError_t)e2, "reduce launch");
-            ++launches;
-        }
-        CK(cudaMemcpyAsync(&dst->stats[0], ctx->dStats.p, 16, cudaMemcpyDeviceToDevice, st), "D2D stats");
-        if (a->cost_out) {
-            ctx->d2h += (size_t)(ce - cb) * sizeof(double);
-            CK(cudaMemcpyAsync(a->cost_out, ctx->dDump.p, (size_t)(ce - cb) * sizeof(double), cudaMemcpyDeviceToHost, st),
-               "D2H dump");
-        }
-        return SMILESS_OK;
+            NvtxRange nv("argmin reduce");
+            for (int s_ = 0; s_ < n_sla; ++s_) {
+                int e2 = smiless_dev_reduce_best(ctx->dBlk.p + 2 * s_, grid_used, n_sla, dst + s_, st);
+                if (e2) return cuda_fail(ctx, (cudaError_t)e2, "reduce launch");
+                ++launches;
+            }
+            CK(cudaMemcpyAsync(&dst->stats[0], ctx->dStats.p, 16, cudaMemcpyDeviceToDevice, st), "D2D stats");
+            if (a->cost_out) {
+                ctx->d2h += (size_t)(ce - cb) * sizeof(double);
+                CK(cudaMemcpyAsync(a->cost_out, ctx->dDump.p, (size_t)(ce - cb) * sizeof(double), cudaMemcpyDeviceToHost, st),
+                   "D2H dump");
+            }
+            return SMILESS_OK;
         };
         if (!digit_mode) {
             if ((rc = run_once(ctx->dRes.p, true))) return rc;
